@@ -1,0 +1,31 @@
+# Build libgsw.so (CUDA, sm_100a) + the C generator and oracle libraries (CPU).
+NVCC ?= nvcc
+PKG := paper_conf_ppopp_menglts19_b200
+CSRC := $(PKG)/csrc
+CU := $(wildcard $(CSRC)/*.cu)
+HDR := $(wildcard $(CSRC)/*.cuh $(CSRC)/*.h) include/gsw.h
+NVFLAGS := -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 \
+           -Xcompiler -fPIC -Iinclude -I$(CSRC) --expt-relaxed-constexpr -Xptxas -v
+LIB := $(PKG)/libgsw.so
+OBJDIR := build/obj
+OBJ := $(patsubst $(CSRC)/%.cu,$(OBJDIR)/%.o,$(CU))
+
+all: $(LIB) gen/libgswgen.so oracle/liboracle.so
+
+$(OBJDIR)/%.o: $(CSRC)/%.cu $(HDR)
+	@mkdir -p $(OBJDIR)
+	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> $(OBJDIR)/$*.ptxas.txt || (cat $(OBJDIR)/$*.ptxas.txt; exit 1)
+
+$(LIB): $(OBJ)
+	$(NVCC) -gencode arch=compute_100a,code=sm_100a -shared -o $@ $(OBJ) -lcudart
+
+gen/libgswgen.so: gen/gen.c
+	gcc -O3 -fopenmp -fPIC -shared -o $@ $< -lm
+
+oracle/liboracle.so: oracle/oracle.c
+	gcc -O2 -fPIC -shared -o $@ $< -lm
+
+clean:
+	rm -rf build $(LIB) gen/libgswgen.so oracle/liboracle.so
+
+.PHONY: all clean

@@ -1,0 +1,168 @@
+/*
+ * gsw.h -- C ABI of the B200-native GSWITCH frontier-step library (libgsw.so).
+ *
+ * What it computes.  GSWITCH standardises a BSP graph algorithm as a two-phase per-iteration
+ * process: "The filtering step (Filter) generates the active set and updates their private data;
+ * then the expansion step (Expand) processes all the neighbors of the generated active set"
+ * (Sec. 2.1).  An algorithm "terminates with no more active elements"
+ * (P:251-252).  Every iteration the library extracts runtime features (Table 1), runs
+ * a decision-tree selector over the five patterns in the order direction -> load balance ->
+ * active-set format -> stepping -> fusion and executes the selected Filter/Expand
+ * variant.  All of this runs on the device inside one persistent kernel per run;
+ * the host is crossed only at entry and at the final synchronisation.
+ *
+ * Conventions (all functions):
+ *   - Vertex ids are int32 in [0, n).  n < 2^31, nnz < 2^32 (else GSW_EOVERFLOW).
+ *   - Array arguments may be HOST or DEVICE pointers: the library classifies every pointer with
+ *     cudaPointerGetAttributes and copies host data in / results out on the handle's stream.
+ *   - Every call is synchronous: it returns after its work on the handle's stream completed, so
+ *     outputs and stats are valid on return.
+ *   - The library never aborts.  A non-OK status leaves a message in gsw_last_error() (thread
+ *     local).  CUDA errors map to GSW_ECUDA, NCCL errors to GSW_ENCCL.
+ *   - A handle is not thread-safe: one call at a time per handle.  Separate handles on separate
+ *     streams are independent.
+ *   - Memory: the library allocates no device memory of its own.  The caller queries
+ *     gsw_workspace_size(), allocates one device buffer (e.g. a torch uint8 tensor) and passes it
+ *     to gsw_graph_create(); the graph copy and all per-run scratch live in it.  The caller keeps
+ *     it alive until gsw_graph_destroy().
+ */
+#ifndef GSW_H
+#define GSW_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    GSW_OK = 0,
+    GSW_EINVAL = 1,          /* bad argument (null pointer, source out of range, bad CSR ...)   */
+    GSW_ENOMEM = 2,          /* workspace too small                                             */
+    GSW_ECUDA = 3,           /* a CUDA runtime/driver call or kernel failed                     */
+    GSW_ENCCL = 4,           /* an NCCL call failed                                             */
+    GSW_EUNSUPPORTED = 5,    /* forced configuration not valid for this algorithm               */
+    GSW_EOVERFLOW = 6        /* sizes or path lengths exceed the 32-bit internal representation */
+} gsw_status;
+
+typedef struct gsw_graph_s *gsw_graph;
+
+/* CSR (out-edges) or CSC (in-edges).  Caller-owned; copied by gsw_graph_create. */
+typedef struct {
+    int64_t n;                    /* vertices                                                  */
+    int64_t nnz;                  /* directed entries (= 2x undirected edges for symmetric)    */
+    const int64_t *row_offsets;   /* n+1, non-decreasing, row_offsets[0]=0, [n]=nnz            */
+    const int32_t *col_indices;   /* nnz, each in [0,n)                                        */
+    const uint32_t *weights;      /* nnz or NULL; required by gsw_sssp                         */
+} gsw_csr;
+
+/* ---- pattern candidates (Sec. 3).  0 = AUTO (selector decides each iteration) ---- */
+enum { GSW_AUTO = 0 };
+/* Pattern 1, direction */
+enum { GSW_PUSH = 1, GSW_PULL = 2 };
+/* Pattern 2, active-set format */
+enum { GSW_BITMAP = 1, GSW_QUEUE = 2, GSW_SORTED_QUEUE = 3 };
+/* Pattern 3, load balance; THREAD = naive one-thread-per-vertex (north_star) */
+enum { GSW_LB_THREAD = 1, GSW_LB_TWC = 2, GSW_LB_WM = 3, GSW_LB_CM = 4, GSW_LB_STRICT = 5 };
+/* Pattern 4, stepping: SSSP priority threshold control.
+ *   INCREASE/DECREASE/REMAIN pin the per-iteration decision of the dynamic controller;
+ *   STATIC = classic delta-stepping with fixed delta0 (theta += delta0 when the near set empties);
+ *   UNORDERED = Bellman-Ford (theta = infinity).                                                  */
+enum { GSW_STEP_INCREASE = 1, GSW_STEP_DECREASE = 2, GSW_STEP_REMAIN = 3,
+       GSW_STEP_STATIC = 4, GSW_STEP_UNORDERED = 5 };
+/* Pattern 5, kernel fusion */
+enum { GSW_STANDALONE = 1, GSW_FUSED = 2 };
+
+typedef struct {
+    int32_t direction;      /* AUTO | GSW_PUSH | GSW_PULL                                     */
+    int32_t format;         /* AUTO | GSW_BITMAP | GSW_QUEUE | GSW_SORTED_QUEUE               */
+    int32_t load_balance;   /* AUTO | GSW_LB_*                                                */
+    int32_t stepping;       /* AUTO | GSW_STEP_*  (ignored by all algorithms but SSSP)        */
+    int32_t fusion;         /* AUTO | GSW_STANDALONE | GSW_FUSED                              */
+    uint32_t delta0;        /* SSSP threshold step; 0 = c*wbar/dbar with c=32     */
+} gsw_config;
+
+/* One record per iteration (the paper's per-iteration feedback). */
+typedef struct {
+    int32_t iteration;
+    int32_t direction, format, load_balance, stepping, fusion;   /* the executed variant     */
+    int64_t Va, Ea, Via, Eia;     /* runtime characteristics of the active set (Table 1)       */
+    int64_t edges;                /* adjacency entries read by this iteration's Expand          */
+    uint32_t theta;               /* SSSP priority threshold in force (0 for other algorithms) */
+    float filter_us, expand_us;   /* device time of the Filter and Expand phases (%globaltimer)*/
+} gsw_iter_record;
+
+typedef struct {
+    int32_t iterations;           /* BSP iterations executed (summed over sources for BC)      */
+    float gpu_ms;                 /* device time of the run, CUDA events on the handle stream  */
+    int64_t edges_touched;        /* adjacency entries read by Expand (summed over iterations)  */
+    int64_t bytes_alg;            /* algorithmic HBM bytes (roofline model D0)      */
+    gsw_iter_record *records;     /* optional HOST buffer of max_records entries, or NULL      */
+    int32_t max_records;          /* records beyond this many are counted but not stored        */
+} gsw_run_stats;
+
+/* Bytes of device workspace gsw_graph_create needs for a graph of this size. */
+gsw_status gsw_workspace_size(int64_t n, int64_t nnz, int32_t has_weights, int32_t has_csc,
+                              size_t *bytes);
+
+/*
+ * Copy a CSR (and optionally a separate CSC for directed graphs; NULL = symmetric, the CSC is the
+ * CSR -- all paper inputs are undirected) into the workspace, converting offsets to u32,
+ * and compute the dataset attributes of Table 1 (N, M, dbar, sigma_d, r_d, Gini, H_er, P:752-759,
+ * "computed only once while loading the data").
+ *   workspace: DEVICE buffer of >= gsw_workspace_size() bytes, 256-byte aligned.
+ *   cuda_stream: cudaStream_t (NULL = legacy default stream) used by every call on the handle.
+ * Errors: GSW_EINVAL (nulls, n<=0, nnz mismatch), GSW_ENOMEM (workspace too small),
+ *         GSW_EOVERFLOW (n >= 2^31 or nnz >= 2^32).  The CSR contents are not validated beyond
+ *         offsets[0]==0 and offsets[n]==nnz (use gsw_graph_validate).
+ */
+gsw_status gsw_graph_create(const gsw_csr *csr, const gsw_csr *csc, void *workspace,
+                            size_t ws_bytes, void *cuda_stream, gsw_graph *out);
+gsw_status gsw_graph_destroy(gsw_graph g);
+/* Full device-side check: monotone offsets and every column in range (GSW_EINVAL otherwise). */
+gsw_status gsw_graph_validate(gsw_graph g);
+
+/* Dataset attributes of Table 1, out[0..6] = N, M, dbar, sigma_d, r_d, Gini, H_er. */
+gsw_status gsw_graph_attributes(gsw_graph g, double out[7]);
+
+/*
+ * Pin pattern choices for every iteration of later runs on this handle (NULL = full autotune).
+ * Each non-AUTO field overrides the selector.  Unsupported combinations return
+ * GSW_EUNSUPPORTED at run time:
+ *   - PR: fusion is ignored (every vertex is active every iteration);
+ *   - BC backward sweep always pulls; forcing applies to the forward (sigma) phase.
+ */
+gsw_status gsw_force_config(gsw_graph g, const gsw_config *cfg);
+
+/* BFS from `source` (Fig. 11).  depth[v] = hop distance, depth[source]=0,
+ * -1 if unreachable.  depth: n int32, host or device.                                        */
+gsw_status gsw_bfs(gsw_graph g, int32_t source, int32_t *depth, gsw_run_stats *stats);
+
+/* SSSP with dynamic stepping (footnote 2 P:411-413).  Requires weights.
+ * dist[v] = shortest-path length (uint32), UINT32_MAX if unreachable.  GSW_EOVERFLOW if
+ * max_w * (n-1) >= 2^32-1.                                                                    */
+gsw_status gsw_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *stats);
+
+/* Connected components: label[v] = min vertex id of v's component.               */
+gsw_status gsw_cc(gsw_graph g, int32_t *label, gsw_run_stats *stats);
+
+/* PageRank power iteration: pr_0 = 1/N, exactly `iters` iterations of
+ *   pr'(v) = (1-d)/N + d * (sum_{u->v} pr(u)/deg_out(u) + D/N),  D = sum of dangling pr.
+ * rank: n doubles, host or device.                                                            */
+gsw_status gsw_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *stats);
+
+/* Betweenness centrality (Brandes): bc[v] = sum_{s in sources, s != v} delta_s(v),
+ * unnormalised.  sources: nsrc int32 on the HOST.  bc: n doubles, host or device.              */
+gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc,
+                  gsw_run_stats *stats);
+
+/* Thread-local message for the last non-OK status of this thread. */
+const char *gsw_last_error(void);
+/* Library version string. */
+const char *gsw_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GSW_H */

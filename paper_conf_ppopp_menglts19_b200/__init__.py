@@ -1,0 +1,194 @@
+"""B200-native GSWITCH frontier-step library: thin Python binding over the C ABI (include/gsw.h).
+
+Every step of the hot path (ingest, features, selector, Filter, Expand) runs in the CUDA kernels
+of ``libgsw.so``; this module only marshals arguments.  PyTorch provides device memory (the
+workspace and output tensors) and the CUDA stream.  There is no CPU fallback.
+
+    g = Graph(row_offsets, col_indices, weights=None)     # numpy / torch (host or device)
+    depth, stats = g.bfs(src)                             # torch int32 on the graph's device
+    g.force_config(direction="pull", load_balance="twc")  # pin patterns (gsw_force_config)
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Optional, Sequence
+
+import numpy as np
+
+from . import _lib
+from ._lib import (AUTO, BITMAP, DIRECTIONS, FORMATS, FUSED, FUSIONS, LB_CM, LB_STRICT,  # noqa: F401
+                   LB_THREAD, LB_TWC, LB_WM, LOAD_BALANCES, PULL, PUSH, QUEUE, SORTED_QUEUE, STANDALONE,
+                   STEPPINGS, GswError, check)
+
+__all__ = ["Graph", "GswError", "version", "force_config_struct"]
+
+
+def version() -> str:
+    return _lib.load().gsw_version().decode()
+
+
+def _ptr_of(a):
+    """(pointer, keepalive, is_device) for a numpy array or torch tensor (contiguous)."""
+    import torch
+    if isinstance(a, torch.Tensor):
+        a = a.contiguous()
+        return a.data_ptr(), a, a.is_cuda
+    a = np.ascontiguousarray(a)
+    return a.ctypes.data, a, False
+
+
+def _as(a, np_dtype, torch_dtype):
+    import torch
+    if isinstance(a, torch.Tensor):
+        return a.to(torch_dtype).contiguous()
+    return np.ascontiguousarray(np.asarray(a, dtype=np_dtype))
+
+
+def force_config_struct(direction=AUTO, format=AUTO, load_balance=AUTO, stepping=AUTO, fusion=AUTO,
+                        delta0=0) -> _lib.gsw_config:
+    def enc(v, table):
+        if isinstance(v, str):
+            return table[v.lower()]
+        return int(v)
+    return _lib.gsw_config(enc(direction, DIRECTIONS), enc(format, FORMATS),
+                           enc(load_balance, LOAD_BALANCES), enc(stepping, STEPPINGS),
+                           enc(fusion, FUSIONS), int(delta0))
+
+
+def _stats_dict(st: _lib.gsw_run_stats, recs) -> dict:
+    d = {"iterations": st.iterations, "gpu_ms": st.gpu_ms, "edges_touched": st.edges_touched,
+         "bytes_alg": st.bytes_alg}
+    if recs is not None:
+        n = min(st.iterations, len(recs))
+        d["records"] = [{k: getattr(recs[i], k) for k, _ in _lib.gsw_iter_record._fields_} for i in range(n)]
+    return d
+
+
+class Graph:
+    """A graph resident in one device workspace (gsw_graph_create)."""
+
+    def __init__(self, row_offsets, col_indices, weights=None, csc: Optional[tuple] = None,
+                 device: str | int = "cuda", stream=None):
+        import torch
+        lib = _lib.load()
+        self.device = torch.device(device)
+        if self.device.type != "cuda":
+            raise ValueError("gsw graphs live on a CUDA device")
+        off = _as(row_offsets, np.int64, torch.int64)
+        col = _as(col_indices, np.int32, torch.int32)
+        w = None if weights is None else _as(weights, np.uint32, torch.int32)
+        self.n = int(off.shape[0]) - 1
+        self.nnz = int(col.shape[0])
+        self.weighted = w is not None
+        with torch.cuda.device(self.device):
+            self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+            keep = []
+
+            def mk(o, c, ww):
+                po, ko, _ = _ptr_of(o)
+                pc, kc, _ = _ptr_of(c) if self.nnz else (None, None, False)
+                pw, kw, _ = _ptr_of(ww) if ww is not None else (None, None, False)
+                keep.extend([ko, kc, kw])
+                return _lib.gsw_csr(self.n, self.nnz, po, pc, pw)
+
+            csr = mk(off, col, w)
+            csc_s = None
+            if csc is not None:
+                coff = _as(csc[0], np.int64, torch.int64)
+                ccol = _as(csc[1], np.int32, torch.int32)
+                cw = None if len(csc) < 3 or csc[2] is None else _as(csc[2], np.uint32, torch.int32)
+                csc_s = mk(coff, ccol, cw)
+            nbytes = ctypes.c_size_t()
+            check(lib.gsw_workspace_size(self.n, self.nnz, int(self.weighted), int(csc is not None),
+                                         ctypes.byref(nbytes)), "gsw_workspace_size")
+            self.workspace = torch.empty(nbytes.value, dtype=torch.uint8, device=self.device)
+            h = ctypes.c_void_p()
+            check(lib.gsw_graph_create(ctypes.byref(csr), ctypes.byref(csc_s) if csc_s is not None else None,
+                                       self.workspace.data_ptr(), nbytes.value, self.stream.cuda_stream,
+                                       ctypes.byref(h)), "gsw_graph_create")
+            self._h = h
+            del keep
+
+    # -------------------------------------------------------------------------------------
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.load().gsw_graph_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def attributes(self) -> dict:
+        out = (ctypes.c_double * 7)()
+        check(_lib.load().gsw_graph_attributes(self._h, out), "gsw_graph_attributes")
+        return dict(zip(["N", "M", "dbar", "sigma_d", "r_d", "gini", "h_er"], list(out)))
+
+    def validate(self) -> None:
+        check(_lib.load().gsw_graph_validate(self._h), "gsw_graph_validate")
+
+    def force_config(self, **kw) -> None:
+        """Pin patterns: direction, format, load_balance, stepping, fusion, delta0 (None = AUTO)."""
+        lib = _lib.load()
+        if not kw or all(v in (None, 0, "auto") for v in kw.values()):
+            check(lib.gsw_force_config(self._h, None), "gsw_force_config")
+            return
+        cfg = force_config_struct(**{k: (AUTO if v in (None, "auto") else v) for k, v in kw.items()})
+        check(lib.gsw_force_config(self._h, ctypes.byref(cfg)), "gsw_force_config")
+
+    # -------------------------------------------------------------------------------------
+    def _stats(self, records: int):
+        st = _lib.gsw_run_stats()
+        recs = None
+        if records:
+            recs = (_lib.gsw_iter_record * records)()
+            st.records = ctypes.cast(recs, ctypes.POINTER(_lib.gsw_iter_record))
+            st.max_records = records
+        return st, recs
+
+    def _out(self, out, dtype):
+        import torch
+        if out is None:
+            return torch.empty(self.n, dtype=dtype, device=self.device)
+        return out
+
+    def bfs(self, source: int, out=None, records: int = 0):
+        """Depths from `source` (-1 = unreachable).  `out` may be a host (pinned) or device tensor."""
+        import torch
+        out = self._out(out, torch.int32)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_bfs(self._h, int(source), out.data_ptr(), ctypes.byref(st)), "gsw_bfs")
+        return out, _stats_dict(st, recs)
+
+    def sssp(self, source: int, out=None, records: int = 0):
+        """Shortest distances (uint32 values in an int32 tensor; 0xFFFFFFFF = unreachable)."""
+        import torch
+        out = self._out(out, torch.int32)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_sssp(self._h, int(source), out.data_ptr(), ctypes.byref(st)), "gsw_sssp")
+        return out, _stats_dict(st, recs)
+
+    def cc(self, out=None, records: int = 0):
+        import torch
+        out = self._out(out, torch.int32)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_cc(self._h, out.data_ptr(), ctypes.byref(st)), "gsw_cc")
+        return out, _stats_dict(st, recs)
+
+    def pr(self, damping: float = 0.85, iters: int = 20, out=None, records: int = 0):
+        import torch
+        out = self._out(out, torch.float64)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_pr(self._h, float(damping), int(iters), out.data_ptr(), ctypes.byref(st)), "gsw_pr")
+        return out, _stats_dict(st, recs)
+
+    def bc(self, sources: Sequence[int], out=None, records: int = 0):
+        import torch
+        out = self._out(out, torch.float64)
+        src = np.ascontiguousarray(np.asarray(list(sources), dtype=np.int32))
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_bc(self._h, src.ctypes.data if src.size else None, int(src.size), out.data_ptr(),
+                                 ctypes.byref(st)), "gsw_bc")
+        return out, _stats_dict(st, recs)

@@ -1,0 +1,236 @@
+// common.cuh -- device building blocks shared by every algorithm of the library.
+//
+// The whole per-iteration loop of GSWITCH (Inspector -> Selector -> Executor, PAPER.md:805-844,
+// Fig. 10) runs inside ONE persistent cooperative kernel per run.  Phases of an iteration are
+// separated by a software grid barrier (below) instead of kernel boundaries, so there is no host
+// round trip per iteration (the paper's 58-120 us feature copy, disappears).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace gsw {
+
+constexpr int kBlock = 256;           // threads per CTA of every persistent kernel
+constexpr int kWarps = kBlock / 32;
+
+// ------------------------------------------------------------------ memory-order helpers
+__device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(unsigned *p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_relaxed(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed64(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ int ld_relaxed_s32(const int *p) {
+    int v;
+    asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// ------------------------------------------------------------------ grid barrier
+// Monotone arrival counter + generation word.  The last CTA to arrive for generation g sees
+// prev == g*gridDim - 1 and publishes g with a release store; the others spin with acquire
+// loads.  Co-residency of all CTAs is guaranteed by cudaLaunchCooperativeKernel.  A spin longer
+// than kBarrierTimeoutNs sets an error code and traps, so a bug becomes a launch failure rather
+// than a hung GPU.
+struct GridBarrier {
+    unsigned *arrive;
+    unsigned *gen;
+    unsigned *err;
+};
+constexpr uint64_t kBarrierTimeoutNs = 20ull * 1000 * 1000 * 1000;
+
+__device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned target = epoch + 1;
+        __threadfence();
+        unsigned prev = atomicAdd(b.arrive, 1u);
+        if (prev == target * gridDim.x - 1) {
+            __threadfence();
+            st_release(b.gen, target);
+        } else {
+            uint64_t t0 = globaltimer();
+            unsigned spins = 0;
+            while (ld_acquire(b.gen) < target) {
+                if (((++spins) & 1023u) == 0 && globaltimer() - t0 > kBarrierTimeoutNs) {
+                    atomicExch(b.err, 0xBA4u);
+                    __trap();
+                }
+            }
+        }
+        __threadfence();
+    }
+    epoch += 1;
+    __syncthreads();
+}
+
+// ------------------------------------------------------------------ warp / block reductions
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+template <typename T>
+__device__ __forceinline__ T warp_max(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) { T x = __shfl_xor_sync(0xffffffffu, v, o); v = x > v ? x : v; }
+    return v;
+}
+template <typename T>
+__device__ __forceinline__ T warp_min(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) { T x = __shfl_xor_sync(0xffffffffu, v, o); v = x < v ? x : v; }
+    return v;
+}
+// inclusive warp scan
+template <typename T>
+__device__ __forceinline__ T warp_incl_scan(T v) {
+    unsigned l = lane_id();
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        T x = __shfl_up_sync(0xffffffffu, v, o);
+        if (l >= (unsigned)o) v += x;
+    }
+    return v;
+}
+
+// Block-wide exclusive scan of one value per thread (kBlock threads).  Returns the exclusive
+// prefix; *total gets the block sum.  Uses `sm` (>= kWarps+1 entries).  Contains __syncthreads.
+template <typename T>
+__device__ __forceinline__ T block_excl_scan(T v, T *sm, T *total) {
+    T inc = warp_incl_scan(v);
+    unsigned w = threadIdx.x >> 5, l = lane_id();
+    __syncthreads();
+    if (l == 31) sm[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+        T s = l < (unsigned)kWarps ? sm[l] : T(0);
+        T si = warp_incl_scan(s);
+        if (l < (unsigned)kWarps) sm[l] = si - s;
+        if (l == kWarps - 1) sm[kWarps] = si;
+    }
+    __syncthreads();
+    T res = sm[w] + inc - v;
+    *total = sm[kWarps];
+    return res;
+}
+
+// Block-wide sum (all threads get the result).  Contains __syncthreads.
+template <typename T>
+__device__ __forceinline__ T block_sum(T v, T *sm) {
+    v = warp_sum(v);
+    unsigned w = threadIdx.x >> 5, l = lane_id();
+    __syncthreads();
+    if (l == 0) sm[w] = v;
+    __syncthreads();
+    T s = l < (unsigned)kWarps ? sm[l] : T(0);
+    s = warp_sum(s);
+    return s;
+}
+
+// ------------------------------------------------------------------ bitmaps
+__device__ __forceinline__ bool test_bit(const unsigned *bm, int v) {
+    return (bm[v >> 5] >> (v & 31)) & 1u;
+}
+__device__ __forceinline__ bool test_bit_relaxed(const unsigned *bm, int v) {
+    return (ld_relaxed(bm + (v >> 5)) >> (v & 31)) & 1u;
+}
+// atomic test-and-set; returns true if this call set the bit (0 -> 1 winner)
+__device__ __forceinline__ bool claim_bit(unsigned *bm, int v) {
+    unsigned bit = 1u << (v & 31);
+    unsigned old = atomicOr(bm + (v >> 5), bit);
+    return !(old & bit);
+}
+
+// ------------------------------------------------------------------ warp-aggregated append
+// Append `v` to q[*len] for every calling lane with pred true; one atomicAdd per warp.
+// Safe under divergence: aggregates over the currently converged lanes.
+__device__ __forceinline__ void warp_append(int *q, unsigned *len, bool pred, int v) {
+    unsigned active = __activemask();
+    unsigned m = __ballot_sync(active, pred);
+    if (m == 0) return;
+    int leader = __ffs(active) - 1;
+    unsigned base = 0;
+    if ((int)lane_id() == leader) base = atomicAdd(len, (unsigned)__popc(m));
+    base = __shfl_sync(active, base, leader);
+    if (pred) q[base + __popc(m & lanemask_lt())] = v;
+}
+
+// ------------------------------------------------------------------ per-iteration counters
+// Runtime characteristics of the NEXT active set, accumulated by whoever activates a vertex
+// (Table 1): Va, Ea, max/min degree; plus edges scanned by this iteration's Expand.
+struct IterCnt {
+    unsigned long long va, ea, edges;
+    unsigned maxd, mind;
+    unsigned qlen;          // length of the queue materialised for this active set (if any)
+    unsigned iqlen;         // length of the inactive (pull workload) queue, if built
+};
+
+struct LocalCnt {
+    unsigned long long va = 0, ea = 0, edges = 0;
+    unsigned maxd = 0, mind = 0xffffffffu;
+    __device__ __forceinline__ void add_vertex(unsigned deg) {
+        va += 1; ea += deg;
+        maxd = deg > maxd ? deg : maxd;
+        mind = deg < mind ? deg : mind;
+    }
+};
+
+// Reduce a thread's counters over the CTA and add them to the global slot (one atomic each per
+// CTA).  Must be called by all threads of the CTA.
+__device__ __forceinline__ void flush_counts(LocalCnt &c, IterCnt *dst) {
+    __shared__ unsigned long long s64[kWarps][3];
+    __shared__ unsigned s32[kWarps][2];
+    unsigned long long va = warp_sum(c.va), ea = warp_sum(c.ea), ed = warp_sum(c.edges);
+    unsigned mx = warp_max(c.maxd), mn = warp_min(c.mind);
+    unsigned w = threadIdx.x >> 5;
+    if (lane_id() == 0) { s64[w][0] = va; s64[w][1] = ea; s64[w][2] = ed; s32[w][0] = mx; s32[w][1] = mn; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int i = 1; i < kWarps; ++i) {
+            va += s64[i][0]; ea += s64[i][1]; ed += s64[i][2];
+            mx = s32[i][0] > mx ? s32[i][0] : mx;
+            mn = s32[i][1] < mn ? s32[i][1] : mn;
+        }
+        if (va) { atomicAdd(&dst->va, va); atomicAdd(&dst->ea, ea); atomicMax(&dst->maxd, mx); atomicMin(&dst->mind, mn); }
+        if (ed) atomicAdd(&dst->edges, ed);
+    }
+    __syncthreads();
+    c = LocalCnt();
+}
+
+__device__ __forceinline__ void reset_cnt(IterCnt *c) {
+    c->va = 0; c->ea = 0; c->edges = 0; c->maxd = 0; c->mind = 0xffffffffu; c->qlen = 0; c->iqlen = 0;
+}
+
+// grid-stride helpers
+__device__ __forceinline__ long long gtid() { return (long long)blockIdx.x * blockDim.x + threadIdx.x; }
+__device__ __forceinline__ long long gthreads() { return (long long)gridDim.x * blockDim.x; }
+__device__ __forceinline__ long long gwarp() { return gtid() >> 5; }
+__device__ __forceinline__ long long gwarps() { return gthreads() >> 5; }
+
+}  // namespace gsw

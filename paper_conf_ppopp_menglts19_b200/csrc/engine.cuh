@@ -1,0 +1,191 @@
+// engine.cuh -- the device-resident iteration engine: control block, history/records, and the
+// Filter-side active-set builders of Pattern 2 (Fig. 4):
+//   bitmap        : one bit per vertex, no scan, idle threads on sparse sets
+//   unsorted queue: compact ids in any order, warp-aggregated atomics
+//   sorted queue  : compact ids ascending via a scan of bitmap words
+#pragma once
+#include "common.cuh"
+#include "gsw.h"
+#include "select.cuh"
+
+namespace gsw {
+
+constexpr int kMaxHist = 1 << 16;   // iterations with stored history / records
+
+struct Hist {
+    float tf, te, Tf, Te;
+};
+
+struct Ctl {
+    unsigned arrive, gen, err, iters;
+    unsigned long long edges_total, bytes_alg;
+    unsigned long long t_start, t_phase, t_expand;
+    float sum_tf, sum_te;
+    unsigned stop;
+    unsigned pad[5];
+};
+
+struct RunCommon {
+    Ctl *ctl;
+    IterCnt *cnt;            // ring of 3
+    Hist *hist;              // kMaxHist
+    gsw_iter_record *rec;    // kMaxHist
+    uint32_t *partial;       // gridDim entries (+1)
+    gsw_config force;
+    Features base;           // dataset attributes (runtime fields filled per iteration)
+};
+
+__device__ __forceinline__ GridBarrier make_bar(const RunCommon &rc) {
+    return GridBarrier{&rc.ctl->arrive, &rc.ctl->gen, &rc.ctl->err};
+}
+
+__device__ __forceinline__ void read_cnt(const IterCnt *c, unsigned long long &va, unsigned long long &ea,
+                                         unsigned &maxd, unsigned &mind, unsigned &qlen, unsigned long long &edges) {
+    va = ld_relaxed64(&c->va);
+    ea = ld_relaxed64(&c->ea);
+    edges = ld_relaxed64(&c->edges);
+    maxd = ld_relaxed(&c->maxd);
+    mind = ld_relaxed(&c->mind);
+    qlen = ld_relaxed(&c->qlen);
+}
+
+// History features of iteration t-2 (written by CTA 0 two barriers ago) -> identical in all CTAs.
+__device__ __forceinline__ void read_hist(const RunCommon &rc, int t, Features &f) {
+    f.tf = f.te = f.Tf = f.Te = 0.f;
+    if (t >= 2 && t - 2 < kMaxHist) {
+        volatile const Hist *h = rc.hist + (t - 2);
+        f.tf = h->tf; f.te = h->te; f.Tf = h->Tf; f.Te = h->Te;
+    }
+}
+
+// CTA 0 / thread 0 bookkeeping at the start of iteration t (after the barrier that ended t-1).
+__device__ __forceinline__ void stamp_iteration_start(const RunCommon &rc, int t) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        Ctl *c = rc.ctl;
+        uint64_t now = globaltimer();
+        if (t >= 1) {
+            float tf = (float)(c->t_expand - c->t_start) * 1e-3f;
+            float te = (float)(now - c->t_expand) * 1e-3f;
+            c->sum_tf += tf; c->sum_te += te;
+            if (t - 1 < kMaxHist) {
+                rc.hist[t - 1] = Hist{tf, te, c->sum_tf / t, c->sum_te / t};
+                rc.rec[t - 1].filter_us = tf;
+                rc.rec[t - 1].expand_us = te;
+            }
+        }
+        c->t_start = now;
+        c->t_expand = now;
+    }
+}
+__device__ __forceinline__ void stamp_expand_start(const RunCommon &rc) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) rc.ctl->t_expand = globaltimer();
+}
+
+__device__ __forceinline__ void write_record(const RunCommon &rc, int t, const DevCfg &c, const Features &f,
+                                             unsigned theta) {
+    if (blockIdx.x == 0 && threadIdx.x == 0 && t < kMaxHist) {
+        gsw_iter_record r;
+        r.iteration = t;
+        r.direction = c.dir; r.format = c.fmt; r.load_balance = c.lb; r.stepping = c.step; r.fusion = c.fused;
+        r.Va = f.Va; r.Ea = f.Ea; r.Via = f.Via; r.Eia = f.Eia;
+        r.edges = 0;
+        r.theta = theta;
+        r.filter_us = 0.f; r.expand_us = 0.f;
+        rc.rec[t] = r;
+    }
+}
+
+// ------------------------------------------------------------------ active-set builders
+// bitmap from a per-vertex predicate: one warp per 32-vertex word, ballot, one store
+template <class Pred>
+__device__ inline void bm_from_pred(unsigned *bm, int n, Pred pred) {
+    int W = (n + 31) >> 5;
+    for (long long w = gwarp(); w < W; w += gwarps()) {
+        int v = (int)(w * 32 + lane_id());
+        bool b = v < n && pred(v);
+        unsigned m = __ballot_sync(0xffffffffu, b);
+        if (lane_id() == 0) bm[w] = m;
+    }
+}
+// unsorted queue from a per-vertex predicate (ascending within a warp, warps in any order)
+template <class Pred>
+__device__ inline void q_from_pred(int *q, unsigned *len, int n, Pred pred) {
+    int W = (n + 31) >> 5;
+    for (long long w = gwarp(); w < W; w += gwarps()) {
+        int v = (int)(w * 32 + lane_id());
+        bool b = v < n && pred(v);
+        unsigned m = __ballot_sync(0xffffffffu, b);
+        if (!m) continue;
+        unsigned base = 0;
+        if (lane_id() == 0) base = atomicAdd(len, (unsigned)__popc(m));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (b) q[base + __popc(m & lanemask_lt())] = v;
+    }
+}
+// unsorted queue from bitmap words (word ^ flip; flip=~0 takes the zero bits)
+__device__ inline void q_from_bm(int *q, unsigned *len, const unsigned *bm, int W, unsigned flip) {
+    for (long long w0 = gwarp() * 32; w0 < W; w0 += gwarps() * 32) {
+        long long w = w0 + lane_id();
+        unsigned word = w < W ? (bm[w] ^ flip) : 0u;
+        unsigned c = __popc(word);
+        unsigned inc = warp_incl_scan(c);
+        unsigned tot = __shfl_sync(0xffffffffu, inc, 31);
+        if (!tot) continue;
+        unsigned base = 0;
+        if (lane_id() == 31) base = atomicAdd(len, tot);
+        base = __shfl_sync(0xffffffffu, base, 31);
+        unsigned pos = base + inc - c;
+        while (word) {
+            int b = __ffs(word) - 1;
+            word &= word - 1;
+            q[pos++] = (int)(w * 32 + b);
+        }
+    }
+}
+// sorted queue from bitmap words, pass 1: per-CTA popcount of a contiguous word range
+__device__ inline void sq_from_bm_p1(const unsigned *bm, int W, unsigned flip, uint32_t *partial, uint32_t *red) {
+    unsigned chunk = (W + gridDim.x - 1) / gridDim.x;
+    unsigned lo = blockIdx.x * chunk, hi = min((unsigned)W, lo + chunk);
+    uint32_t s = 0;
+    for (unsigned w = lo + threadIdx.x; w < hi; w += kBlock) s += __popc(bm[w] ^ flip);
+    s = block_sum(s, red);
+    if (threadIdx.x == 0) partial[blockIdx.x] = s;
+}
+// pass 2 (after a grid barrier): scatter ids in ascending order; the last CTA stores the length
+__device__ inline void sq_from_bm_p2(int *q, unsigned *len, const unsigned *bm, int W, unsigned flip,
+                              const uint32_t *partial, uint32_t *red) {
+    unsigned chunk = (W + gridDim.x - 1) / gridDim.x;
+    unsigned lo = blockIdx.x * chunk, hi = min((unsigned)W, lo + chunk);
+    uint32_t before = 0;
+    for (unsigned j = threadIdx.x; j < blockIdx.x; j += kBlock) before += ((volatile const uint32_t *)partial)[j];
+    before = block_sum(before, red);
+    uint32_t base = before;
+    for (unsigned t0 = lo; t0 < hi; t0 += kBlock) {
+        unsigned w = t0 + threadIdx.x;
+        unsigned word = w < hi ? (bm[w] ^ flip) : 0u;
+        uint32_t tot;
+        uint32_t ex = block_excl_scan((uint32_t)__popc(word), red, &tot);
+        uint32_t pos = base + ex;
+        while (word) {
+            int b = __ffs(word) - 1;
+            word &= word - 1;
+            q[pos++] = (int)(w * 32 + b);
+        }
+        base += tot;
+    }
+    if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) *len = base;
+}
+__device__ inline void bm_from_q(unsigned *bm, const int *q, unsigned len) {
+    for (long long i = gtid(); i < len; i += gthreads()) {
+        int v = q[i];
+        atomicOr(bm + (v >> 5), 1u << (v & 31));
+    }
+}
+__device__ inline void clear_words(unsigned *bm, int W) {
+    for (long long w = gtid(); w < W; w += gthreads()) bm[w] = 0u;
+}
+__device__ inline void copy_words(unsigned *dst, const unsigned *src, int W) {
+    for (long long w = gtid(); w < W; w += gthreads()) dst[w] = src[w];
+}
+
+}  // namespace gsw

@@ -1,0 +1,211 @@
+// graph.cu -- step a0 of the hot path: ingest + dataset attributes (Table 1; "computed
+// only once while loading the data into the memory").  Not inside any timed run.
+#include <cmath>
+#include <cstring>
+#include <vector>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace gsw {
+
+namespace {
+
+__global__ void k_offsets_to_u32(const int64_t *in, uint32_t *out, long long n1) {
+    for (long long i = gtid(); i < n1; i += gthreads()) out[i] = (uint32_t)in[i];
+}
+
+// isolated bitmap: bit v = 1 if deg(v) == 0 or v >= n (padding bits)
+__global__ void k_isolated_bitmap(const uint32_t *off, int n, unsigned *iso, int W) {
+    for (long long w = gwarp(); w < W; w += gwarps()) {
+        int v = (int)(w * 32 + lane_id());
+        bool b = v >= n || off[v + 1] == off[v];
+        unsigned m = __ballot_sync(0xffffffffu, b);
+        if (lane_id() == 0) iso[w] = m;
+    }
+}
+
+struct AttrAcc {
+    unsigned long long sum, iso;
+    double sumsq, dlnd;
+    unsigned maxd, mind, maxw, bad;
+};
+
+__global__ void k_attrs(const uint32_t *off, int n, AttrAcc *acc) {
+    __shared__ double sd[kWarps];
+    __shared__ unsigned long long su[kWarps];
+    unsigned long long s = 0, iso = 0;
+    double sq = 0, dl = 0;
+    unsigned mx = 0, mn = 0xffffffffu;
+    for (long long v = gtid(); v < n; v += gthreads()) {
+        unsigned d = off[v + 1] - off[v];
+        s += d; sq += (double)d * d;
+        if (d) dl += (double)d * log((double)d); else iso++;
+        mx = max(mx, d); mn = min(mn, d);
+    }
+    s = block_sum(s, su);
+    iso = block_sum(iso, su);
+    sq = block_sum(sq, sd);
+    dl = block_sum(dl, sd);
+    __shared__ unsigned smx[kWarps], smn[kWarps];
+    mx = warp_max(mx); mn = warp_min(mn);
+    if (lane_id() == 0) { smx[threadIdx.x >> 5] = mx; smn[threadIdx.x >> 5] = mn; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int i = 1; i < kWarps; ++i) { mx = max(mx, smx[i]); mn = min(mn, smn[i]); }
+        atomicAdd(&acc->sum, s); atomicAdd(&acc->iso, iso);
+        atomicAdd(&acc->sumsq, sq); atomicAdd(&acc->dlnd, dl);
+        atomicMax(&acc->maxd, mx); atomicMin(&acc->mind, mn);
+    }
+}
+
+__global__ void k_degree_hist(const uint32_t *off, int n, unsigned long long *hist) {
+    for (long long v = gtid(); v < n; v += gthreads()) atomicAdd(&hist[off[v + 1] - off[v]], 1ull);
+}
+
+__global__ void k_maxw(const uint32_t *w, long long nnz, AttrAcc *acc) {
+    unsigned mx = 0;
+    for (long long e = gtid(); e < nnz; e += gthreads()) mx = max(mx, w[e]);
+    mx = warp_max(mx);
+    if (lane_id() == 0) atomicMax(&acc->maxw, mx);
+}
+
+__global__ void k_validate(const uint32_t *off, const int32_t *col, int n, long long nnz, unsigned *bad) {
+    for (long long v = gtid(); v < n; v += gthreads())
+        if (off[v + 1] < off[v]) atomicOr(bad, 1u);
+    for (long long e = gtid(); e < nnz; e += gthreads())
+        if (col[e] < 0 || col[e] >= n) atomicOr(bad, 2u);
+}
+
+inline int grid_for(long long work, int sms) {
+    long long b = (work + kBlock - 1) / kBlock;
+    long long cap = (long long)sms * 8;
+    return (int)std::max(1LL, std::min(b, cap));
+}
+
+}  // namespace
+
+size_t graph_bytes(int64_t n, int64_t nnz, int has_w, int has_csc) {
+    size_t W = (size_t)((n + 31) / 32);
+    size_t b = 0;
+    auto add = [&](size_t x) { b += (x + 255) & ~size_t(255); };
+    add((n + 1) * 4); add(nnz * 4); if (has_w) add(nnz * 4);
+    if (has_csc) { add((n + 1) * 4); add(nnz * 4); if (has_w) add(nnz * 4); }
+    add(W * 4);  // isolated bitmap
+    return b;
+}
+
+// Per-run scratch: the maximum over algorithms.
+size_t scratch_bytes_for(int64_t n, int64_t nnz) {
+    (void)nnz;
+    size_t W = (size_t)((n + 31) / 32);
+    size_t per_v = 64;                         // BC: depth 4 + sigma 8 + delta 8 + stack 4 + bc 8 + queues
+    size_t b = per_v * (size_t)(n + 64) + 16 * W * 4;
+    b += (size_t)(n + 1) * 8;                  // i64 offset staging at ingest / scan arrays
+    b += 8u << 20;                             // control blocks, per-CTA partials, history, records
+    return b;
+}
+
+int is_device_ptr(const void *p) {
+    if (!p) return 0;
+    cudaPointerAttributes a;
+    cudaError_t e = cudaPointerGetAttributes(&a, p);
+    if (e != cudaSuccess) { cudaGetLastError(); return 0; }
+    return (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) ? 1 : 0;
+}
+
+static gsw_status copy_in(void *dst, const void *src, size_t bytes, cudaStream_t s) {
+    if (bytes == 0) return GSW_OK;
+    cudaMemcpyKind k = is_device_ptr(src) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+    GSW_CUDA(cudaMemcpyAsync(dst, src, bytes, k, s));
+    return GSW_OK;
+}
+
+gsw_status load_csr(gsw_graph g, const gsw_csr *c, Workspace &ws, uint32_t **off, int32_t **col,
+                    uint32_t **w, int64_t *staging) {
+    int64_t n = c->n, nnz = c->nnz;
+    *off = (uint32_t *)ws.take((n + 1) * 4);
+    *col = (int32_t *)ws.take(std::max<int64_t>(nnz, 1) * 4);
+    *w = nullptr;
+    if (c->weights) *w = (uint32_t *)ws.take(std::max<int64_t>(nnz, 1) * 4);
+    if (!*off || !*col || (c->weights && !*w)) { set_error("workspace too small for the graph"); return GSW_ENOMEM; }
+    gsw_status st;
+    const int64_t *off64 = c->row_offsets;
+    if (!is_device_ptr(off64)) {
+        if ((st = copy_in(staging, off64, (n + 1) * 8, g->stream)) != GSW_OK) return st;
+        off64 = staging;
+    }
+    k_offsets_to_u32<<<grid_for(n + 1, g->sms), kBlock, 0, g->stream>>>(off64, *off, n + 1);
+    GSW_CUDA(cudaGetLastError());
+    if ((st = copy_in(*col, c->col_indices, nnz * 4, g->stream)) != GSW_OK) return st;
+    if (c->weights && (st = copy_in(*w, c->weights, nnz * 4, g->stream)) != GSW_OK) return st;
+    return GSW_OK;
+}
+
+gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp) {
+    const DevGraph &G = g->g;
+    int n = G.n;
+    int W = (n + 31) / 32;
+    k_isolated_bitmap<<<grid_for((long long)W * 32, g->sms), kBlock, 0, g->stream>>>(G.off, n, iso_bitmap, W);
+    AttrAcc *acc = (AttrAcc *)tmp;
+    AttrAcc init{};
+    init.mind = 0xffffffffu;
+    GSW_CUDA(cudaMemcpyAsync(acc, &init, sizeof(init), cudaMemcpyHostToDevice, g->stream));
+    k_attrs<<<grid_for(n, g->sms), kBlock, 0, g->stream>>>(G.off, n, acc);
+    if (G.w) k_maxw<<<grid_for(G.nnz, g->sms), kBlock, 0, g->stream>>>(G.w, G.nnz, acc);
+    GSW_CUDA(cudaGetLastError());
+    AttrAcc h;
+    GSW_CUDA(cudaMemcpyAsync(&h, acc, sizeof(h), cudaMemcpyDeviceToHost, g->stream));
+    GSW_CUDA(cudaStreamSynchronize(g->stream));
+    // degree histogram -> Gini over ascending degrees (counting sort order)
+    size_t nb = (size_t)h.maxd + 1;
+    unsigned long long *hist = (unsigned long long *)((char *)tmp + 256);
+    GSW_CUDA(cudaMemsetAsync(hist, 0, nb * 8, g->stream));
+    k_degree_hist<<<grid_for(n, g->sms), kBlock, 0, g->stream>>>(G.off, n, hist);
+    GSW_CUDA(cudaGetLastError());
+    std::vector<unsigned long long> hh(nb);
+    GSW_CUDA(cudaMemcpyAsync(hh.data(), hist, nb * 8, cudaMemcpyDeviceToHost, g->stream));
+    GSW_CUDA(cudaStreamSynchronize(g->stream));
+    double N = n, S = (double)h.sum, dbar = S / N;
+    double gnum = 0.0, r = 0.0;                 // sum_i (2i - N - 1) d_(i), ranks r+1..r+c
+    for (size_t k = 0; k < nb; ++k) {
+        double c = (double)hh[k];
+        if (c == 0) continue;
+        gnum += (double)k * (c * (2.0 * r + c + 1.0) - c * (N + 1.0));
+        r += c;
+    }
+    Attrs &A = g->attrs;
+    A.N = N;
+    A.M = S / 2.0;
+    A.dbar = dbar;
+    double var = h.sumsq / N - dbar * dbar;
+    A.sd = std::sqrt(std::max(0.0, var));
+    A.rd = dbar > 0 ? (double)(h.maxd - h.mind) / dbar : 0.0;
+    A.gini = S > 0 ? gnum / (N * S) : 0.0;
+    // H_er = -sum (d/S) ln(d/S) / ln N = (ln S - (1/S) sum d ln d) / ln N
+    A.her = (S > 0 && n > 1) ? (std::log(S) - h.dlnd / S) / std::log(N) : 0.0;
+    A.maxdeg = h.maxd;
+    A.mindeg = h.mind;
+    A.maxw = h.maxw;
+    A.isolated = (int64_t)h.iso;
+    return GSW_OK;
+}
+
+gsw_status validate_graph(gsw_graph g) {
+    unsigned *bad = (unsigned *)g->scratch;
+    GSW_CUDA(cudaMemsetAsync(bad, 0, 4, g->stream));
+    k_validate<<<grid_for(std::max<long long>(g->g.n, g->g.nnz), g->sms), kBlock, 0, g->stream>>>(
+        g->g.off, g->g.col, g->g.n, g->g.nnz, bad);
+    if (!g->symmetric)
+        k_validate<<<grid_for(std::max<long long>(g->g.n, g->g.nnz), g->sms), kBlock, 0, g->stream>>>(
+            g->g.in_off, g->g.in_col, g->g.n, g->g.nnz, bad);
+    GSW_CUDA(cudaGetLastError());
+    unsigned hb = 0;
+    GSW_CUDA(cudaMemcpyAsync(&hb, bad, 4, cudaMemcpyDeviceToHost, g->stream));
+    GSW_CUDA(cudaStreamSynchronize(g->stream));
+    if (hb & 1u) { set_error("row offsets are not monotone"); return GSW_EINVAL; }
+    if (hb & 2u) { set_error("column index out of range"); return GSW_EINVAL; }
+    return GSW_OK;
+}
+
+}  // namespace gsw

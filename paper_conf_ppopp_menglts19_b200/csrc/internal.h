@@ -1,0 +1,86 @@
+// internal.h -- host-side internals of libgsw (graph handle, workspace carving, error plumbing).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <string>
+#include <cuda_runtime.h>
+
+#include "gsw.h"
+
+namespace gsw {
+
+// Device view of the graph: u32 offsets (nnz < 2^32), int32 columns, optional u32 weights.
+// For symmetric inputs the CSC fields alias the CSR (all graphs undirected).
+struct DevGraph {
+    int n;
+    uint32_t nnz;
+    const uint32_t *off;      // n+1  (out-edges, push)
+    const int32_t *col;       // nnz
+    const uint32_t *w;        // nnz or nullptr
+    const uint32_t *in_off;   // n+1  (in-edges, pull)
+    const int32_t *in_col;
+    const uint32_t *in_w;
+};
+
+// Dataset attributes (Table 1), computed once at load.
+struct Attrs {
+    double N, M, dbar, sd, rd, gini, her;
+    uint32_t maxdeg, mindeg, maxw;
+    int64_t isolated;
+};
+
+// Packed per-iteration configuration (Fig. 13: one choice per pattern).
+struct Cfg {
+    int8_t dir, fmt, lb, step, fused;
+};
+
+struct Workspace {
+    char *base = nullptr;
+    size_t size = 0, used = 0;
+    void *take(size_t bytes) {
+        size_t a = (used + 255) & ~size_t(255);
+        if (a + bytes > size) return nullptr;
+        used = a + bytes;
+        return base + a;
+    }
+};
+
+}  // namespace gsw
+
+struct gsw_graph_s {
+    gsw::DevGraph g{};
+    gsw::Attrs attrs{};
+    bool symmetric = true;
+    cudaStream_t stream = nullptr;
+    int device = 0, sms = 0;
+    gsw_config forced{};
+    unsigned *iso = nullptr;      // isolated-vertex bitmap (deg 0 or padding), W words
+    // workspace regions
+    char *ws = nullptr;
+    size_t ws_bytes = 0;
+    char *scratch = nullptr;      // per-run scratch (after the graph copy)
+    size_t scratch_bytes = 0;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+};
+
+namespace gsw {
+
+void set_error(const std::string &msg);
+gsw_status cuda_fail(cudaError_t e, const char *what);
+
+#define GSW_CUDA(call)                                                   \
+    do {                                                                 \
+        cudaError_t _e = (call);                                         \
+        if (_e != cudaSuccess) return ::gsw::cuda_fail(_e, #call);       \
+    } while (0)
+
+// scratch bytes for a graph of n vertices (max over algorithms), see DESIGN.md "HBM layout"
+size_t scratch_bytes_for(int64_t n, int64_t nnz);
+
+// 1 if p is device (or managed) memory, 0 if host, -1 on error
+int is_device_ptr(const void *p);
+
+// records copy-out helper
+struct RunRecords;
+
+}  // namespace gsw

@@ -1,0 +1,76 @@
+// launch.cu -- persistent cooperative launch + run bookkeeping shared by all algorithms.
+#include <algorithm>
+#include <map>
+#include <mutex>
+
+#include "launch.h"
+
+namespace gsw {
+
+static int blocks_per_sm(const void *kernel) {
+    static std::mutex mu;
+    static std::map<const void *, int> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(kernel);
+    if (it != cache.end()) return it->second;
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, kBlock, 0) != cudaSuccess) {
+        cudaGetLastError();
+        nb = 1;
+    }
+    nb = std::max(1, std::min(nb, kMinBlocks));
+    cache[kernel] = nb;
+    return nb;
+}
+
+gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li) {
+    li.grid = g->sms * blocks_per_sm(kernel);
+    rc.ctl = (Ctl *)ws.take(sizeof(Ctl));
+    rc.cnt = (IterCnt *)ws.take(3 * sizeof(IterCnt));
+    rc.hist = (Hist *)ws.take(sizeof(Hist) * kMaxHist);
+    rc.rec = (gsw_iter_record *)ws.take(sizeof(gsw_iter_record) * kMaxHist);
+    rc.partial = (uint32_t *)ws.take(sizeof(uint32_t) * (li.grid + 1));
+    if (!rc.ctl || !rc.cnt || !rc.hist || !rc.rec || !rc.partial) {
+        set_error("workspace too small for the run's control blocks");
+        return GSW_ENOMEM;
+    }
+    rc.force = g->forced;
+    const Attrs &A = g->attrs;
+    Features f{};
+    f.N = (float)A.N; f.M = (float)A.M; f.dbar = (float)A.dbar; f.sd = (float)A.sd; f.rd = (float)A.rd;
+    f.gini = (float)A.gini; f.her = (float)A.her;
+    rc.base = f;
+    GSW_CUDA(cudaMemsetAsync(rc.ctl, 0, sizeof(Ctl), g->stream));
+    return GSW_OK;
+}
+
+gsw_status launch_persistent(gsw_graph g, const void *kernel, void **args, const LaunchInfo &li) {
+    GSW_CUDA(cudaEventRecord(g->ev0, g->stream));
+    GSW_CUDA(cudaLaunchCooperativeKernel(kernel, dim3(li.grid), dim3(kBlock), args, 0, g->stream));
+    GSW_CUDA(cudaEventRecord(g->ev1, g->stream));
+    return GSW_OK;
+}
+
+gsw_status finish_run(gsw_graph g, const RunCommon &rc, const LaunchInfo &li, gsw_run_stats *st) {
+    (void)li;
+    Ctl h{};
+    GSW_CUDA(cudaMemcpyAsync(&h, rc.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g->stream));
+    GSW_CUDA(cudaStreamSynchronize(g->stream));
+    if (h.err) { set_error("device error code " + std::to_string(h.err)); return GSW_ECUDA; }
+    if (st) {
+        float ms = 0.f;
+        GSW_CUDA(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+        st->iterations = (int32_t)h.iters;
+        st->gpu_ms = ms;
+        st->edges_touched = (int64_t)h.edges_total;
+        st->bytes_alg = (int64_t)h.bytes_alg;
+        if (st->records && st->max_records > 0) {
+            int nr = std::min<int>({(int)h.iters, st->max_records, kMaxHist});
+            if (nr > 0)
+                GSW_CUDA(cudaMemcpy(st->records, rc.rec, sizeof(gsw_iter_record) * nr, cudaMemcpyDeviceToHost));
+        }
+    }
+    return GSW_OK;
+}
+
+}  // namespace gsw

@@ -1,0 +1,71 @@
+// select.cuh -- Inspector features + Selector (Sec. 4.3-4.5, Table 1, Fig. 12-13).
+//
+// The paper trains one CART tree per pattern offline on 386,780 records from 644 real graphs
+// and applies them in the order direction -> load balance -> format -> stepping ->
+// fusion.  Those trees are not printed and the corpus is out of scope, so the trees
+// below are shallow hand-set if-else rules that encode the paper's stated findings (each rule
+// cites the sentence it follows) with thresholds calibrated on B200.
+// Every CTA evaluates the selector redundantly on identical inputs, so all CTAs agree on the
+// configuration without an extra barrier.
+#pragma once
+#include "common.cuh"
+#include "gsw.h"
+
+namespace gsw {
+
+struct Features {
+    // dataset attributes (Table 1)
+    float N, M, dbar, sd, rd, gini, her;
+    // runtime characteristics of the current iteration
+    long long Va, Ea, Via, Eia;
+    unsigned maxd, mind;
+    // historical information, lagged by one iteration (reading R9)
+    float tf, te, Tf, Te;
+    int iter;
+};
+
+struct DevCfg {
+    int dir, fmt, lb, step, fused;
+};
+
+__device__ __forceinline__ int pick(int forced, int chosen) { return forced != GSW_AUTO ? forced : chosen; }
+
+// BFS-like traversal (BFS, BC forward): active = frontier, inactive = unvisited.
+__device__ __forceinline__ DevCfg select_traversal(const Features &f, const gsw_config &force) {
+    DevCfg c;
+    // P1 direction: "the pull mode is preferable ... when the number of the active edges is
+    // greater than that of inactive edges".
+    c.dir = pick(force.direction, f.Ea > f.Eia ? GSW_PULL : GSW_PUSH);
+    float cd = f.Va > 0 ? (float)f.Ea / (float)f.Va : 0.f;
+    // P3 load balance: "TWC has the lowest overhead", "CM and WM perform better with irregular
+    // workloads", "when the workload contains a hub vertex ... STRICT is the best";
+    // Fig. 14 picks TWC for every pull iteration.
+    int lb;
+    if (c.dir == GSW_PULL) lb = GSW_LB_TWC;
+    else if (f.Ea < 8192) lb = GSW_LB_WM;                                   // tiny, latency-bound
+    else if (f.maxd > 32u * kBlock && f.maxd > 64.f * cd) lb = GSW_LB_STRICT;  // hub in workload
+    else if (f.maxd > 16.f * cd) lb = GSW_LB_CM;                             // irregular
+    else lb = GSW_LB_TWC;
+    c.lb = pick(force.load_balance, lb);
+    // P2 format: "bitmap is more friendly to dense workloads, the unsorted queue is more friendly
+    // to sparse workloads, and the sorted queue is in the middle"; Fig. 12(b): queue
+    // when the number of active vertices is small.
+    float vap = f.N > 0 ? (float)f.Va / f.N : 0.f;
+    int fmt;
+    if (c.dir == GSW_PULL) fmt = GSW_BITMAP;
+    else if (vap > 1.f / 32.f) fmt = GSW_BITMAP;
+    else if (vap > 1.f / 512.f) fmt = GSW_SORTED_QUEUE;
+    else fmt = GSW_QUEUE;
+    c.fmt = pick(force.format, fmt);
+    c.step = GSW_STEP_REMAIN;
+    // P5 fusion: fused kernels are preferred when degrees are similar (Fig. 12(f));
+    // fall back to standalone when the last iteration took far longer than the fused average
+    // (P:681-682).  With atomic bitmap claiming the fused variant generates no
+    // duplicates on B200, so it is also the default on skewed graphs.
+    int fused = GSW_FUSED;
+    if (f.iter >= 3 && f.Te > 0.f && (f.te + f.tf) > 4.f * (f.Te + f.Tf)) fused = GSW_STANDALONE;
+    c.fused = pick(force.fusion, fused);
+    return c;
+}
+
+}  // namespace gsw

@@ -1,0 +1,123 @@
+"""BFS parity: CUDA path (through the C ABI) vs the CPU oracle, bit-exact depths and per-level
+runtime characteristics (forced-variant sweep c7)."""
+import itertools
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from tests.conftest import tiny_graphs
+
+pytestmark = pytest.mark.gpu
+
+DIRS = ["push", "pull"]
+FMTS = ["bitmap", "queue", "sorted_queue"]
+LBS = ["thread", "twc", "wm", "cm", "strict"]
+FUS = ["standalone", "fused"]
+ALL_VARIANTS = list(itertools.product(DIRS, FMTS, LBS, FUS))
+
+
+@pytest.fixture(scope="module")
+def gsw():
+    import torch
+    assert torch.cuda.is_available()
+    import paper_conf_ppopp_menglts19_b200 as m
+    return m
+
+
+def _bfs(G, s, **kw):
+    d, st = G.bfs(s, **kw)
+    return d.cpu().numpy(), st
+
+
+@pytest.mark.parametrize("name", sorted(tiny_graphs()))
+def test_tiny_all_sources(gsw, name):
+    g = tiny_graphs()[name]
+    G = gsw.Graph(g.off, g.col)
+    for s in range(g.n):
+        d, _ = _bfs(G, s)
+        assert np.array_equal(d, oracle.bfs(g, s)), (name, s)
+
+
+@pytest.mark.parametrize("variant", ALL_VARIANTS, ids=["-".join(v) for v in ALL_VARIANTS])
+def test_forced_variant_sweep(gsw, variant):
+    d_, f_, l_, u_ = variant
+    for g in (gen.rmat(13, seed=3), gen.grid(64, 37)):
+        G = gsw.Graph(g.off, g.col)
+        G.force_config(direction=d_, format=f_, load_balance=l_, fusion=u_)
+        for s in gen.sources(g, 2, seed=11):
+            d, st = _bfs(G, s, records=64)
+            assert np.array_equal(d, oracle.bfs(g, s)), (variant, g.name, s)
+            for r in st["records"]:
+                assert r["direction"] == gsw.DIRECTIONS[d_] and r["load_balance"] == gsw.LOAD_BALANCES[l_]
+
+
+def test_features_match_oracle_per_level(gsw):
+    g = gen.rmat(14, seed=2)
+    G = gsw.Graph(g.off, g.col)
+    for s in gen.sources(g, 3):
+        _, st = _bfs(G, s, records=256)
+        Va, Ea, Via, Eia = oracle.bfs_features(g, s)
+        rec = st["records"]
+        assert st["iterations"] == len(Va) == len(rec)
+        assert [r["Va"] for r in rec] == Va.tolist()
+        assert [r["Ea"] for r in rec] == Ea.tolist()
+        assert [r["Via"] for r in rec] == Via.tolist()
+        assert [r["Eia"] for r in rec] == Eia.tolist()
+        # direction rule "pull when active edges > inactive edges" reproduced exactly
+        for r in rec:
+            assert r["direction"] == (gsw.PULL if r["Ea"] > r["Eia"] else gsw.PUSH)
+
+
+def test_attributes_match_oracle(gsw):
+    g = gen.rmat(14, seed=2)
+    a = gsw.Graph(g.off, g.col).attributes()
+    o = oracle.attrs(g)
+    for k in o:
+        assert abs(a[k] - o[k]) <= 1e-9 * max(1.0, abs(o[k])), k
+
+
+def test_c1_full_size(gsw):
+    g = gen.config_graph("C1")
+    G = gsw.Graph(g.off, g.col)
+    for s in gen.sources(g, 8):
+        d, _ = _bfs(G, s)
+        assert np.array_equal(d, oracle.bfs(g, s))
+
+
+def test_host_buffers_e2e(gsw):
+    import torch
+    g = gen.rmat(12)
+    G = gsw.Graph(g.off, g.col)
+    out = torch.empty(g.n, dtype=torch.int32).pin_memory()
+    s = gen.sources(g, 1)[0]
+    G.bfs(s, out=out)
+    assert np.array_equal(out.numpy(), oracle.bfs(g, s))
+    # graph created from device tensors
+    G2 = gsw.Graph(torch.from_numpy(g.off).cuda(), torch.from_numpy(g.col).cuda())
+    d, _ = _bfs(G2, s)
+    assert np.array_equal(d, oracle.bfs(g, s))
+
+
+def test_edge_cases(gsw):
+    g = gen.from_edges(5, [(1, 2)])
+    G = gsw.Graph(g.off, g.col)
+    d, st = _bfs(G, 0)                    # isolated source
+    assert d.tolist() == [0, -1, -1, -1, -1] and st["iterations"] == 1
+    with pytest.raises(gsw.GswError):
+        G.bfs(5)
+    with pytest.raises(gsw.GswError):
+        G.bfs(-1)
+    one = gen.from_edges(1, [])
+    d, _ = _bfs(gsw.Graph(one.off, one.col), 0)
+    assert d.tolist() == [0]
+
+
+@pytest.mark.slow
+def test_c3_full_size(gsw):
+    g = gen.config_graph("C3")
+    G = gsw.Graph(g.off, g.col)
+    for s in gen.sources(g, 2):
+        d, st = _bfs(G, s, records=64)
+        assert np.array_equal(d, oracle.bfs(g, s))
