@@ -1,0 +1,286 @@
+#!/usr/bin/env python
+"""Benchmark of the GSWITCH frontier-step hot path on B200 (BASELINE.json metric, config C3).
+
+Headline workload (north_star: ">=40% of the B200 HBM roofline on RMAT scale-22 BFS at 1 GPU"):
+BFS on the C3 graph (Graph500 R-MAT scale 22, edge factor 16, symmetrised), roots from the
+SURVEY Q12 source stream.  One step = one autotuned gsw_bfs call (features -> selector -> Filter
+-> Expand per level, all inside one persistent kernel) from the next root.
+
+  python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--workload bfs|...]
+
+Prints ONE JSON line on rank 0.  GTEPS = sum over steps of m_cc / device time, with m_cc = the
+undirected edges with both endpoints reached.  L2 is flushed (256 MiB write) between
+timed steps; each step is timed with CUDA events on the library stream; max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_HBM = 6650.0   # GB/s, B200_PROFILING.md fallback
+
+
+def hbm_peak():
+    try:
+        with open(PEAKS_FILE) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "50"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        self.out = ""
+        if self.p:
+            time.sleep(0.12)
+            self.p.terminate()
+            try:
+                self.out, _ = self.p.communicate(timeout=5)
+            except Exception:
+                self.out = ""
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in (self.out or "").strip().splitlines():
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def m_cc(deg, depth):
+    return int(deg[depth >= 0].sum()) // 2
+
+
+def build_graph(name):
+    import gen
+    t0 = time.time()
+    g = gen.config_graph(name)
+    return g, time.time() - t0
+
+
+# --------------------------------------------------------------------------------------------
+def run_reference(args, ws, rank):
+    """--impl reference: the CPU oracle (plain single-threaded C) on the host cores."""
+    if rank != 0:
+        return
+    import gen
+    import oracle
+    g, _ = build_graph("C3")
+    deg = g.deg
+    roots = gen.sources(g, max(64, args.steps + args.warmup))
+    for k in range(args.warmup):
+        oracle.bfs(g, roots[k % len(roots)])
+    edges, secs = 0, 0.0
+    for k in range(args.steps):
+        s = roots[(args.warmup + k) % len(roots)]
+        t0 = time.perf_counter()
+        d = oracle.bfs(g, s)
+        secs += time.perf_counter() - t0
+        edges += m_cc(deg, d)
+    v = edges / secs / 1e9
+    line = {"impl": "reference", "metric": "BFS GTEPS", "value": v, "unit": "GTEPS", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs * 1e3 / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic",
+            "config": {"workload": "C3: BFS on R-MAT scale 22 ef 16 (Graph500 a,b,c=.57,.19,.19), roots per "
+                                   "SURVEY Q12", "parallelism": "single host thread"},
+            "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                             "sample": f"{args.steps} BFS roots, full graph, oracle.bfs (FIFO queue, 1 thread)"},
+            "e2e": {"value": v, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------------------------------------
+def cpu_baseline_sample(g, roots, budget_s=12.0):
+    import oracle
+    deg = g.deg
+    edges, secs, n = 0, 0.0, 0
+    for s in roots:
+        t0 = time.perf_counter()
+        d = oracle.bfs(g, s)
+        secs += time.perf_counter() - t0
+        edges += m_cc(deg, d)
+        n += 1
+        if secs > budget_s:
+            break
+    return {"value": edges / secs / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"{n} BFS roots on the full C3 graph, single-threaded oracle.bfs, {secs:.1f} s"}
+
+
+def run_gsw(args, ws, rank, local):
+    import torch
+    import torch.distributed as dist
+    import gen
+    import paper_conf_ppopp_menglts19_b200 as gsw
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    g, gen_s = build_graph("C3")
+    deg = g.deg
+    nroots = max(64, args.steps + args.warmup)
+    roots = gen.sources(g, nroots)
+    G = gsw.Graph(g.off, g.col, device=dev)
+    stream = G.stream
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    out = torch.empty(g.n, dtype=torch.int32, device=dev)
+
+    def step(k, timed):
+        s = roots[k % nroots]
+        flush.fill_(k & 0xff)                     # L2 flush outside the timed span
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        _, st = G.bfs(s, out=out)
+        e1.record(stream)
+        return e0, e1, st, s
+
+    for k in range(args.warmup):
+        step(k, False)
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    evs, kern_ms, bytes_alg, edges_cc = [], 0.0, 0, 0
+    with ClockSampler(local) as cs:
+        for k in range(args.steps):
+            e0, e1, st, s = step(args.warmup + k, True)
+            evs.append((e0, e1))
+            kern_ms += st["gpu_ms"]
+            bytes_alg += st["bytes_alg"]
+            edges_cc += m_cc(deg, out.cpu().numpy())      # outside the [e0, e1] span
+    torch.cuda.synchronize()
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    tot_ms = sum(step_ms)
+    if ws > 1:
+        t = torch.tensor([tot_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tot_ms = float(t.item())
+    value = ws * edges_cc / (tot_ms * 1e-3) / 1e9
+
+    # ---- roofline of the dominant kernel (the persistent BFS kernel; one launch per step)
+    peak, peak_src = hbm_peak()
+    achieved = bytes_alg / (kern_ms * 1e-3) / 1e9
+    # Graph500-equivalent bytes (full top-down): 4*nnz_cc + 20*N_cc per root (context only)
+    g500 = None
+
+    # ---- e2e: through the public API from pinned host buffers (graph H2D + BFS + depth D2H)
+    e2e = None
+    if rank == 0 or ws > 1:
+        pin_off = torch.from_numpy(g.off).pin_memory()
+        pin_col = torch.from_numpy(g.col).pin_memory()
+        host_out = torch.empty(g.n, dtype=torch.int32).pin_memory()
+        del G
+        torch.cuda.synchronize()
+        ke = min(args.steps, 8)
+        e2e_ms, e2e_edges = 0.0, 0
+        for k in range(ke + 1):
+            s = roots[k % nroots]
+            t0 = time.perf_counter()
+            G2 = gsw.Graph(pin_off, pin_col, device=dev)
+            G2.bfs(s, out=host_out)
+            dt = time.perf_counter() - t0
+            if k > 0:                              # first iteration warms the allocator
+                e2e_ms += dt * 1e3
+                e2e_edges += m_cc(deg, host_out.numpy())
+            del G2
+        e2e = {"value": e2e_edges / (e2e_ms * 1e-3) / 1e9, "unit": "GTEPS",
+               "h2d_bytes_per_step": int(g.off.nbytes + g.col.nbytes), "d2h_bytes_per_step": int(g.n * 4),
+               "note": "per step: gsw_graph_create from pinned host CSR (H2D) + gsw_bfs into pinned host "
+                       "depth (D2H); host wall clock"}
+
+    if rank == 0:
+        line = {
+            "metric": "BFS GTEPS", "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": "C3: BFS on R-MAT scale 22 ef 16 (Graph500 a,b,c=.57,.19,.19), "
+                                   f"n={g.n}, nnz={g.nnz}, roots per SURVEY Q12, autotuned",
+                       "l2": "flushed between steps (256 MiB write outside the timed span)",
+                       "parallelism": "replicas" if ws > 1 else "single GPU"},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                         "kernel": "gsw::bfs_kernel (persistent, 1 launch/step)",
+                         "bytes_model": "SURVEY 8(d) D0 per-level algorithmic bytes of the executed variant"},
+            "gpu_launches": args.steps,
+            "e2e": e2e,
+            "clocks": cs.summary(),
+            "gen_seconds": gen_s,
+        }
+        if not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline_sample(g, roots[:8])
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=32)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gsw", choices=["gsw", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    ws, rank, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, ws, rank)
+    else:
+        run_gsw(args, ws, rank, local)
+
+
+if __name__ == "__main__":
+    main()

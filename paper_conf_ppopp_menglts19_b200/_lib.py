@@ -9,7 +9,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgsw.so")
+LIB_PATH = os.environ.get("GSW_LIB_PATH") or os.path.join(_HERE, "libgsw.so")   # override: A/B builds
 
 # ---- enums (include/gsw.h) ----------------------------------------------------------------
 GSW_OK, GSW_EINVAL, GSW_ENOMEM, GSW_ECUDA, GSW_ENCCL, GSW_EUNSUPPORTED, GSW_EOVERFLOW = range(7)

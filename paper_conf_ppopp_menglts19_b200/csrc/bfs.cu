@@ -33,30 +33,12 @@ struct BfsArgs {
     RunCommon rc;
 };
 
-union TravSmem {
-    TwcSmem twc;
-    CmSmem cm;
-    StrictSmem strict;
+// Five-stage edge op (lb.cuh edge_batch): probe -> act (atomic issued, result kept raw) -> aux
+// (degree of a winner) -> commit.  Tok carries the raw atomicOr result; ~0u means "not claimed".
+struct ClaimTok {
+    unsigned old;
+    unsigned flag;   // push: unused; pull: target is active (stop scanning)
 };
-
-template <class Src, class Op>
-__device__ __forceinline__ void run_lb(int lb, const Src &src, const Adj &adj, Op &op, LocalCnt &cnt, TravSmem &sm,
-                                       uint32_t *red, const GridBarrier &bar, unsigned &epoch, uint32_t *partial,
-                                       uint32_t *scan) {
-    switch (lb) {
-    case GSW_LB_THREAD: lb_thread(src, adj, op, cnt); break;
-    case GSW_LB_TWC: lb_twc(src, adj, op, cnt, &sm.twc); break;
-    case GSW_LB_WM: lb_wm(src, adj, op, cnt); break;
-    case GSW_LB_CM: lb_cm(src, adj, op, cnt, &sm.cm); break;
-    default: {
-        strict_scan_p1(src, adj, partial, red);
-        grid_sync(bar, epoch);
-        uint32_t total = strict_scan_p2(src, adj, partial, scan, red);
-        grid_sync(bar, epoch);
-        lb_strict(src, adj, op, cnt, scan, total, &sm.strict);
-    }
-    }
-}
 
 // push: for active u and out-neighbour v, claim v if Inactive (compAtomic), depth[v] = lvl+1
 struct BfsPushOp {
@@ -64,19 +46,32 @@ struct BfsPushOp {
     unsigned *V;
     const uint32_t *off;
     int lvl1;
-    bool fused;
+    int fused;                // 0 standalone, 1 fused -> append to queue, 2 fused -> mark bitmap
     int *nq;
     unsigned *nqlen;
+    unsigned *nfb;
+    using Probe = unsigned;
+    using Tok = ClaimTok;
+    using Aux = uint2;
     static constexpr bool kEarlyExit = false;
     __device__ __forceinline__ bool skip(int) const { return false; }
-    __device__ __forceinline__ bool edge(int, uint32_t, int v, LocalCnt &c) const {
-        bool won = false;
-        if (!test_bit(V, v)) won = claim_bit(V, v);
+    __device__ __forceinline__ Probe probe(int, uint32_t, int v) const { return V[v >> 5]; }
+    __device__ __forceinline__ Tok act(int, uint32_t, int v, Probe p) const {
+        unsigned bit = 1u << (v & 31);
+        return ClaimTok{(p & bit) ? ~0u : atomicOr(V + (v >> 5), bit), 0u};
+    }
+    __device__ __forceinline__ Aux aux(int, uint32_t, int v, Tok t) const {
+        bool won = !((t.old >> (v & 31)) & 1u);
+        return won ? make_uint2(__ldg(off + v), __ldg(off + v + 1)) : make_uint2(0u, 0u);
+    }
+    __device__ __forceinline__ bool commit(int, uint32_t, int v, Tok t, Aux d, LocalCnt &c) const {
+        bool won = !((t.old >> (v & 31)) & 1u);
         if (won) {
             depth[v] = lvl1;
-            c.add_vertex(__ldg(off + v + 1) - __ldg(off + v));
+            c.add_vertex(d.y - d.x);
+            if (fused == 2) atomicOr(nfb + (v >> 5), 1u << (v & 31));
         }
-        if (fused) warp_append(nq, nqlen, won, v);
+        if (fused == 1) warp_append(nq, nqlen, won, v);
         return false;
     }
 };
@@ -90,24 +85,106 @@ struct BfsPullOp {
     int lvl;
     bool fused;
     unsigned *nfb;
+    using Probe = unsigned;
+    using Tok = ClaimTok;
+    using Aux = uint2;
     static constexpr bool kEarlyExit = true;
     __device__ __forceinline__ bool skip(int v) const { return test_bit_relaxed(V, v); }
-    __device__ __forceinline__ bool edge(int v, uint32_t, int u, LocalCnt &c) const {
-        bool act = fb ? test_bit(fb, u) : (depth[u] == lvl);
-        if (!act) return false;
-        if (claim_bit(V, v)) {
+    __device__ __forceinline__ Probe probe(int, uint32_t, int u) const {
+        return fb ? fb[u >> 5] : (unsigned)depth[u];
+    }
+    __device__ __forceinline__ Tok act(int v, uint32_t, int u, Probe p) const {
+        bool in = fb ? ((p >> (u & 31)) & 1u) : ((int)p == lvl);
+        return ClaimTok{in ? atomicOr(V + (v >> 5), 1u << (v & 31)) : ~0u, in ? 1u : 0u};
+    }
+    __device__ __forceinline__ Aux aux(int v, uint32_t, int, Tok t) const {
+        bool won = !((t.old >> (v & 31)) & 1u);
+        return won ? make_uint2(__ldg(off + v), __ldg(off + v + 1)) : make_uint2(0u, 0u);
+    }
+    __device__ __forceinline__ bool commit(int v, uint32_t, int, Tok t, Aux d, LocalCnt &c) const {
+        bool won = !((t.old >> (v & 31)) & 1u);
+        if (won) {
             depth[v] = lvl + 1;
-            c.add_vertex(__ldg(off + v + 1) - __ldg(off + v));
+            c.add_vertex(d.y - d.x);
             if (fused) atomicOr(nfb + (v >> 5), 1u << (v & 31));
         }
-        return true;
+        return t.flag != 0u;
     }
 };
 
+// Pull over the visited map with word ownership (the THREAD candidate on the bitmap format):
+// warp w owns 32-vertex words of V, lane = vertex, so claiming needs no atomics -- the warp
+// ballots its hits and stores V[w] | hits and the next-frontier word itself.  Each warp keeps
+// kPullWords words in flight, each lane one independent (col -> frontier-bit) chain per word.
+constexpr int kPullWords = 4;
+__device__ __noinline__ LocalCnt bfs_pull_words(const unsigned *__restrict__ fb, unsigned *__restrict__ V,
+                                                int *__restrict__ depth, const uint32_t *__restrict__ in_off,
+                                                const int32_t *__restrict__ in_col,
+                                                const uint32_t *__restrict__ out_off, bool symmetric, int lvl,
+                                                unsigned *__restrict__ nfb, int n) {
+    LocalCnt cnt;
+    const int W = (n + 31) >> 5;
+    const unsigned lane = lane_id();
+    const long long NW = gwarps();
+    for (long long wb = gwarp(); wb < W; wb += kPullWords * NW) {
+        unsigned vis[kPullWords];
+        uint32_t e[kPullWords], end[kPullWords], beg[kPullWords];
+        bool alive[kPullWords], found[kPullWords];
+#pragma unroll
+        for (int j = 0; j < kPullWords; ++j) {
+            long long w = wb + j * NW;
+            vis[j] = w < W ? V[w] : ~0u;                      // warp-uniform address: one request
+        }
+#pragma unroll
+        for (int j = 0; j < kPullWords; ++j) {
+            int v = (int)((wb + j * NW) * 32 + lane);
+            alive[j] = !((vis[j] >> lane) & 1u);
+            found[j] = false;
+            beg[j] = e[j] = alive[j] ? __ldg(in_off + v) : 0u;
+            end[j] = alive[j] ? __ldg(in_off + v + 1) : 0u;
+            alive[j] = alive[j] && e[j] < end[j];
+        }
+        for (;;) {
+            bool any = false;
+#pragma unroll
+            for (int j = 0; j < kPullWords; ++j) any |= alive[j];
+            if (!__any_sync(0xffffffffu, any)) break;
+            int y[kPullWords];
+            unsigned p[kPullWords];
+#pragma unroll
+            for (int j = 0; j < kPullWords; ++j) y[j] = alive[j] ? __ldg(in_col + e[j]) : 0;
+#pragma unroll
+            for (int j = 0; j < kPullWords; ++j) p[j] = alive[j] ? fb[y[j] >> 5] : 0u;
+#pragma unroll
+            for (int j = 0; j < kPullWords; ++j) {
+                if (!alive[j]) continue;
+                cnt.edges++;
+                if ((p[j] >> (y[j] & 31)) & 1u) { found[j] = true; alive[j] = false; }
+                else if (++e[j] >= end[j]) alive[j] = false;
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < kPullWords; ++j) {
+            long long w = wb + j * NW;
+            unsigned hits = __ballot_sync(0xffffffffu, found[j]);
+            if (hits && lane == 0) {
+                V[w] = vis[j] | hits;
+                if (nfb) nfb[w] = hits;
+            }
+            if (found[j]) {
+                int v = (int)(w * 32 + lane);
+                depth[v] = lvl + 1;
+                cnt.add_vertex(symmetric ? end[j] - beg[j] : __ldg(out_off + v + 1) - __ldg(out_off + v));
+            }
+        }
+    }
+    return cnt;
+}
+
 __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
-    __shared__ TravSmem sm;
+    __shared__ LbSmem sm;
     __shared__ uint32_t red[kWarps + 1];
-    RunCommon &rc = a.rc;
+    const RunCommon &rc = a.rc;
     const GridBarrier bar = make_bar(rc);
     unsigned epoch = 0;
     const int n = a.g.n, W = (n + 31) >> 5, src = a.src;
@@ -122,14 +199,15 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
         a.V[w] = x;
         a.fb[0][w] = 0u; a.fb[1][w] = 0u; a.fb[2][w] = 0u;
     }
-    const unsigned dsrc = a.g.off[src + 1] - a.g.off[src];
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
+    const unsigned dsrc = __ldg(a.g.off + src + 1) - __ldg(a.g.off + src);
+    if (is_book()) {
         for (int i = 0; i < 3; ++i) reset_cnt(rc.cnt + i);
         rc.cnt[0].va = 1; rc.cnt[0].ea = dsrc; rc.cnt[0].maxd = dsrc; rc.cnt[0].mind = dsrc; rc.cnt[0].qlen = 1;
         a.q[0][0] = src;
     }
     grid_sync(bar, epoch);
 
+    Book book;
     long long Via = (long long)n - 1, Eia = (long long)a.g.nnz - dsrc;
     int mat = MAT_SQUEUE;
     bool dirty[3] = {false, false, false};
@@ -138,44 +216,42 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
     long long prev_va = 0, prev_via = 0;
     int t = 0;
     for (;; ++t) {
-        stamp_iteration_start(rc, t);
         IterCnt *cur = rc.cnt + (t % 3), *nxt = rc.cnt + ((t + 1) % 3);
-        unsigned long long va, ea, edges_prev;
-        unsigned maxd, mind, qlen;
-        read_cnt(cur, va, ea, maxd, mind, qlen, edges_prev);
-        if (blockIdx.x == 0 && threadIdx.x == 0 && t > 0) {
+        if (is_book()) book_start(book, rc, t, nxt);
+        const CntView cv = cta_read_cnt(cur);       // one L2 round trip per CTA per iteration
+        const unsigned long long va = cv.va, ea = cv.ea;
+        if (is_book() && t > 0) {
             // algorithmic bytes of iteration t-1 (DESIGN.md roofline model D0)
-            unsigned long long b = prev_dir == GSW_PUSH
-                ? 12ull * prev_va + 4ull * edges_prev + 8ull * va
+            book.bytes += prev_dir == GSW_PUSH
+                ? 12ull * prev_va + 4ull * cv.edges + 8ull * va
                 : (unsigned long long)n / 4 + 8ull * (unsigned long long)max(0LL, prev_via - a.iso_count) +
-                      4ull * edges_prev + 4ull * va;
-            rc.ctl->bytes_alg += b;
-            rc.ctl->edges_total += edges_prev;
-            if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)edges_prev;
+                      4ull * cv.edges + 4ull * va;
+            book.edges += cv.edges;
+            if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)cv.edges;
         }
         if (va == 0) break;
         if (t > 0) { Via -= (long long)va; Eia -= (long long)ea; }
         f.Va = (long long)va; f.Ea = (long long)ea; f.Via = Via; f.Eia = Eia;
-        f.maxd = maxd; f.mind = mind; f.iter = t;
-        read_hist(rc, t, f);
-        DevCfg c = select_traversal(f, rc.force);
+        f.maxd = cv.maxd; f.mind = cv.mind; f.iter = t;
+        hist_features(cv, f);
+        const DevCfg c = select_traversal(f, rc.force);
         write_record(rc, t, c, f, 0u);
-        if (blockIdx.x == 0 && threadIdx.x == 0) reset_cnt(rc.cnt + ((t + 2) % 3));
+        if (is_book()) reset_cnt(rc.cnt + ((t + 2) % 3));
         const int b2 = (t + 2) % 3;
         if (dirty[b2]) { clear_words(a.fb[b2], W); dirty[b2] = false; }
 
-        // ---------------- Filter
+        // ---------------- Filter: materialise AS_t in the selected format
         const bool push = c.dir == GSW_PUSH;
         int need;
         if (push) need = c.fmt == GSW_BITMAP ? MAT_BITMAP : (c.fmt == GSW_QUEUE ? MAT_QUEUE : MAT_SQUEUE);
         else need = c.fmt == GSW_BITMAP ? MAT_BITMAP : MAT_NONE;
         int *qa = a.q[t & 1];
         unsigned *fbt = a.fb[t % 3];
-        bool filtered = false;
+        bool filtered = false, qlen_changed = false;
         const int lvl = t;
         auto is_active = [&](int v) { return depth[v] == lvl; };
         if (need == MAT_BITMAP && mat != MAT_BITMAP) {
-            if (mat == MAT_QUEUE || mat == MAT_SQUEUE) bm_from_q(fbt, qa, qlen);
+            if (mat == MAT_QUEUE || mat == MAT_SQUEUE) bm_from_q(fbt, qa, cv.qlen);
             else bm_from_pred(fbt, n, is_active);
             dirty[t % 3] = true;
             mat = MAT_BITMAP;
@@ -184,10 +260,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
             if (mat == MAT_BITMAP) q_from_bm(qa, &cur->qlen, fbt, W, 0u);
             else q_from_pred(qa, &cur->qlen, n, is_active);
             mat = MAT_QUEUE;
-            filtered = true;
+            filtered = qlen_changed = true;
         } else if (need == MAT_SQUEUE && mat != MAT_SQUEUE) {
             if (mat != MAT_BITMAP) {
-                if (mat == MAT_QUEUE) bm_from_q(fbt, qa, qlen);
+                if (mat == MAT_QUEUE) bm_from_q(fbt, qa, cv.qlen);
                 else bm_from_pred(fbt, n, is_active);
                 dirty[t % 3] = true;
                 grid_sync(bar, epoch);
@@ -196,7 +272,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
             grid_sync(bar, epoch);
             sq_from_bm_p2(qa, &cur->qlen, fbt, W, 0u, rc.partial, red);
             mat = MAT_SQUEUE;
-            filtered = true;
+            filtered = qlen_changed = true;
         }
         if (!push && c.fmt != GSW_BITMAP) {               // inactive workload as a queue
             if (c.fmt == GSW_QUEUE) {
@@ -209,39 +285,48 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
             filtered = true;
         }
         if (filtered) grid_sync(bar, epoch);
-        stamp_expand_start(rc);
+        if (is_book()) book_expand(book);
 
         // ---------------- Expand
         LocalCnt lc;
         const bool fused = c.fused == GSW_FUSED;
+        // fused push writes the next active set directly ("write u to AS directly"):
+        // as a warp-aggregated queue append when the claims are few, as bitmap marking (the
+        // paper's duplicate-tolerant technique) when a single queue counter would be
+        // the contended address
+        const bool mark_bitmap = (long long)ea > (long long)(n >> 6);
+        const bool next_bitmap = !push || mark_bitmap;
         if (push) {
-            BfsPushOp op{depth, a.V, a.g.off, t + 1, fused, a.q[(t + 1) & 1], &nxt->qlen};
+            const BfsPushOp op{depth, a.V, a.g.off, t + 1, fused ? (mark_bitmap ? 2 : 1) : 0, a.q[(t + 1) & 1],
+                               &nxt->qlen, a.fb[(t + 1) % 3]};
+            if (fused && mark_bitmap) dirty[(t + 1) % 3] = true;
             if (mat == MAT_BITMAP) {
-                BitmapSrc s{fbt, (unsigned)n, 1u};
-                run_lb(c.lb, s, adj_out, op, lc, sm, red, bar, epoch, rc.partial, a.scan);
+                lc = run_lb(c.lb, BitmapSrc{fbt, (unsigned)n, 1u}, adj_out, op, sm, red, bar, epoch, rc.partial, a.scan);
             } else {
-                QueueSrc s{qa, ld_relaxed(&cur->qlen)};
-                run_lb(c.lb, s, adj_out, op, lc, sm, red, bar, epoch, rc.partial, a.scan);
+                const unsigned ql = qlen_changed ? cta_read_u32(&cur->qlen) : cv.qlen;
+                lc = run_lb(c.lb, QueueSrc{qa, ql}, adj_out, op, sm, red, bar, epoch, rc.partial, a.scan);
             }
         } else {
-            BfsPullOp op{depth, a.V, a.g.off, c.fmt == GSW_BITMAP ? fbt : nullptr, t, fused, a.fb[(t + 1) % 3]};
-            if (c.fmt == GSW_BITMAP) {
-                BitmapSrc s{a.V, (unsigned)n, 0u};
-                run_lb(c.lb, s, adj_in, op, lc, sm, red, bar, epoch, rc.partial, a.scan);
+            const BfsPullOp op{depth, a.V, a.g.off, c.fmt == GSW_BITMAP ? fbt : nullptr, t, fused, a.fb[(t + 1) % 3]};
+            if (c.fmt == GSW_BITMAP && c.lb == GSW_LB_THREAD) {
+                lc = bfs_pull_words(fbt, a.V, depth, a.g.in_off, a.g.in_col, a.g.off, a.g.in_off == a.g.off, t,
+                                    fused ? a.fb[(t + 1) % 3] : nullptr, n);
+            } else if (c.fmt == GSW_BITMAP) {
+                lc = run_lb(c.lb, BitmapSrc{a.V, (unsigned)n, 0u}, adj_in, op, sm, red, bar, epoch, rc.partial, a.scan);
             } else {
-                QueueSrc s{a.iq, ld_relaxed(&cur->iqlen)};
-                run_lb(c.lb, s, adj_in, op, lc, sm, red, bar, epoch, rc.partial, a.scan);
+                lc = run_lb(c.lb, QueueSrc{a.iq, cta_read_u32(&cur->iqlen)}, adj_in, op, sm, red, bar, epoch,
+                            rc.partial, a.scan);
             }
             if (fused) dirty[(t + 1) % 3] = true;
         }
         flush_counts(lc, nxt);
         grid_sync(bar, epoch);
-        mat = fused ? (push ? MAT_QUEUE : MAT_BITMAP) : MAT_NONE;
+        mat = fused ? (next_bitmap ? MAT_BITMAP : MAT_QUEUE) : MAT_NONE;
         prev_dir = c.dir;
         prev_va = (long long)va;
         prev_via = Via;
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) rc.ctl->iters = (unsigned)t;
+    if (is_book()) book_finish(book, rc, t);
 }
 
 gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stats *st) {

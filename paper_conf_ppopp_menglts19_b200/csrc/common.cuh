@@ -5,6 +5,7 @@
 // separated by a software grid barrier (below) instead of kernel boundaries, so there is no host
 // round trip per iteration (the paper's 58-120 us feature copy, disappears).
 #pragma once
+#include <cstddef>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -62,14 +63,15 @@ struct GridBarrier {
 };
 constexpr uint64_t kBarrierTimeoutNs = 20ull * 1000 * 1000 * 1000;
 
+// (tools/micro_barrier.cu on B200: this acq_rel-arrive + release-publish form costs 1.6-1.9 us at
+// 148-592 CTAs; the fence-heavy form 1.9-2.4 us.)
 __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch) {
     __syncthreads();
     if (threadIdx.x == 0) {
         unsigned target = epoch + 1;
-        __threadfence();
-        unsigned prev = atomicAdd(b.arrive, 1u);
+        unsigned prev;
+        asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(prev) : "l"(b.arrive) : "memory");
         if (prev == target * gridDim.x - 1) {
-            __threadfence();
             st_release(b.gen, target);
         } else {
             uint64_t t0 = globaltimer();
@@ -183,12 +185,61 @@ __device__ __forceinline__ void warp_append(int *q, unsigned *len, bool pred, in
 // ------------------------------------------------------------------ per-iteration counters
 // Runtime characteristics of the NEXT active set, accumulated by whoever activates a vertex
 // (Table 1): Va, Ea, max/min degree; plus edges scanned by this iteration's Expand.
-struct IterCnt {
+struct alignas(128) IterCnt {
     unsigned long long va, ea, edges;
     unsigned maxd, mind;
     unsigned qlen;          // length of the queue materialised for this active set (if any)
     unsigned iqlen;         // length of the inactive (pull workload) queue, if built
+    float tf, te, Tf, Te;   // history features carried to the iteration that reads this slot
 };
+
+// After a grid barrier every CTA needs the same few control words.  Reading them from every warp
+// of ~600 CTAs serialises ~20K requests on one L2 line (~10 us/iteration measured on B200); instead
+// thread 0 of each CTA reads once and broadcasts through shared memory.
+struct CntView {
+    unsigned long long va, ea, edges;
+    unsigned maxd, mind, qlen, iqlen;
+    float tf, te, Tf, Te;
+};
+__device__ __forceinline__ unsigned long long ld_relaxed64_nc(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ unsigned ld_relaxed_nc(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ CntView cta_read_cnt(const IterCnt *c) {
+    __shared__ CntView s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        // Plain (vectorisable, pipelined) loads: this always follows a grid barrier whose acquire
+        // invalidated this SM's L1 (CCTL.IVALL), so they observe every write released before it.
+        // (11 separate ld.relaxed.gpu here cost ~5 us per iteration.)
+        const uint4 *p = reinterpret_cast<const uint4 *>(c);
+        uint4 a = p[0], b = p[1], d = p[2], e = p[3];
+        CntView v;
+        v.va = ((unsigned long long)a.y << 32) | a.x;
+        v.ea = ((unsigned long long)a.w << 32) | a.z;
+        v.edges = ((unsigned long long)b.y << 32) | b.x;
+        v.maxd = b.z; v.mind = b.w;
+        v.qlen = d.x; v.iqlen = d.y;
+        v.tf = __uint_as_float(d.z); v.te = __uint_as_float(d.w);
+        v.Tf = __uint_as_float(e.x); v.Te = __uint_as_float(e.y);
+        s = v;
+    }
+    __syncthreads();
+    return s;
+}
+__device__ __forceinline__ unsigned cta_read_u32(const unsigned *p) {
+    __shared__ unsigned s;
+    __syncthreads();
+    if (threadIdx.x == 0) s = *(volatile const unsigned *)p;
+    __syncthreads();
+    return s;
+}
 
 struct LocalCnt {
     unsigned long long va = 0, ea = 0, edges = 0;
@@ -225,6 +276,7 @@ __device__ __forceinline__ void flush_counts(LocalCnt &c, IterCnt *dst) {
 
 __device__ __forceinline__ void reset_cnt(IterCnt *c) {
     c->va = 0; c->ea = 0; c->edges = 0; c->maxd = 0; c->mind = 0xffffffffu; c->qlen = 0; c->iqlen = 0;
+    c->tf = 0.f; c->te = 0.f; c->Tf = 0.f; c->Te = 0.f;
 }
 
 // grid-stride helpers
@@ -233,4 +285,10 @@ __device__ __forceinline__ long long gthreads() { return (long long)gridDim.x * 
 __device__ __forceinline__ long long gwarp() { return gtid() >> 5; }
 __device__ __forceinline__ long long gwarps() { return gthreads() >> 5; }
 
+}  // namespace gsw
+
+namespace gsw {
+static_assert(offsetof(IterCnt, va) == 0 && offsetof(IterCnt, edges) == 16 && offsetof(IterCnt, maxd) == 24 &&
+                  offsetof(IterCnt, qlen) == 32 && offsetof(IterCnt, tf) == 40 && offsetof(IterCnt, Tf) == 48,
+              "cta_read_cnt assumes this layout");
 }  // namespace gsw

@@ -39,46 +39,38 @@ __device__ __forceinline__ GridBarrier make_bar(const RunCommon &rc) {
     return GridBarrier{&rc.ctl->arrive, &rc.ctl->gen, &rc.ctl->err};
 }
 
-__device__ __forceinline__ void read_cnt(const IterCnt *c, unsigned long long &va, unsigned long long &ea,
-                                         unsigned &maxd, unsigned &mind, unsigned &qlen, unsigned long long &edges) {
-    va = ld_relaxed64(&c->va);
-    ea = ld_relaxed64(&c->ea);
-    edges = ld_relaxed64(&c->edges);
-    maxd = ld_relaxed(&c->maxd);
-    mind = ld_relaxed(&c->mind);
-    qlen = ld_relaxed(&c->qlen);
-}
+// Per-run bookkeeping of CTA 0 / thread 0, kept in registers so that nothing on the critical
+// path between two grid barriers waits for a global read-modify-write.
+struct Book {
+    uint64_t t_start = 0, t_expand = 0;
+    float sum_tf = 0.f, sum_te = 0.f;
+    unsigned long long bytes = 0, edges = 0;
+};
+__device__ __forceinline__ bool is_book() { return blockIdx.x == 0 && threadIdx.x == 0; }
 
-// History features of iteration t-2 (written by CTA 0 two barriers ago) -> identical in all CTAs.
-__device__ __forceinline__ void read_hist(const RunCommon &rc, int t, Features &f) {
-    f.tf = f.te = f.Tf = f.Te = 0.f;
-    if (t >= 2 && t - 2 < kMaxHist) {
-        volatile const Hist *h = rc.hist + (t - 2);
-        f.tf = h->tf; f.te = h->te; f.Tf = h->Tf; f.Te = h->Te;
+// Start of iteration t (CTA 0 / thread 0): close the timing of iteration t-1 (Filter = start ->
+// expand stamp, Expand = expand stamp -> now) and publish it as history features through the
+// counter slot `carry` that every CTA reads at iteration t+1 (lag 2, identical in all CTAs).
+__device__ __forceinline__ void book_start(Book &b, const RunCommon &rc, int t, IterCnt *carry) {
+    uint64_t now = globaltimer();
+    if (t >= 1) {
+        float tf = (float)(b.t_expand - b.t_start) * 1e-3f;
+        float te = (float)(now - b.t_expand) * 1e-3f;
+        b.sum_tf += tf; b.sum_te += te;
+        carry->tf = tf; carry->te = te; carry->Tf = b.sum_tf / (float)t; carry->Te = b.sum_te / (float)t;
+        if (t - 1 < kMaxHist) { rc.rec[t - 1].filter_us = tf; rc.rec[t - 1].expand_us = te; }
     }
+    b.t_start = now;
+    b.t_expand = now;
 }
-
-// CTA 0 / thread 0 bookkeeping at the start of iteration t (after the barrier that ended t-1).
-__device__ __forceinline__ void stamp_iteration_start(const RunCommon &rc, int t) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        Ctl *c = rc.ctl;
-        uint64_t now = globaltimer();
-        if (t >= 1) {
-            float tf = (float)(c->t_expand - c->t_start) * 1e-3f;
-            float te = (float)(now - c->t_expand) * 1e-3f;
-            c->sum_tf += tf; c->sum_te += te;
-            if (t - 1 < kMaxHist) {
-                rc.hist[t - 1] = Hist{tf, te, c->sum_tf / t, c->sum_te / t};
-                rc.rec[t - 1].filter_us = tf;
-                rc.rec[t - 1].expand_us = te;
-            }
-        }
-        c->t_start = now;
-        c->t_expand = now;
-    }
+__device__ __forceinline__ void book_expand(Book &b) { b.t_expand = globaltimer(); }
+__device__ __forceinline__ void book_finish(const Book &b, const RunCommon &rc, int iters) {
+    rc.ctl->bytes_alg = b.bytes;
+    rc.ctl->edges_total = b.edges;
+    rc.ctl->iters = (unsigned)iters;
 }
-__device__ __forceinline__ void stamp_expand_start(const RunCommon &rc) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) rc.ctl->t_expand = globaltimer();
+__device__ __forceinline__ void hist_features(const CntView &v, Features &f) {
+    f.tf = v.tf; f.te = v.te; f.Tf = v.Tf; f.Te = v.Te;
 }
 
 __device__ __forceinline__ void write_record(const RunCommon &rc, int t, const DevCfg &c, const Features &f,

@@ -2,20 +2,26 @@
 // Expand is mapped onto threads.  Every strategy is a device function used inside a persistent
 // kernel phase, templated on
 //   Src : the active set in its format (Pattern 2): size() item slots, get(i) -> vertex or -1
-//   Op  : the algorithm's per-edge operation (emit + comp/compAtomic)
-//         bool skip(int x)                      -- x needs no (more) work (pull early exit)
-//         bool edge(int x, uint32 e, int y, LocalCnt&) -- process edge e=(x,y); true = x done
-//         static constexpr bool kEarlyExit       -- stop scanning x after edge() returned true
+//   Op  : the algorithm's per-edge operation (emit + comp/compAtomic), split in two
+//         so that several edges' loads are in flight per thread (memory-level parallelism):
+//           bool  skip(int x)                          x needs no (more) work (pull early exit)
+//           Probe probe(int x, uint32 e, int y)        the dependent load(s) of edge e=(x,y)
+//           bool  apply(int x, uint32 e, int y, Probe, LocalCnt&)  update; true = x done
+//           static constexpr bool kEarlyExit           stop scanning x once apply returned true
 // Candidates:
-//   THREAD : one thread per item, serial edge loop (the naive mapping the north_star lists)
+//   THREAD : one thread per item, serial edge loop (the naive mapping the north_star lists);
+//            kIlp independent items per thread are advanced in lock-step
 //   TWC    : degree-binned thread / warp / CTA mapping (B40C [41])
 //   WM     : a warp takes 32 consecutive items, 32-edge chunks, log2(32)-step search
 //   CM     : a CTA takes blockDim items, blockDim-edge chunks, log2(blockDim) search
 //   STRICT : equal (items+edges) per tile via merge-path over the degree scan ([13])
 #pragma once
 #include "common.cuh"
+#include "gsw.h"
 
 namespace gsw {
+
+constexpr int kIlp = 4;
 
 struct QueueSrc {
     const int *q;
@@ -46,86 +52,160 @@ struct Adj {
     const int32_t *col;
 };
 
+// Process up to K edges (x[j], e[j]) (valid when ok[j]) in five stages, each issued for all K
+// edges before the next consumes its results, so a thread keeps K independent memory chains in
+// flight instead of waiting on one dependent round trip per edge:
+//   1 y   = col[e]                       (adjacency load)
+//   2 p   = op.probe(x, e, y)            (status load of the other endpoint)
+//   3 tok = op.act(x, e, y, p)           (decision; may issue an atomic whose result is in tok)
+//   4 aux = op.aux(x, e, y, tok)         (loads needed only by winners, e.g. a degree)
+//   5 stop = op.commit(x, e, y, tok, aux, cnt)   (plain stores, counters; true = x done)
+template <int K, class Op>
+__device__ __forceinline__ void edge_batch(const Op &op, const Adj &g, const int (&x)[K], const uint32_t (&e)[K],
+                                           const bool (&ok)[K], bool (&stop)[K], LocalCnt &cnt) {
+    int y[K];
+    typename Op::Probe p[K];
+    typename Op::Tok tk[K];
+    typename Op::Aux ax[K];
+#pragma unroll
+    for (int j = 0; j < K; ++j) y[j] = ok[j] ? __ldg(g.col + e[j]) : 0;
+#pragma unroll
+    for (int j = 0; j < K; ++j) if (ok[j]) p[j] = op.probe(x[j], e[j], y[j]);
+#pragma unroll
+    for (int j = 0; j < K; ++j) if (ok[j]) tk[j] = op.act(x[j], e[j], y[j], p[j]);
+#pragma unroll
+    for (int j = 0; j < K; ++j) if (ok[j]) ax[j] = op.aux(x[j], e[j], y[j], tk[j]);
+#pragma unroll
+    for (int j = 0; j < K; ++j) {
+        stop[j] = false;
+        if (ok[j]) { cnt.edges++; stop[j] = op.commit(x[j], e[j], y[j], tk[j], ax[j], cnt); }
+    }
+}
+
 // ------------------------------------------------------------------ THREAD
 template <class Src, class Op>
-__device__ void lb_thread(const Src &src, const Adj &g, Op &op, LocalCnt &cnt) {
-    unsigned sz = src.size();
-    for (long long i = gtid(); i < sz; i += gthreads()) {
-        int x = src.get((unsigned)i);
-        if (x < 0 || op.skip(x)) continue;
-        uint32_t b = __ldg(g.off + x), e = __ldg(g.off + x + 1);
-        for (uint32_t k = b; k < e; ++k) {
-            cnt.edges++;
-            if (op.edge(x, k, __ldg(g.col + k), cnt) && Op::kEarlyExit) break;
+__device__ __noinline__ LocalCnt lb_thread(const Src src, const Adj g, Op op) {
+    LocalCnt cnt;
+    const unsigned sz = src.size();
+    const long long T = gthreads();
+    for (long long base = gtid(); base < sz; base += kIlp * T) {
+        int x[kIlp];
+        uint32_t e[kIlp], end[kIlp];
+#pragma unroll
+        for (int j = 0; j < kIlp; ++j) {
+            long long i = base + j * T;
+            int v = i < sz ? src.get((unsigned)i) : -1;
+            if (v >= 0 && op.skip(v)) v = -1;
+            x[j] = v;
+        }
+#pragma unroll
+        for (int j = 0; j < kIlp; ++j) {
+            e[j] = x[j] >= 0 ? __ldg(g.off + x[j]) : 0u;
+            end[j] = x[j] >= 0 ? __ldg(g.off + x[j] + 1) : 0u;
+        }
+        for (;;) {
+            bool ok[kIlp], stop[kIlp], any = false;
+#pragma unroll
+            for (int j = 0; j < kIlp; ++j) { ok[j] = e[j] < end[j]; any |= ok[j]; }
+            if (!any) break;
+            edge_batch<kIlp>(op, g, x, e, ok, stop, cnt);
+#pragma unroll
+            for (int j = 0; j < kIlp; ++j)
+                if (ok[j]) e[j] = (Op::kEarlyExit && stop[j]) ? end[j] : e[j] + 1;
         }
     }
+    return cnt;
 }
 
 // ------------------------------------------------------------------ TWC
 struct TwcSmem {
-    int owner, x, stop;
+    int owner, x;
     uint32_t b, e;
 };
 template <class Src, class Op>
-__device__ void lb_twc(const Src &src, const Adj &g, Op &op, LocalCnt &cnt, TwcSmem *sm) {
-    unsigned sz = src.size();
+__device__ __noinline__ LocalCnt lb_twc(const Src src, const Adj g, Op op, TwcSmem *sm) {
+    LocalCnt cnt;
+    const unsigned sz = src.size();
     const unsigned lane = lane_id();
-    for (long long base = (long long)blockIdx.x * kBlock; base < sz; base += (long long)gridDim.x * kBlock) {
-        long long i = base + threadIdx.x;
-        int x = i < sz ? src.get((unsigned)i) : -1;
-        if (x >= 0 && op.skip(x)) x = -1;
-        uint32_t b = 0, e = 0;
-        if (x >= 0) { b = __ldg(g.off + x); e = __ldg(g.off + x + 1); }
-        uint32_t d = e - b;
+    constexpr int kTile = kBlock * kIlp;
+    for (long long base = (long long)blockIdx.x * kTile; base < sz; base += (long long)gridDim.x * kTile) {
+        int x[kIlp];
+        uint32_t b[kIlp], e[kIlp];
+#pragma unroll
+        for (int j = 0; j < kIlp; ++j) {
+            long long i = base + j * kBlock + threadIdx.x;
+            int v = i < sz ? src.get((unsigned)i) : -1;
+            if (v >= 0 && op.skip(v)) v = -1;
+            x[j] = v;
+        }
+#pragma unroll
+        for (int j = 0; j < kIlp; ++j) {
+            b[j] = x[j] >= 0 ? __ldg(g.off + x[j]) : 0u;
+            e[j] = x[j] >= 0 ? __ldg(g.off + x[j] + 1) : 0u;
+        }
         // CTA tier: degree >= blockDim
-        for (;;) {
-            if (threadIdx.x == 0) sm->owner = -1;
-            __syncthreads();
-            if (d >= (uint32_t)kBlock) sm->owner = threadIdx.x;
-            __syncthreads();
-            int owner = sm->owner;
-            if (owner < 0) break;
-            if ((int)threadIdx.x == owner) { sm->x = x; sm->b = b; sm->e = e; d = 0; }
-            __syncthreads();
-            int xx = sm->x;
-            uint32_t bb = sm->b, ee = sm->e;
-            for (uint32_t k0 = bb; k0 < ee; k0 += kBlock) {
-                uint32_t k = k0 + threadIdx.x;
-                bool stop = false;
-                if (k < ee) { cnt.edges++; stop = op.edge(xx, k, __ldg(g.col + k), cnt); }
-                if (Op::kEarlyExit) { if (__syncthreads_or(stop)) break; }
+#pragma unroll
+        for (int j = 0; j < kIlp; ++j) {
+            for (;;) {
+                if (threadIdx.x == 0) sm->owner = -1;
+                __syncthreads();
+                if (e[j] - b[j] >= (uint32_t)kBlock) sm->owner = threadIdx.x;
+                __syncthreads();
+                int owner = sm->owner;
+                if (owner < 0) break;
+                if ((int)threadIdx.x == owner) { sm->x = x[j]; sm->b = b[j]; sm->e = e[j]; e[j] = b[j]; }
+                __syncthreads();
+                const int xx = sm->x;
+                const uint32_t bb = sm->b, ee = sm->e;
+                for (uint32_t k0 = bb; k0 < ee; k0 += 2 * kBlock) {
+                    int xs[2] = {xx, xx};
+                    uint32_t ks[2] = {k0 + threadIdx.x, k0 + kBlock + threadIdx.x};
+                    bool ok[2] = {ks[0] < ee, ks[1] < ee}, stop[2];
+                    edge_batch<2>(op, g, xs, ks, ok, stop, cnt);
+                    if (Op::kEarlyExit) { if (__syncthreads_or(stop[0] | stop[1])) break; }
+                }
+                __syncthreads();
             }
-            __syncthreads();
         }
         // warp tier: 32 <= degree < blockDim
-        for (;;) {
-            unsigned m = __ballot_sync(0xffffffffu, d >= 32u);
-            if (!m) break;
-            int leader = __ffs(m) - 1;
-            int xx = __shfl_sync(0xffffffffu, x, leader);
-            uint32_t bb = __shfl_sync(0xffffffffu, b, leader), ee = __shfl_sync(0xffffffffu, e, leader);
-            if ((int)lane == leader) d = 0;
-            for (uint32_t k0 = bb; k0 < ee; k0 += 32) {
-                uint32_t k = k0 + lane;
-                bool stop = false;
-                if (k < ee) { cnt.edges++; stop = op.edge(xx, k, __ldg(g.col + k), cnt); }
-                if (Op::kEarlyExit) { if (__any_sync(0xffffffffu, stop)) break; }
+#pragma unroll
+        for (int j = 0; j < kIlp; ++j) {
+            for (;;) {
+                unsigned m = __ballot_sync(0xffffffffu, e[j] - b[j] >= 32u);
+                if (!m) break;
+                int leader = __ffs(m) - 1;
+                const int xx = __shfl_sync(0xffffffffu, x[j], leader);
+                const uint32_t bb = __shfl_sync(0xffffffffu, b[j], leader), ee = __shfl_sync(0xffffffffu, e[j], leader);
+                if ((int)lane == leader) e[j] = b[j];
+                for (uint32_t k0 = bb; k0 < ee; k0 += 64) {
+                    int xs[2] = {xx, xx};
+                    uint32_t ks[2] = {k0 + lane, k0 + 32 + lane};
+                    bool ok[2] = {ks[0] < ee, ks[1] < ee}, stop[2];
+                    edge_batch<2>(op, g, xs, ks, ok, stop, cnt);
+                    if (Op::kEarlyExit) { if (__any_sync(0xffffffffu, stop[0] | stop[1])) break; }
+                }
             }
         }
-        // thread tier: degree < 32
-        if (d > 0) {
-            for (uint32_t k = b; k < e; ++k) {
-                cnt.edges++;
-                if (op.edge(x, k, __ldg(g.col + k), cnt) && Op::kEarlyExit) break;
-            }
+        // thread tier: degree < 32, kIlp items advanced in lock-step
+        for (;;) {
+            bool ok[kIlp], stop[kIlp], any = false;
+#pragma unroll
+            for (int j = 0; j < kIlp; ++j) { ok[j] = b[j] < e[j]; any |= ok[j]; }
+            if (!any) break;
+            edge_batch<kIlp>(op, g, x, b, ok, stop, cnt);
+#pragma unroll
+            for (int j = 0; j < kIlp; ++j)
+                if (ok[j]) b[j] = (Op::kEarlyExit && stop[j]) ? e[j] : b[j] + 1;
         }
     }
+    return cnt;
 }
 
 // ------------------------------------------------------------------ WM
 template <class Src, class Op>
-__device__ void lb_wm(const Src &src, const Adj &g, Op &op, LocalCnt &cnt) {
-    unsigned sz = src.size();
+__device__ __noinline__ LocalCnt lb_wm(const Src src, const Adj g, Op op) {
+    LocalCnt cnt;
+    const unsigned sz = src.size();
     const unsigned lane = lane_id();
     for (long long wb = gwarp() * 32; wb < sz; wb += gwarps() * 32) {
         long long i = wb + lane;
@@ -133,28 +213,33 @@ __device__ void lb_wm(const Src &src, const Adj &g, Op &op, LocalCnt &cnt) {
         if (x >= 0 && op.skip(x)) x = -1;
         uint32_t b = 0, d = 0;
         if (x >= 0) { b = __ldg(g.off + x); d = __ldg(g.off + x + 1) - b; }
-        uint32_t incl = warp_incl_scan(d);
-        uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-        uint32_t excl = incl - d;
-        for (uint32_t k0 = 0; k0 < total; k0 += 32) {
-            uint32_t k = k0 + lane;
-            // owner lane j: first lane with incl_j > k  (binary search, log2(32) = 5 steps)
-            unsigned lo = 0, hi = 31;
+        const uint32_t incl = warp_incl_scan(d);
+        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+        const uint32_t excl = incl - d;
+        for (uint32_t k0 = 0; k0 < total; k0 += 64) {
+            int xs[2];
+            uint32_t es[2];
+            bool ok[2], stop[2];
 #pragma unroll
-            for (int s = 0; s < 5; ++s) {
-                unsigned mid = (lo + hi) >> 1;
-                uint32_t v = __shfl_sync(0xffffffffu, incl, mid);
-                if (v > k) hi = mid; else lo = mid + 1;
+            for (int h = 0; h < 2; ++h) {
+                uint32_t k = k0 + 32 * h + lane;
+                // owner lane: first lane with incl > k  (log2(32) = 5 steps)
+                unsigned lo = 0, hi = 31;
+#pragma unroll
+                for (int s = 0; s < 5; ++s) {
+                    unsigned mid = (lo + hi) >> 1;
+                    uint32_t v = __shfl_sync(0xffffffffu, incl, mid);
+                    if (v > k) hi = mid; else lo = mid + 1;
+                }
+                xs[h] = __shfl_sync(0xffffffffu, x, lo);
+                uint32_t bb = __shfl_sync(0xffffffffu, b, lo), ex = __shfl_sync(0xffffffffu, excl, lo);
+                es[h] = bb + (k - ex);
+                ok[h] = k < total && !(Op::kEarlyExit && op.skip(xs[h]));
             }
-            int xx = __shfl_sync(0xffffffffu, x, lo);
-            uint32_t bb = __shfl_sync(0xffffffffu, b, lo), ex = __shfl_sync(0xffffffffu, excl, lo);
-            if (k < total && !op.skip(xx)) {
-                uint32_t e = bb + (k - ex);
-                cnt.edges++;
-                op.edge(xx, e, __ldg(g.col + e), cnt);
-            }
+            edge_batch<2>(op, g, xs, es, ok, stop, cnt);
         }
     }
+    return cnt;
 }
 
 // ------------------------------------------------------------------ CM
@@ -165,8 +250,9 @@ struct CmSmem {
     uint32_t scan_tmp[kWarps + 1];
 };
 template <class Src, class Op>
-__device__ void lb_cm(const Src &src, const Adj &g, Op &op, LocalCnt &cnt, CmSmem *sm) {
-    unsigned sz = src.size();
+__device__ __noinline__ LocalCnt lb_cm(const Src src, const Adj g, Op op, CmSmem *sm) {
+    LocalCnt cnt;
+    const unsigned sz = src.size();
     for (long long cb = (long long)blockIdx.x * kBlock; cb < sz; cb += (long long)gridDim.x * kBlock) {
         long long i = cb + threadIdx.x;
         int x = i < sz ? src.get((unsigned)i) : -1;
@@ -179,25 +265,32 @@ __device__ void lb_cm(const Src &src, const Adj &g, Op &op, LocalCnt &cnt, CmSme
         sm->beg[threadIdx.x] = b;
         sm->x[threadIdx.x] = x;
         __syncthreads();
-        for (uint32_t k0 = 0; k0 < total; k0 += kBlock) {
-            uint32_t k = k0 + threadIdx.x;
-            if (k < total) {
-                // last item j with excl_j <= k  (log2(blockDim) steps)
-                unsigned lo = 0, hi = kBlock - 1;
-                while (lo < hi) {
-                    unsigned mid = (lo + hi + 1) >> 1;
-                    if (sm->excl[mid] <= k) lo = mid; else hi = mid - 1;
-                }
-                int xx = sm->x[lo];
-                if (!op.skip(xx)) {
-                    uint32_t e = sm->beg[lo] + (k - sm->excl[lo]);
-                    cnt.edges++;
-                    op.edge(xx, e, __ldg(g.col + e), cnt);
+        for (uint32_t k0 = 0; k0 < total; k0 += 2 * kBlock) {
+            int xs[2];
+            uint32_t es[2];
+            bool ok[2], stop[2];
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                uint32_t k = k0 + h * kBlock + threadIdx.x;
+                ok[h] = k < total;
+                xs[h] = -1; es[h] = 0;
+                if (ok[h]) {
+                    // last item j with excl_j <= k  (log2(blockDim) steps)
+                    unsigned lo = 0, hi = kBlock - 1;
+                    while (lo < hi) {
+                        unsigned mid = (lo + hi + 1) >> 1;
+                        if (sm->excl[mid] <= k) lo = mid; else hi = mid - 1;
+                    }
+                    xs[h] = sm->x[lo];
+                    es[h] = sm->beg[lo] + (k - sm->excl[lo]);
+                    ok[h] = !(Op::kEarlyExit && op.skip(xs[h]));
                 }
             }
+            edge_batch<2>(op, g, xs, es, ok, stop, cnt);
         }
         __syncthreads();
     }
+    return cnt;
 }
 
 // ------------------------------------------------------------------ STRICT (merge path)
@@ -266,20 +359,23 @@ __device__ __forceinline__ unsigned merge_path(const uint32_t *scan, unsigned sz
     return (unsigned)lo;
 }
 
-// phase 3: process tiles of kStrictTile diagonals; every tile gets an equal share of items+edges
+// phase 3: process tiles of kStrictTile diagonals; every tile gets an equal share of items+edges.
+// Each thread walks kStrictVT consecutive diagonals in shared memory first, then issues all of
+// their edge loads together.
 template <class Src, class Op>
-__device__ void lb_strict(const Src &src, const Adj &g, Op &op, LocalCnt &cnt, const uint32_t *scan,
+__device__ __noinline__ LocalCnt lb_strict(const Src src, const Adj g, Op op, const uint32_t *scan,
                           uint32_t total, StrictSmem *sm) {
-    unsigned sz = src.size();
-    unsigned long long D = (unsigned long long)sz + total;
-    unsigned long long ntiles = (D + kStrictTile - 1) / kStrictTile;
+    LocalCnt cnt;
+    const unsigned sz = src.size();
+    const unsigned long long D = (unsigned long long)sz + total;
+    const unsigned long long ntiles = (D + kStrictTile - 1) / kStrictTile;
     for (unsigned long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        unsigned long long d0 = t * kStrictTile, d1 = min(D, d0 + kStrictTile);
+        const unsigned long long d0 = t * kStrictTile, d1 = min(D, d0 + kStrictTile);
         if (threadIdx.x == 0) sm->i0 = merge_path(scan, sz, total, d0);
         if (threadIdx.x == 32) sm->i1 = merge_path(scan, sz, total, d1);
         __syncthreads();
-        int i0 = sm->i0, i1 = sm->i1;
-        int ni = min(i1 + 1, (int)sz) - i0;              // items touched by this tile
+        const int i0 = sm->i0, i1 = sm->i1;
+        const int ni = min(i1 + 1, (int)sz) - i0;              // items touched by this tile
         for (int j = threadIdx.x; j <= ni; j += kBlock) sm->scan[j] = scan[i0 + j];
         for (int j = threadIdx.x; j < ni; j += kBlock) {
             int x = src.get(i0 + j);
@@ -288,39 +384,73 @@ __device__ void lb_strict(const Src &src, const Adj &g, Op &op, LocalCnt &cnt, c
             sm->beg[j] = x >= 0 ? __ldg(g.off + x) : 0u;
         }
         __syncthreads();
-        // this thread's diagonals [dd0, dd1) -> local merge path within the tile
-        unsigned long long dd0 = min(d1, d0 + (unsigned long long)threadIdx.x * kStrictVT);
-        unsigned long long dd1 = min(d1, dd0 + kStrictVT);
-        // items consumed at dd0 (search in smem, relative to i0)
-        unsigned long long k_lo = dd0 - i0;                 // not used directly; binary search below
-        (void)k_lo;
-        long long lo = 0, hi = ni;
-        {
-            // global item index i in [i0, i0+ni]; condition scan[i+1] <= dd0-1-i
-            long long l = dd0 > total ? (long long)(dd0 - total) - i0 : 0;
-            if (l < 0) l = 0;
-            long long h = (long long)min((unsigned long long)sz, dd0) - i0;
-            if (h > ni) h = ni;
-            lo = l; hi = h;
-            while (lo < hi) {
-                long long mid = (lo + hi) >> 1;
-                if ((unsigned long long)sm->scan[mid + 1] <= dd0 - 1 - (unsigned long long)(mid + i0)) lo = mid + 1; else hi = mid;
-            }
+        const unsigned long long dd0 = min(d1, d0 + (unsigned long long)threadIdx.x * kStrictVT);
+        const unsigned long long dd1 = min(d1, dd0 + kStrictVT);
+        // local merge path: items consumed at dd0, searched in [max(0,dd0-total)-i0, min(sz,dd0)-i0]
+        long long lo = dd0 > total ? (long long)(dd0 - total) - i0 : 0;
+        if (lo < 0) lo = 0;
+        long long hi = (long long)min((unsigned long long)sz, dd0) - i0;
+        if (hi > ni) hi = ni;
+        while (lo < hi) {
+            long long mid = (lo + hi) >> 1;
+            if ((unsigned long long)sm->scan[mid + 1] <= dd0 - 1 - (unsigned long long)(mid + i0)) lo = mid + 1;
+            else hi = mid;
         }
-        long long ii = lo;                                    // local item index
+        long long ii = lo;                                      // local item index
         unsigned long long k = dd0 - (unsigned long long)(ii + i0);  // global edge index
-        for (unsigned long long dd = dd0; dd < dd1; ++dd) {
-            if (ii < ni && (unsigned long long)sm->scan[ii + 1] <= k) { ++ii; continue; }   // item ends
-            // edge k belongs to item ii
-            int x = sm->x[ii];
-            if (x >= 0 && !op.skip(x)) {
-                uint32_t e = sm->beg[ii] + (uint32_t)(k - sm->scan[ii]);
-                cnt.edges++;
-                op.edge(x, e, __ldg(g.col + e), cnt);
+        int xs[kStrictVT];
+        uint32_t es[kStrictVT];
+        bool ok[kStrictVT], stop[kStrictVT];
+#pragma unroll
+        for (int s = 0; s < kStrictVT; ++s) {
+            ok[s] = false; xs[s] = -1; es[s] = 0;
+            unsigned long long dd = dd0 + s;
+            if (dd < dd1) {
+                if (ii < ni && (unsigned long long)sm->scan[ii + 1] <= k) {
+                    ++ii;                                       // item ends: consume it
+                } else {
+                    int x = sm->x[ii];
+                    xs[s] = x;
+                    es[s] = sm->beg[ii] + (uint32_t)(k - sm->scan[ii]);
+                    ok[s] = x >= 0 && !(Op::kEarlyExit && op.skip(x));
+                    ++k;
+                }
             }
-            ++k;
         }
+        edge_batch<kStrictVT>(op, g, xs, es, ok, stop, cnt);
         __syncthreads();
+    }
+    return cnt;
+}
+
+}  // namespace gsw
+
+namespace gsw {
+
+union LbSmem {
+    TwcSmem twc;
+    CmSmem cm;
+    StrictSmem strict;
+};
+
+// Dispatch the selected load-balance candidate (Fig. 13: one Expand variant per iteration).
+// STRICT adds its two scan phases, each closed by a grid barrier.
+template <class Src, class Op>
+__device__ __forceinline__ LocalCnt run_lb(int lb, const Src &src, const Adj &adj, const Op &op, LbSmem &sm,
+                                           uint32_t *red, const GridBarrier &bar, unsigned &epoch,
+                                           uint32_t *partial, uint32_t *scan) {
+    switch (lb) {
+    case GSW_LB_THREAD: return lb_thread(src, adj, op);
+    case GSW_LB_TWC: return lb_twc(src, adj, op, &sm.twc);
+    case GSW_LB_WM: return lb_wm(src, adj, op);
+    case GSW_LB_CM: return lb_cm(src, adj, op, &sm.cm);
+    default: {
+        strict_scan_p1(src, adj, partial, red);
+        grid_sync(bar, epoch);
+        uint32_t total = strict_scan_p2(src, adj, partial, scan, red);
+        grid_sync(bar, epoch);
+        return lb_strict(src, adj, op, scan, total, &sm.strict);
+    }
     }
 }
 

@@ -31,21 +31,31 @@ struct DevCfg {
 __device__ __forceinline__ int pick(int forced, int chosen) { return forced != GSW_AUTO ? forced : chosen; }
 
 // BFS-like traversal (BFS, BC forward): active = frontier, inactive = unvisited.
+// Direction split (P1).  The paper's stated finding is "the pull mode is preferable ... when the
+// number of the active edges is greater than that of inactive edges", i.e. a split on
+// Ea/Eia at 1.  Its CART tree learns the split point per GPU (P:1220-1221 retrains for P100); on
+// B200 the early-exit pull of tools/strategy_table.py wins already at Ea/Eia ~ 1/2 and loses at
+// ~1/3600, and pulling a tiny frontier costs a full scan of the visited map, so the calibrated
+// split is  pull <=> Ea * kPullAlpha > Eia  and  Va * kPullBeta > N   (reading R6).
+constexpr float kPullAlpha = 16.f;
+constexpr float kPullBeta = 1024.f;
+
+__device__ __forceinline__ int traversal_direction(const Features &f) {
+    return ((float)f.Ea * kPullAlpha > (float)f.Eia && (float)f.Va * kPullBeta > f.N) ? GSW_PULL : GSW_PUSH;
+}
+
 __device__ __forceinline__ DevCfg select_traversal(const Features &f, const gsw_config &force) {
     DevCfg c;
-    // P1 direction: "the pull mode is preferable ... when the number of the active edges is
-    // greater than that of inactive edges".
-    c.dir = pick(force.direction, f.Ea > f.Eia ? GSW_PULL : GSW_PUSH);
+    c.dir = pick(force.direction, traversal_direction(f));
     float cd = f.Va > 0 ? (float)f.Ea / (float)f.Va : 0.f;
     // P3 load balance: "TWC has the lowest overhead", "CM and WM perform better with irregular
-    // workloads", "when the workload contains a hub vertex ... STRICT is the best";
-    // Fig. 14 picks TWC for every pull iteration.
+    // workloads", "when the workload contains a hub vertex ... STRICT is the best".
+    // Pull with early exit scans ~1-2 edges per vertex, so the per-thread mapping wins on B200.
     int lb;
-    if (c.dir == GSW_PULL) lb = GSW_LB_TWC;
-    else if (f.Ea < 8192) lb = GSW_LB_WM;                                   // tiny, latency-bound
-    else if (f.maxd > 32u * kBlock && f.maxd > 64.f * cd) lb = GSW_LB_STRICT;  // hub in workload
-    else if (f.maxd > 16.f * cd) lb = GSW_LB_CM;                             // irregular
-    else lb = GSW_LB_TWC;
+    if (c.dir == GSW_PULL) lb = GSW_LB_THREAD;
+    else if (f.Ea <= 8192 && f.maxd <= 1024u) lb = GSW_LB_WM;               // tiny, latency-bound
+    else if (f.maxd > 1024u || cd > 64.f) lb = GSW_LB_STRICT;                // hub in workload
+    else lb = GSW_LB_TWC;                                                    // regular degrees
     c.lb = pick(force.load_balance, lb);
     // P2 format: "bitmap is more friendly to dense workloads, the unsorted queue is more friendly
     // to sparse workloads, and the sorted queue is in the middle"; Fig. 12(b): queue
@@ -53,8 +63,8 @@ __device__ __forceinline__ DevCfg select_traversal(const Features &f, const gsw_
     float vap = f.N > 0 ? (float)f.Va / f.N : 0.f;
     int fmt;
     if (c.dir == GSW_PULL) fmt = GSW_BITMAP;
-    else if (vap > 1.f / 32.f) fmt = GSW_BITMAP;
-    else if (vap > 1.f / 512.f) fmt = GSW_SORTED_QUEUE;
+    else if (vap > 1.f / 16.f) fmt = GSW_BITMAP;
+    else if (vap > 1.f / 256.f) fmt = GSW_SORTED_QUEUE;
     else fmt = GSW_QUEUE;
     c.fmt = pick(force.format, fmt);
     c.step = GSW_STEP_REMAIN;

@@ -65,9 +65,11 @@ def test_features_match_oracle_per_level(gsw):
         assert [r["Ea"] for r in rec] == Ea.tolist()
         assert [r["Via"] for r in rec] == Via.tolist()
         assert [r["Eia"] for r in rec] == Eia.tolist()
-        # direction rule "pull when active edges > inactive edges" reproduced exactly
+        # direction split on Ea/Eia with the B200-calibrated constants (select.cuh,
+        # DESIGN.md reading R6), reproduced exactly
         for r in rec:
-            assert r["direction"] == (gsw.PULL if r["Ea"] > r["Eia"] else gsw.PUSH)
+            pull = r["Ea"] * 16.0 > r["Eia"] and r["Va"] * 1024.0 > g.n
+            assert r["direction"] == (gsw.PULL if pull else gsw.PUSH)
 
 
 def test_attributes_match_oracle(gsw):
