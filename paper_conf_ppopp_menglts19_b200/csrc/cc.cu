@@ -1,0 +1,247 @@
+// cc.cu -- connected components ("edge-centric") as min-label
+// propagation in GSWITCH's Filter/Expand form (reading R8): label[v] starts at v; the
+// active set is the vertices whose label changed in the previous iteration; Expand propagates
+// labels either by push (compAtomic = atomicMin on the neighbour) or by pull (comp = min over the
+// active in-neighbours, an atomic-free reduction for owner mappings).  The fixpoint is
+// label[v] = min vertex id of v's component.  Terminates when no label changed.
+//   Filter: fused  -> Expand marks changed vertices in the next active-set bitmap
+//           standalone -> a Filter pass compares label with its value at the iteration start
+#include "engine.cuh"
+#include "internal.h"
+#include "launch.h"
+#include "lb.cuh"
+#include "lb_reduce.cuh"
+
+namespace gsw {
+
+struct CcArgs {
+    DevGraph g;
+    const unsigned *iso;
+    int *label;
+    unsigned *chg;        // per-vertex "label changed" status flags (standalone filter)
+    unsigned *fb[3];      // active-set bitmaps, ring of 3
+    int *q;               // active-set queue (push in queue formats)
+    uint32_t *scan;
+    long long iso_count;
+    RunCommon rc;
+};
+
+struct CcPushTok { unsigned old; int lu; };
+struct CcPushAux { unsigned claim; uint32_t d0, d1; };
+
+// push: for active u, every neighbour v gets atomicMin(label[v], label[u])
+struct CcPushOp {
+    int *label;
+    const uint32_t *off;
+    bool fused;
+    unsigned *nfb;
+    using Probe = int2;          // (label[u], label[v])
+    using Tok = CcPushTok;
+    using Aux = CcPushAux;
+    static constexpr bool kEarlyExit = false;
+    __device__ __forceinline__ bool skip(int) const { return false; }
+    __device__ __forceinline__ Probe probe(int u, uint32_t, int v) const { return make_int2(label[u], label[v]); }
+    __device__ __forceinline__ Tok act(int, uint32_t, int v, Probe p) const {
+        return CcPushTok{p.x < p.y ? (unsigned)atomicMin(label + v, p.x) : 0x80000000u, p.x};
+    }
+    __device__ __forceinline__ Aux aux(int, uint32_t, int v, Tok t) const {
+        bool improved = t.old != 0x80000000u && t.lu < (int)t.old;
+        if (!improved) return CcPushAux{~0u, 0u, 0u};
+        unsigned bit = 1u << (v & 31);
+        if (!fused) { atomicOr(nfb + (v >> 5), bit); return CcPushAux{~0u, 0u, 0u}; }   // status flag only
+        unsigned c = atomicOr(nfb + (v >> 5), bit);
+        return CcPushAux{c, __ldg(off + v), __ldg(off + v + 1)};
+    }
+    __device__ __forceinline__ bool commit(int, uint32_t, int v, Tok, Aux a, LocalCnt &c) const {
+        if (fused && !((a.claim >> (v & 31)) & 1u)) c.add_vertex(a.d1 - a.d0);
+        return false;
+    }
+};
+
+// pull: label[v] = min(label[v], min over active in-neighbours u of label[u])
+struct CcPullOp {
+    int *label;
+    const unsigned *fb;          // active set
+    const uint32_t *off;         // out-offsets (degree of a changed vertex)
+    bool fused;
+    unsigned *nfb;
+    using Probe = uint2;         // (active-set word of u, label[u])
+    using Acc = unsigned long long;
+    static constexpr bool kFlushEmpty = false;
+    static __device__ __forceinline__ Acc identity() { return 0x7fffffffull; }
+    static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a < b ? a : b; }
+    __device__ __forceinline__ bool skip(int) const { return false; }
+    __device__ __forceinline__ Probe probe(int, uint32_t, int u) const {
+        return make_uint2(fb[u >> 5], (unsigned)label[u]);
+    }
+    __device__ __forceinline__ Acc val(int, uint32_t, int u, Probe p) const {
+        return ((p.x >> (u & 31)) & 1u) ? (Acc)p.y : identity();
+    }
+    __device__ __forceinline__ void flush(int v, Acc m, bool exclusive, LocalCnt &c) const {
+        if (m == identity()) return;
+        int mi = (int)m;
+        unsigned bit = 1u << (v & 31);
+        if (exclusive) {
+            if (mi < label[v]) {
+                label[v] = mi;
+                atomicOr(nfb + (v >> 5), bit);
+                if (fused) c.add_vertex(__ldg(off + v + 1) - __ldg(off + v));
+            }
+        } else {
+            int old = atomicMin(label + v, mi);
+            if (mi < old) {
+                if (!fused) atomicOr(nfb + (v >> 5), bit);
+                else if (!(atomicOr(nfb + (v >> 5), bit) & bit)) c.add_vertex(__ldg(off + v + 1) - __ldg(off + v));
+            }
+        }
+    }
+};
+
+__device__ __forceinline__ DevCfg select_cc(const Features &f, const gsw_config &force) {
+    DevCfg c = select_traversal(f, force);
+    // the pull workload is every non-isolated vertex: reduce with the owner mappings
+    if (c.dir == GSW_PULL && force.load_balance == GSW_AUTO) c.lb = GSW_LB_TWC;
+    return c;
+}
+
+union CcSmem {
+    LbSmem push;
+    LbRedSmem pull;
+};
+
+__global__ void __launch_bounds__(kBlock, kMinBlocks) cc_kernel(CcArgs a) {
+    __shared__ CcSmem sm;
+    __shared__ uint32_t red[kWarps + 1];
+    const RunCommon &rc = a.rc;
+    const GridBarrier bar = make_bar(rc);
+    unsigned epoch = 0;
+    const int n = a.g.n, W = (n + 31) >> 5;
+    const Adj adj_out{a.g.off, a.g.col}, adj_in{a.g.in_off, a.g.in_col};
+
+    // ---- init: label = id, AS_0 = every non-isolated vertex
+    for (long long v = gtid(); v < n; v += gthreads()) a.label[v] = (int)v;
+    for (long long w = gtid(); w < W; w += gthreads()) {
+        unsigned valid = (w == W - 1 && (n & 31)) ? ((1u << (n & 31)) - 1u) : ~0u;
+        a.fb[0][w] = ~a.iso[w] & valid;
+        a.fb[1][w] = 0u; a.fb[2][w] = 0u;
+        a.chg[w] = 0u;
+    }
+    if (is_book()) {
+        for (int i = 0; i < 3; ++i) reset_cnt(rc.cnt + i);
+        rc.cnt[0].va = (unsigned long long)(n - a.iso_count);
+        rc.cnt[0].ea = a.g.nnz;
+        rc.cnt[0].maxd = 0; rc.cnt[0].mind = 0;
+    }
+    grid_sync(bar, epoch);
+
+    Book book;
+    Features f = rc.base;
+    bool dirty[3] = {true, false, false};
+    int prev_dir = GSW_PULL;
+    unsigned long long prev_va = 0;
+    int t = 0;
+    for (;; ++t) {
+        IterCnt *cur = rc.cnt + (t % 3), *nxt = rc.cnt + ((t + 1) % 3);
+        if (is_book()) book_start(book, rc, t, nxt);
+        const CntView cv = cta_read_cnt(cur);
+        if (is_book() && t > 0) {
+            book.bytes += 12ull * prev_va + 4ull * cv.edges + (prev_dir == GSW_PULL ? 4ull * n + n / 8 : 0ull);
+            book.edges += cv.edges;
+            if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)cv.edges;
+        }
+        if (cv.va == 0) break;
+        f.Va = (long long)cv.va; f.Ea = (long long)cv.ea;
+        f.Via = (long long)n - f.Va; f.Eia = (long long)a.g.nnz - f.Ea;
+        f.maxd = cv.maxd; f.mind = cv.mind; f.iter = t;
+        hist_features(cv, f);
+        const DevCfg c = select_cc(f, rc.force);
+        write_record(rc, t, c, f, 0u);
+        if (is_book()) reset_cnt(rc.cnt + ((t + 2) % 3));
+        const int b2 = (t + 2) % 3;
+        if (dirty[b2]) { clear_words(a.fb[b2], W); dirty[b2] = false; }
+        unsigned *fbt = a.fb[t % 3];
+        const bool push = c.dir == GSW_PUSH;
+        const bool fused = c.fused == GSW_FUSED;
+        unsigned *nfb = a.fb[(t + 1) % 3];
+
+        // ---------------- Filter: AS_t is a bitmap; queue formats compact it for push
+        unsigned qlen = 0;
+        if (push && c.fmt != GSW_BITMAP) {
+            if (c.fmt == GSW_QUEUE) {
+                q_from_bm(a.q, &cur->qlen, fbt, W, 0u);
+            } else {
+                sq_from_bm_p1(fbt, W, 0u, rc.partial, red);
+                grid_sync(bar, epoch);
+                sq_from_bm_p2(a.q, &cur->qlen, fbt, W, 0u, rc.partial, red);
+            }
+            grid_sync(bar, epoch);
+            qlen = cta_read_u32(&cur->qlen);
+        }
+        if (is_book()) book_expand(book);
+
+        // ---------------- Expand
+        // fused: Expand claims changed vertices straight into AS_{t+1} (counting the winners);
+        // standalone: Expand only raises the per-vertex "changed" status flag
+        unsigned *mark = fused ? nfb : a.chg;
+        LocalCnt lc;
+        if (push) {
+            const CcPushOp op{a.label, a.g.off, fused, mark};
+            if (c.fmt == GSW_BITMAP)
+                lc = run_lb(c.lb, BitmapSrc{fbt, (unsigned)n, 1u}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
+            else
+                lc = run_lb(c.lb, QueueSrc{a.q, qlen}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
+        } else {
+            const CcPullOp op{a.label, fbt, a.g.off, fused, mark};
+            lc = run_lb_reduce(c.lb, BitmapSrc{a.iso, (unsigned)n, 0u}, adj_in, op, sm.pull, red, bar, epoch,
+                               rc.partial, a.scan);
+        }
+        dirty[(t + 1) % 3] = true;
+        if (fused) {
+            flush_counts(lc, nxt);
+            grid_sync(bar, epoch);
+        } else {
+            // standalone Filter: generate AS_{t+1} from the vertex status flags
+            LocalCnt ec;
+            ec.edges = lc.edges;
+            grid_sync(bar, epoch);
+            for (long long w = gwarp(); w < W; w += gwarps()) {
+                unsigned m = a.chg[w];                     // warp-uniform word
+                int v = (int)(w * 32 + lane_id());
+                if ((m >> lane_id()) & 1u) ec.add_vertex(__ldg(a.g.off + v + 1) - __ldg(a.g.off + v));
+                if (lane_id() == 0) { nfb[w] = m; a.chg[w] = 0u; }
+            }
+            flush_counts(ec, nxt);
+            grid_sync(bar, epoch);
+        }
+        prev_dir = c.dir;
+        prev_va = cv.va;
+    }
+    if (is_book()) book_finish(book, rc, t);
+}
+
+gsw_status run_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
+    const int n = g->g.n, W = (n + 31) / 32;
+    if (!label_out) { set_error("gsw_cc: label is NULL"); return GSW_EINVAL; }
+    Workspace ws{g->scratch, g->scratch_bytes, 0};
+    const bool dev_out = is_device_ptr(label_out) == 1;
+    CcArgs a{};
+    a.g = g->g;
+    a.iso = g->iso;
+    a.label = dev_out ? label_out : (int *)ws.take((size_t)n * 4);
+    a.chg = (unsigned *)ws.take((size_t)W * 4);
+    for (int i = 0; i < 3; ++i) a.fb[i] = (unsigned *)ws.take((size_t)W * 4);
+    a.q = (int *)ws.take((size_t)n * 4);
+    a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
+    a.iso_count = g->attrs.isolated;
+    LaunchInfo li;
+    gsw_status s = prepare_common(g, ws, (const void *)cc_kernel, a.rc, li);
+    if (s != GSW_OK) return s;
+    if (!a.label || !a.chg || !a.fb[2] || !a.q || !a.scan) { set_error("workspace too small"); return GSW_ENOMEM; }
+    void *args[] = {&a};
+    s = launch_persistent(g, (const void *)cc_kernel, args, li);
+    if (s != GSW_OK) return s;
+    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(label_out, a.label, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
+    return finish_run(g, a.rc, li, st);
+}
+
+}  // namespace gsw

@@ -244,6 +244,7 @@ __device__ __forceinline__ unsigned cta_read_u32(const unsigned *p) {
 struct LocalCnt {
     unsigned long long va = 0, ea = 0, edges = 0;
     unsigned maxd = 0, mind = 0xffffffffu;
+    double facc = 0.0;          // algorithm-specific fp64 side sum (PR dangling mass)
     __device__ __forceinline__ void add_vertex(unsigned deg) {
         va += 1; ea += deg;
         maxd = deg > maxd ? deg : maxd;
