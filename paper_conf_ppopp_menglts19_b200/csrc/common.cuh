@@ -191,6 +191,7 @@ struct alignas(128) IterCnt {
     unsigned qlen;          // length of the queue materialised for this active set (if any)
     unsigned iqlen;         // length of the inactive (pull workload) queue, if built
     float tf, te, Tf, Te;   // history features carried to the iteration that reads this slot
+    unsigned aux0, aux1;    // algorithm-specific control words (SSSP: far-set length / min)
 };
 
 // After a grid barrier every CTA needs the same few control words.  Reading them from every warp
@@ -200,6 +201,7 @@ struct CntView {
     unsigned long long va, ea, edges;
     unsigned maxd, mind, qlen, iqlen;
     float tf, te, Tf, Te;
+    unsigned aux0, aux1;
 };
 __device__ __forceinline__ unsigned long long ld_relaxed64_nc(const unsigned long long *p) {
     unsigned long long v;
@@ -228,6 +230,7 @@ __device__ __forceinline__ CntView cta_read_cnt(const IterCnt *c) {
         v.qlen = d.x; v.iqlen = d.y;
         v.tf = __uint_as_float(d.z); v.te = __uint_as_float(d.w);
         v.Tf = __uint_as_float(e.x); v.Te = __uint_as_float(e.y);
+        v.aux0 = e.z; v.aux1 = e.w;
         s = v;
     }
     __syncthreads();
@@ -245,6 +248,7 @@ struct LocalCnt {
     unsigned long long va = 0, ea = 0, edges = 0;
     unsigned maxd = 0, mind = 0xffffffffu;
     double facc = 0.0;          // algorithm-specific fp64 side sum (PR dangling mass)
+    unsigned aux = 0;           // algorithm-specific count (SSSP far-set appends) -> IterCnt::aux0
     __device__ __forceinline__ void add_vertex(unsigned deg) {
         va += 1; ea += deg;
         maxd = deg > maxd ? deg : maxd;
@@ -258,18 +262,20 @@ __device__ __forceinline__ void flush_counts(LocalCnt &c, IterCnt *dst) {
     __shared__ unsigned long long s64[kWarps][3];
     __shared__ unsigned s32[kWarps][2];
     unsigned long long va = warp_sum(c.va), ea = warp_sum(c.ea), ed = warp_sum(c.edges);
-    unsigned mx = warp_max(c.maxd), mn = warp_min(c.mind);
+    unsigned mx = warp_max(c.maxd), mn = warp_min(c.mind), ax = warp_sum(c.aux);
     unsigned w = threadIdx.x >> 5;
-    if (lane_id() == 0) { s64[w][0] = va; s64[w][1] = ea; s64[w][2] = ed; s32[w][0] = mx; s32[w][1] = mn; }
+    __shared__ unsigned sax[kWarps];
+    if (lane_id() == 0) { s64[w][0] = va; s64[w][1] = ea; s64[w][2] = ed; s32[w][0] = mx; s32[w][1] = mn; sax[w] = ax; }
     __syncthreads();
     if (threadIdx.x == 0) {
         for (int i = 1; i < kWarps; ++i) {
-            va += s64[i][0]; ea += s64[i][1]; ed += s64[i][2];
+            va += s64[i][0]; ea += s64[i][1]; ed += s64[i][2]; ax += sax[i];
             mx = s32[i][0] > mx ? s32[i][0] : mx;
             mn = s32[i][1] < mn ? s32[i][1] : mn;
         }
         if (va) { atomicAdd(&dst->va, va); atomicAdd(&dst->ea, ea); atomicMax(&dst->maxd, mx); atomicMin(&dst->mind, mn); }
         if (ed) atomicAdd(&dst->edges, ed);
+        if (ax) atomicAdd(&dst->aux0, ax);
     }
     __syncthreads();
     c = LocalCnt();
@@ -278,6 +284,7 @@ __device__ __forceinline__ void flush_counts(LocalCnt &c, IterCnt *dst) {
 __device__ __forceinline__ void reset_cnt(IterCnt *c) {
     c->va = 0; c->ea = 0; c->edges = 0; c->maxd = 0; c->mind = 0xffffffffu; c->qlen = 0; c->iqlen = 0;
     c->tf = 0.f; c->te = 0.f; c->Tf = 0.f; c->Te = 0.f;
+    c->aux0 = 0u; c->aux1 = 0xffffffffu;
 }
 
 // grid-stride helpers

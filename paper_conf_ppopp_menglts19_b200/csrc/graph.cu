@@ -26,7 +26,7 @@ __global__ void k_isolated_bitmap(const uint32_t *off, int n, unsigned *iso, int
 }
 
 struct AttrAcc {
-    unsigned long long sum, iso;
+    unsigned long long sum, iso, wsum;
     double sumsq, dlnd;
     unsigned maxd, mind, maxw, bad;
 };
@@ -65,9 +65,11 @@ __global__ void k_degree_hist(const uint32_t *off, int n, unsigned long long *hi
 
 __global__ void k_maxw(const uint32_t *w, long long nnz, AttrAcc *acc) {
     unsigned mx = 0;
-    for (long long e = gtid(); e < nnz; e += gthreads()) mx = max(mx, w[e]);
+    unsigned long long s = 0;
+    for (long long e = gtid(); e < nnz; e += gthreads()) { mx = max(mx, w[e]); s += w[e]; }
     mx = warp_max(mx);
-    if (lane_id() == 0) atomicMax(&acc->maxw, mx);
+    s = warp_sum(s);
+    if (lane_id() == 0) { atomicMax(&acc->maxw, mx); atomicAdd(&acc->wsum, s); }
 }
 
 __global__ void k_validate(const uint32_t *off, const int32_t *col, int n, long long nnz, unsigned *bad) {
@@ -187,6 +189,7 @@ gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp) {
     A.maxdeg = h.maxd;
     A.mindeg = h.mind;
     A.maxw = h.maxw;
+    A.wbar = G.nnz ? (double)h.wsum / (double)G.nnz : 0.0;
     A.isolated = (int64_t)h.iso;
     return GSW_OK;
 }

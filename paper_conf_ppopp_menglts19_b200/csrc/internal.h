@@ -27,6 +27,7 @@ struct Attrs {
     double N, M, dbar, sd, rd, gini, her;
     uint32_t maxdeg, mindeg, maxw;
     int64_t isolated;
+    double wbar;              // mean edge weight (SSSP static step c*wbar/dbar)
 };
 
 // Packed per-iteration configuration (Fig. 13: one choice per pattern).

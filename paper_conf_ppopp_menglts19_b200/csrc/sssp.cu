@@ -1,0 +1,434 @@
+// sssp.cu -- single-source shortest paths with GSWITCH's stepping pattern (P4, PAPER.md:548-556,
+// 646-666; footnote 2 P:411-413) on the persistent Filter/Expand engine.
+// Ordered, label-correcting near/far scheme (reading R5/R7):
+//   - the active (near) set N_t = vertices improved in round t-1 with dist < theta;
+//   - improved vertices with dist >= theta go to the far set F (deferred);
+//   - Expand relaxes every edge out of N_t: nd = dist[u] + w(u,v); atomicMin(dist[v], nd)
+//     (compAtomic, push) or dist[v] = min over near in-neighbours (comp, pull reduction);
+//   - when N_t is empty, theta advances and F is split: dist < theta -> N, the rest stays in F;
+//   - terminate when N and F are empty.
+// Stepping candidates for the threshold theta (gsw_config.stepping):
+//   AUTO (dynamic stepping): per round, Increase (theta += delta0) when the active edges dropped by
+//   more than 35% (Fig. 12(e): increase when Ea is small), Decrease (theta -= delta0/2,
+//   never below the last split point) when they grew by more than 35%, otherwise Remain;
+//   INCREASE / DECREASE / REMAIN pin that per-round decision; STATIC = delta-stepping with a fixed
+//   step (theta moves only at splits); UNORDERED = Bellman-Ford (theta = infinity).
+// delta0 = gsw_config.delta0, or c*wbar/dbar with c = 32 (reading R6b).
+// Any schedule reaches the exact distances (they are the unique fixpoint); only speed differs.
+#include "engine.cuh"
+#include "internal.h"
+#include "launch.h"
+#include "lb.cuh"
+#include "lb_reduce.cuh"
+
+namespace gsw {
+
+enum { SM_NONE = 0, SM_QUEUE = 1, SM_SQUEUE = 2, SM_BITMAP = 3 };
+enum { ST_DYNAMIC = 0, ST_STATIC = 1, ST_UNORDERED = 2, ST_INC = 3, ST_DEC = 4, ST_REMAIN = 5 };
+
+struct SplitCnt {
+    unsigned long long va, ea;
+    unsigned qlen, kept, minf, pad;
+};
+
+struct SsspArgs {
+    DevGraph g;
+    int src;
+    unsigned *dist;
+    unsigned *nb[3];      // near-set bitmaps (ring of 3); also the claim map of the next near set
+    int *q[2];            // near queues
+    unsigned *chg;        // "improved this round" status flags (standalone filter)
+    unsigned *farbit;     // far-set membership
+    int *fq[2];           // far queues
+    unsigned *flen;       // far queue append counters [2]
+    SplitCnt *split;      // [2]
+    uint32_t *scan;
+    unsigned delta0;
+    int mode;
+    RunCommon rc;
+};
+
+struct SsTok { unsigned old, nd; };
+struct SsAux { unsigned nclaim, fclaim; uint32_t d0, d1; };
+
+// classify an improved vertex: near (claim the next near map) or far (claim the far map)
+struct SsClassify {
+    unsigned *nnb;
+    unsigned *farbit;
+    unsigned theta;
+    bool fused;
+    unsigned *chg;
+};
+
+// push: relax (u, v): nd = dist[u] + w; atomicMin(dist[v], nd)
+struct SsspPushOp {
+    unsigned *dist;
+    const uint32_t *w;
+    const uint32_t *off;
+    SsClassify cl;
+    int *nq;              // next near queue (fused, few claims) or nullptr (bitmap marking)
+    unsigned *nqlen;
+    int *fq;
+    unsigned *fqlen;
+    using Probe = uint2;  // (dist[u] + w(u,v), dist[v])
+    using Tok = SsTok;
+    using Aux = SsAux;
+    static constexpr bool kEarlyExit = false;
+    __device__ __forceinline__ bool skip(int) const { return false; }
+    __device__ __forceinline__ Probe probe(int u, uint32_t e, int v) const {
+        return make_uint2(dist[u] + __ldg(w + e), dist[v]);
+    }
+    __device__ __forceinline__ Tok act(int, uint32_t, int v, Probe p) const {
+        return SsTok{p.x < p.y ? atomicMin(dist + v, p.x) : 0u, p.x < p.y ? p.x : 0xffffffffu};
+    }
+    __device__ __forceinline__ Aux aux(int, uint32_t, int v, Tok t) const {
+        SsAux a{~0u, ~0u, 0u, 0u};
+        if (!(t.nd < t.old)) return a;
+        const unsigned bit = 1u << (v & 31);
+        if (!cl.fused) { atomicOr(cl.chg + (v >> 5), bit); return a; }
+        if (t.nd < cl.theta) {
+            a.nclaim = atomicOr(cl.nnb + (v >> 5), bit);
+            a.d0 = __ldg(off + v); a.d1 = __ldg(off + v + 1);
+        } else {
+            a.fclaim = atomicOr(cl.farbit + (v >> 5), bit);
+        }
+        return a;
+    }
+    __device__ __forceinline__ bool commit(int, uint32_t, int v, Tok, Aux a, LocalCnt &c) const {
+        const unsigned bit = 1u << (v & 31);
+        const bool nw = !(a.nclaim & bit), fw = !(a.fclaim & bit);
+        if (nw) c.add_vertex(a.d1 - a.d0);
+        if (nq) warp_append(nq, nqlen, nw, v);
+        if (fw) c.aux++;
+        warp_append(fq, fqlen, fw, v);
+        return false;
+    }
+};
+
+// pull: dist[v] = min(dist[v], min over near in-neighbours u of dist[u] + w(u,v))
+struct SsspPullOp {
+    unsigned *dist;
+    const uint32_t *w;        // in-edge weights
+    const unsigned *nbt;      // near set N_t
+    const uint32_t *off;      // out-offsets
+    SsClassify cl;
+    int *fq;
+    unsigned *fqlen;
+    using Probe = uint2;      // (near word of u, dist[u])
+    using Acc = unsigned long long;
+    static constexpr bool kFlushEmpty = false;
+    static __device__ __forceinline__ Acc identity() { return 0xffffffffull; }
+    static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a < b ? a : b; }
+    __device__ __forceinline__ bool skip(int) const { return false; }
+    __device__ __forceinline__ Probe probe(int, uint32_t, int u) const { return make_uint2(nbt[u >> 5], dist[u]); }
+    __device__ __forceinline__ Acc val(int, uint32_t e, int u, Probe p) const {
+        return ((p.x >> (u & 31)) & 1u) ? (Acc)p.y + (Acc)__ldg(w + e) : identity();
+    }
+    __device__ __forceinline__ void flush(int v, Acc m, bool exclusive, LocalCnt &c) const {
+        if (m >= 0xffffffffull) return;
+        const unsigned nd = (unsigned)m;
+        unsigned old;
+        if (exclusive) { old = dist[v]; if (nd < old) dist[v] = nd; }
+        else old = atomicMin(dist + v, nd);
+        if (!(nd < old)) return;
+        const unsigned bit = 1u << (v & 31);
+        if (!cl.fused) { atomicOr(cl.chg + (v >> 5), bit); return; }
+        if (nd < cl.theta) {
+            if (!(atomicOr(cl.nnb + (v >> 5), bit) & bit)) c.add_vertex(__ldg(off + v + 1) - __ldg(off + v));
+        } else if (!(atomicOr(cl.farbit + (v >> 5), bit) & bit)) {
+            c.aux++;
+            fq[atomicAdd(fqlen, 1u)] = v;
+        }
+    }
+};
+
+__device__ __forceinline__ DevCfg select_sssp(const Features &f, const gsw_config &force) {
+    DevCfg c = select_traversal(f, force);
+    if (c.dir == GSW_PULL && force.load_balance == GSW_AUTO) c.lb = GSW_LB_TWC;   // reduction: owner tiers
+    return c;
+}
+
+union SsSmem {
+    LbSmem push;
+    LbRedSmem pull;
+};
+
+__global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
+    __shared__ SsSmem sm;
+    __shared__ uint32_t red[kWarps + 1];
+    const RunCommon &rc = a.rc;
+    const GridBarrier bar = make_bar(rc);
+    unsigned epoch = 0;
+    const int n = a.g.n, W = (n + 31) >> 5, src = a.src;
+    const Adj adj_out{a.g.off, a.g.col}, adj_in{a.g.in_off, a.g.in_col};
+    unsigned *dist = a.dist;
+
+    // ---- init
+    for (long long v = gtid(); v < n; v += gthreads()) dist[v] = (v == src) ? 0u : 0xffffffffu;
+    for (long long w = gtid(); w < W; w += gthreads()) {
+        a.nb[0][w] = 0u; a.nb[1][w] = 0u; a.nb[2][w] = 0u;
+        a.chg[w] = 0u; a.farbit[w] = 0u;
+    }
+    const unsigned dsrc = __ldg(a.g.off + src + 1) - __ldg(a.g.off + src);
+    if (is_book()) {
+        for (int i = 0; i < 3; ++i) reset_cnt(rc.cnt + i);
+        rc.cnt[0].va = 1; rc.cnt[0].ea = dsrc; rc.cnt[0].maxd = dsrc; rc.cnt[0].mind = dsrc; rc.cnt[0].qlen = 1;
+        a.q[0][0] = src;
+        a.flen[0] = 0u; a.flen[1] = 0u;
+        for (int i = 0; i < 2; ++i) { a.split[i] = SplitCnt{0ull, 0ull, 0u, 0u, 0xffffffffu, 0u}; }
+    }
+    grid_sync(bar, epoch);
+
+    Book book;
+    Features f = rc.base;
+    const unsigned long long kInf = 0xffffffffull;
+    const unsigned d0 = a.delta0;
+    unsigned long long theta = a.mode == ST_UNORDERED ? kInf : (unsigned long long)d0;
+    unsigned long long floor_t = 0;
+    unsigned long long flen = 0;          // |F| (identical in every thread)
+    int fcur = 0;                         // far queue buffer receiving appends
+    int nsplit = 0;
+    unsigned long long prev_ea = 0;
+    int mat = SM_SQUEUE;
+    bool dirty[3] = {false, false, false};
+    int prev_dir = GSW_PUSH;
+    unsigned long long prev_va = 0;
+    int t = 0;
+    for (;; ++t) {
+        IterCnt *cur = rc.cnt + (t % 3), *nxt = rc.cnt + ((t + 1) % 3);
+        if (is_book()) book_start(book, rc, t, nxt);
+        CntView cv = cta_read_cnt(cur);
+        flen += cv.aux0;
+        if (is_book() && t > 0) {
+            book.bytes += 12ull * prev_va + 8ull * cv.edges + 8ull * cv.va +
+                          (prev_dir == GSW_PULL ? 4ull * n + n / 8 : 0ull);
+            book.edges += cv.edges;
+            if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)cv.edges;
+        }
+        // ---- near set empty: advance theta and split the far set (Filter of the far queue)
+        while (cv.va == 0 && flen > 0) {
+            SplitCnt *sp = a.split + (nsplit & 1);
+            theta = theta + d0;
+            floor_t = theta;
+            const int fsrc = fcur, fdst = fcur ^ 1;
+            // everything appended to fq[fsrc] so far: flen entries
+            const unsigned L = (unsigned)flen;
+            LocalCnt lc;
+            unsigned lmin = 0xffffffffu;
+            int *qa = a.q[t & 1];
+            for (long long base = gwarp() * 32; base < L; base += gwarps() * 32) {
+                long long i = base + lane_id();
+                int v = i < L ? a.fq[fsrc][i] : -1;
+                unsigned dv = v >= 0 ? dist[v] : 0xffffffffu;
+                bool to_near = v >= 0 && (unsigned long long)dv < theta;
+                bool keep = v >= 0 && !to_near;
+                if (to_near) {
+                    atomicAnd(a.farbit + (v >> 5), ~(1u << (v & 31)));
+                    lc.add_vertex(__ldg(a.g.off + v + 1) - __ldg(a.g.off + v));
+                }
+                warp_append(qa, &sp->qlen, to_near, v);
+                warp_append(a.fq[fdst], a.flen + fdst, keep, v);
+                if (keep) { lc.aux++; lmin = min(lmin, dv); }
+            }
+            // per-CTA reduction into the split counters
+            {
+                unsigned long long va = block_sum(lc.va, (unsigned long long *)sm.push.cm.excl);
+                unsigned long long ea = block_sum(lc.ea, (unsigned long long *)sm.push.cm.excl);
+                unsigned kept = block_sum(lc.aux, red);
+                unsigned mn = warp_min(lmin);
+                __shared__ unsigned smin[kWarps];
+                if (lane_id() == 0) smin[threadIdx.x >> 5] = mn;
+                __syncthreads();
+                if (threadIdx.x == 0) {
+                    for (int i = 0; i < kWarps; ++i) mn = min(mn, smin[i]);
+                    if (va) { atomicAdd(&sp->va, va); atomicAdd(&sp->ea, ea); }
+                    if (kept) atomicAdd(&sp->kept, kept);
+                    if (mn != 0xffffffffu) atomicMin(&sp->minf, mn);
+                }
+            }
+            grid_sync(bar, epoch);
+            __shared__ SplitCnt ssp;
+            if (threadIdx.x == 0) {
+                // plain loads after the barrier's acquire (L1 invalidated)
+                ssp.va = sp->va; ssp.ea = sp->ea; ssp.qlen = sp->qlen; ssp.kept = sp->kept; ssp.minf = sp->minf;
+            }
+            __syncthreads();
+            const SplitCnt r = ssp;
+            __syncthreads();
+            if (is_book()) {
+                a.flen[fsrc] = 0u;                                   // drained buffer
+                a.split[(nsplit + 1) & 1] = SplitCnt{0ull, 0ull, 0u, 0u, 0xffffffffu, 0u};
+            }
+            nsplit++;
+            fcur = fdst;
+            flen = r.kept;
+            cv.va = r.va; cv.ea = r.ea; cv.qlen = r.qlen;
+            cv.maxd = 0; cv.mind = 0;
+            mat = SM_QUEUE;
+            if (r.va == 0 && r.minf != 0xffffffffu && (unsigned long long)r.minf + 1 > theta + d0)
+                theta = (unsigned long long)r.minf + 1 - d0;              // jump over empty buckets
+        }
+        if (cv.va == 0) break;
+        f.Va = (long long)cv.va; f.Ea = (long long)cv.ea;
+        f.Via = (long long)n - f.Va; f.Eia = (long long)a.g.nnz - f.Ea;
+        f.maxd = cv.maxd; f.mind = cv.mind; f.iter = t;
+        hist_features(cv, f);
+        DevCfg c = select_sssp(f, rc.force);
+        // ---- P4 stepping decision for this round
+        int step = GSW_STEP_REMAIN;
+        if (a.mode == ST_DYNAMIC && t > 0 && prev_ea > 0) {
+            if ((double)cv.ea < 0.65 * (double)prev_ea) step = GSW_STEP_INCREASE;
+            else if ((double)cv.ea > 1.35 * (double)prev_ea) step = GSW_STEP_DECREASE;
+        } else if (a.mode == ST_INC) step = GSW_STEP_INCREASE;
+        else if (a.mode == ST_DEC) step = GSW_STEP_DECREASE;
+        if (a.mode != ST_UNORDERED && a.mode != ST_STATIC) {
+            if (step == GSW_STEP_INCREASE) theta = min(kInf, theta + d0);
+            else if (step == GSW_STEP_DECREASE) theta = max(floor_t, theta > d0 / 2 ? theta - d0 / 2 : 0ull);
+        }
+        c.step = a.mode == ST_STATIC ? GSW_STEP_STATIC : (a.mode == ST_UNORDERED ? GSW_STEP_UNORDERED : step);
+        prev_ea = cv.ea;
+        const unsigned th = (unsigned)min(theta, kInf);
+        write_record(rc, t, c, f, th);
+        if (is_book()) reset_cnt(rc.cnt + ((t + 2) % 3));
+        const int b2 = (t + 2) % 3;
+        if (dirty[b2]) { clear_words(a.nb[b2], W); dirty[b2] = false; }
+
+        // ---------------- Filter: materialise N_t in the selected format
+        const bool push = c.dir == GSW_PUSH;
+        int need;
+        if (push) need = c.fmt == GSW_BITMAP ? SM_BITMAP : (c.fmt == GSW_QUEUE ? SM_QUEUE : SM_SQUEUE);
+        else need = SM_BITMAP;                     // pull tests membership in N_t
+        int *qa = a.q[t & 1];
+        unsigned *nbt = a.nb[t % 3];
+        bool filtered = false, qlen_changed = false;
+        if (need == SM_BITMAP && mat != SM_BITMAP) {
+            bm_from_q(nbt, qa, cv.qlen);
+            dirty[t % 3] = true;
+            mat = SM_BITMAP;
+            filtered = true;
+        } else if (need == SM_QUEUE && mat == SM_BITMAP) {
+            q_from_bm(qa, &cur->qlen, nbt, W, 0u);
+            mat = SM_QUEUE;
+            filtered = qlen_changed = true;
+        } else if (need == SM_SQUEUE && mat != SM_SQUEUE) {
+            if (mat != SM_BITMAP) {
+                bm_from_q(nbt, qa, cv.qlen);
+                dirty[t % 3] = true;
+                grid_sync(bar, epoch);
+            }
+            sq_from_bm_p1(nbt, W, 0u, rc.partial, red);
+            grid_sync(bar, epoch);
+            sq_from_bm_p2(qa, &cur->qlen, nbt, W, 0u, rc.partial, red);
+            mat = SM_SQUEUE;
+            filtered = qlen_changed = true;
+        }
+        if (filtered) grid_sync(bar, epoch);
+        if (is_book()) book_expand(book);
+
+        // ---------------- Expand
+        const bool fused = c.fused == GSW_FUSED;
+        unsigned *nnb = a.nb[(t + 1) % 3];
+        const SsClassify cl{nnb, a.farbit, th, fused, a.chg};
+        const bool use_q = push && fused && (long long)cv.ea <= (long long)(n >> 6);
+        LocalCnt lc;
+        if (push) {
+            const SsspPushOp op{dist, a.g.w, a.g.off, cl, use_q ? a.q[(t + 1) & 1] : nullptr, &nxt->qlen,
+                                a.fq[fcur], a.flen + fcur};
+            if (mat == SM_BITMAP) {
+                lc = run_lb(c.lb, BitmapSrc{nbt, (unsigned)n, 1u}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
+            } else {
+                const unsigned ql = qlen_changed ? cta_read_u32(&cur->qlen) : cv.qlen;
+                lc = run_lb(c.lb, QueueSrc{qa, ql}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
+            }
+        } else {
+            const SsspPullOp op{dist, a.g.in_w, nbt, a.g.off, cl, a.fq[fcur], a.flen + fcur};
+            lc = run_lb_reduce(c.lb, AllSrc{(unsigned)n}, adj_in, op, sm.pull, red, bar, epoch, rc.partial, a.scan);
+        }
+        dirty[(t + 1) % 3] = true;
+        if (fused) {
+            flush_counts(lc, nxt);
+            grid_sync(bar, epoch);
+            mat = use_q ? SM_QUEUE : SM_BITMAP;
+        } else {
+            // standalone Filter: classify the improved vertices of this round
+            LocalCnt ec;
+            ec.edges = lc.edges;
+            grid_sync(bar, epoch);
+            for (long long w = gwarp(); w < W; w += gwarps()) {
+                const unsigned m = a.chg[w];
+                const int v = (int)(w * 32 + lane_id());
+                bool near = false, far = false;
+                if ((m >> lane_id()) & 1u) {
+                    if ((unsigned long long)dist[v] < theta) {
+                        near = true;
+                        ec.add_vertex(__ldg(a.g.off + v + 1) - __ldg(a.g.off + v));
+                    } else {
+                        far = !(atomicOr(a.farbit + w, 1u << lane_id()) & (1u << lane_id()));
+                    }
+                }
+                const unsigned nm = __ballot_sync(0xffffffffu, near);
+                if (lane_id() == 0) { nnb[w] = nm; a.chg[w] = 0u; }
+                if (far) ec.aux++;
+                warp_append(a.fq[fcur], a.flen + fcur, far, v);
+            }
+            flush_counts(ec, nxt);
+            grid_sync(bar, epoch);
+            mat = SM_BITMAP;
+        }
+        prev_dir = c.dir;
+        prev_va = cv.va;
+    }
+    if (is_book()) book_finish(book, rc, t);
+}
+
+gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_stats *st) {
+    const int n = g->g.n, W = (n + 31) / 32;
+    if (!dist_out) { set_error("gsw_sssp: dist is NULL"); return GSW_EINVAL; }
+    if (source < 0 || source >= n) { set_error("gsw_sssp: source out of range"); return GSW_EINVAL; }
+    if (!g->g.w) { set_error("gsw_sssp: the graph has no weights"); return GSW_EINVAL; }
+    if ((double)g->attrs.maxw * (double)(n - 1) >= 4294967295.0) {
+        set_error("gsw_sssp: max_w * (n-1) does not fit the 32-bit distance type");
+        return GSW_EOVERFLOW;
+    }
+    Workspace ws{g->scratch, g->scratch_bytes, 0};
+    const bool dev_out = is_device_ptr(dist_out) == 1;
+    SsspArgs a{};
+    a.g = g->g;
+    a.src = source;
+    a.dist = dev_out ? dist_out : (unsigned *)ws.take((size_t)n * 4);
+    for (int i = 0; i < 3; ++i) a.nb[i] = (unsigned *)ws.take((size_t)W * 4);
+    for (int i = 0; i < 2; ++i) a.q[i] = (int *)ws.take((size_t)n * 4);
+    for (int i = 0; i < 2; ++i) a.fq[i] = (int *)ws.take((size_t)n * 4);
+    a.chg = (unsigned *)ws.take((size_t)W * 4);
+    a.farbit = (unsigned *)ws.take((size_t)W * 4);
+    a.flen = (unsigned *)ws.take(64);
+    a.split = (SplitCnt *)ws.take(2 * sizeof(SplitCnt));
+    a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
+    // P4 stepping mode and the static step delta0 = c*wbar/dbar (c = 32)
+    const gsw_config &fc = g->forced;
+    double dbar = g->attrs.dbar > 0 ? g->attrs.dbar : 1.0;
+    double d0 = fc.delta0 ? (double)fc.delta0 : 32.0 * g->attrs.wbar / dbar;
+    a.delta0 = (unsigned)std::max(1.0, std::min(d0, 2147483647.0));
+    switch (fc.stepping) {
+    case GSW_STEP_STATIC: a.mode = ST_STATIC; break;
+    case GSW_STEP_UNORDERED: a.mode = ST_UNORDERED; break;
+    case GSW_STEP_INCREASE: a.mode = ST_INC; break;
+    case GSW_STEP_DECREASE: a.mode = ST_DEC; break;
+    case GSW_STEP_REMAIN: a.mode = ST_REMAIN; break;
+    default: a.mode = ST_DYNAMIC;
+    }
+    LaunchInfo li;
+    gsw_status s = prepare_common(g, ws, (const void *)sssp_kernel, a.rc, li);
+    if (s != GSW_OK) return s;
+    if (!a.dist || !a.nb[2] || !a.q[1] || !a.fq[1] || !a.chg || !a.farbit || !a.flen || !a.split || !a.scan) {
+        set_error("workspace too small");
+        return GSW_ENOMEM;
+    }
+    void *args[] = {&a};
+    s = launch_persistent(g, (const void *)sssp_kernel, args, li);
+    if (s != GSW_OK) return s;
+    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(dist_out, a.dist, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
+    return finish_run(g, a.rc, li, st);
+}
+
+}  // namespace gsw

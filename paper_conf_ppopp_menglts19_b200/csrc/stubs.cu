@@ -2,7 +2,6 @@
 #include "launch.h"
 
 namespace gsw {
-gsw_status run_sssp(gsw_graph, int32_t, uint32_t *, gsw_run_stats *) { set_error("sssp: not built yet"); return GSW_EUNSUPPORTED; }
 
 gsw_status run_bc(gsw_graph, const int32_t *, int32_t, double *, gsw_run_stats *) { set_error("bc: not built yet"); return GSW_EUNSUPPORTED; }
 }  // namespace gsw
