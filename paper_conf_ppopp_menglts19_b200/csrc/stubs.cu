@@ -3,5 +3,4 @@
 
 namespace gsw {
 
-gsw_status run_bc(gsw_graph, const int32_t *, int32_t, double *, gsw_run_stats *) { set_error("bc: not built yet"); return GSW_EUNSUPPORTED; }
 }  // namespace gsw
