@@ -250,7 +250,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
                 }
             }
             const int lb = rc.force.load_balance ? rc.force.load_balance : GSW_LB_TWC;
-            const bool owner = lb == GSW_LB_THREAD || lb == GSW_LB_TWC;
+            const bool owner = lb == GSW_LB_THREAD || lb == GSW_LB_TWC || lb == GSW_LB_WM;
             const BcBackOp op{a.depth, a.sigma, a.omega, a.bc, a.dacc, lvl, owner};
             LocalCnt lc = run_lb_reduce(lb, QueueSrc{a.S + lo, hi - lo}, adj_out, op, sm.pull, red, bar, epoch,
                                         rc.partial, a.scan);

@@ -10,8 +10,9 @@
 //     void  flush(int x, Acc a, bool exclusive, LocalCnt&)   apply the reduced value to x;
 //           exclusive = this call carries the reduction of ALL of x's edges (owner mappings), else
 //           a partial that must be combined atomically (edge-parallel mappings: seg_reduce)
-//   THREAD and TWC (thread/warp/CTA tiers) own whole rows and flush once per row; WM, CM and STRICT
-//   split rows across lanes and flush per edge (STRICT merges runs of the same row first).
+//   THREAD, TWC (thread/warp/CTA tiers) and WM own whole rows and flush once per row (the TWC
+//   thread tier and WM reduce short rows with a warp-segmented scan); CM and STRICT split rows
+//   across threads and flush partials (STRICT merges runs of the same row first).
 #pragma once
 #include "lb.cuh"
 
@@ -27,6 +28,70 @@ __device__ __forceinline__ typename Op::Acc warp_combine(typename Op::Acc a) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) a = Op::combine(a, shfl_xor_any(a, o));
     return a;
+}
+
+// ------------------------------------------------------------------ warp-segmented row batch
+// A warp reduces the rows of its 32 lanes (lane r owns row x_r with edges [b_r, b_r + d_r)) edge-
+// parallel: the warp walks the concatenated edge list 64 edges at a time (two 32-edge chunks in
+// flight), each lane loads one edge per chunk, a 5-step segmented shuffle scan sums runs of the
+// same row, and lane r collects its row's run total.  All lanes stay busy regardless of the degree
+// mix (the per-thread serial loop idles lanes on skewed short rows).  Returns lane r's row total.
+template <class Op>
+__device__ __forceinline__ typename Op::Acc warp_seg_rows(const Op &op, const Adj &g, int x, uint32_t b, uint32_t d,
+                                                          LocalCnt &cnt) {
+    using Acc = typename Op::Acc;
+    const unsigned lane = lane_id();
+    const uint32_t incl = warp_incl_scan(d);
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    const uint32_t excl = incl - d;
+    Acc acc = Op::identity();
+    for (uint32_t k0 = 0; k0 < total; k0 += 64) {
+        uint32_t kk[2];
+        unsigned jj[2];
+        int xs[2], ys[2];
+        uint32_t es[2];
+        bool ok[2];
+        typename Op::Probe p[2];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            kk[h] = k0 + 32 * h + lane;
+            unsigned lo = 0, hi = 31;
+#pragma unroll
+            for (int s = 0; s < 5; ++s) {
+                unsigned mid = (lo + hi) >> 1;
+                uint32_t v = __shfl_sync(0xffffffffu, incl, mid);
+                if (v > kk[h]) hi = mid; else lo = mid + 1;
+            }
+            jj[h] = lo;
+            xs[h] = __shfl_sync(0xffffffffu, x, lo);
+            const uint32_t bb = __shfl_sync(0xffffffffu, b, lo), ex = __shfl_sync(0xffffffffu, excl, lo);
+            es[h] = bb + (kk[h] - ex);
+            ok[h] = kk[h] < total;
+        }
+#pragma unroll
+        for (int h = 0; h < 2; ++h) ys[h] = ok[h] ? __ldg(g.col + es[h]) : 0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) if (ok[h]) p[h] = op.probe(xs[h], es[h], ys[h]);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            Acc v = ok[h] ? op.val(xs[h], es[h], ys[h], p[h]) : Op::identity();
+            if (ok[h]) cnt.edges++;
+            // segmented inclusive scan over runs of equal row index
+#pragma unroll
+            for (int s = 1; s < 32; s <<= 1) {
+                Acc o = __shfl_up_sync(0xffffffffu, v, s);
+                unsigned oj = __shfl_up_sync(0xffffffffu, jj[h], s);
+                if (lane >= (unsigned)s && oj == jj[h]) v = Op::combine(v, o);
+            }
+            // row `lane` collects the run that ends inside this chunk
+            const uint32_t c0 = k0 + 32 * h, c1 = min(c0 + 32, total);
+            const uint32_t lo = max(excl, c0), hi = min(incl, c1);
+            const unsigned src = hi > lo ? hi - 1 - c0 : 0u;
+            Acc tv = __shfl_sync(0xffffffffu, v, src);
+            if (hi > lo) acc = Op::combine(acc, tv);
+        }
+    }
+    return acc;
 }
 
 // ------------------------------------------------------------------ THREAD (owner, ILP cursors)
@@ -170,34 +235,13 @@ __device__ __noinline__ LocalCnt lbr_twc(const Src src, const Adj g, Op op, TwcR
                 if ((int)lane == leader) op.flush(xx, a, true, cnt);
             }
         }
-        // thread tier: degree < 32, ILP cursors
-        Acc acc[kIlp];
+        // thread tier (degree < 32): the warp reduces its lanes' short rows edge-parallel
 #pragma unroll
-        for (int j = 0; j < kIlp; ++j) acc[j] = Op::identity();
-        bool own[kIlp];
-#pragma unroll
-        for (int j = 0; j < kIlp; ++j) own[j] = x[j] >= 0 && d0[j] < 32u && d0[j] > 0u;
-        for (;;) {
-            bool ok[kIlp], any = false;
-#pragma unroll
-            for (int j = 0; j < kIlp; ++j) { ok[j] = b[j] < e[j]; any |= ok[j]; }
-            if (!any) break;
-            int y[kIlp];
-            typename Op::Probe p[kIlp];
-#pragma unroll
-            for (int j = 0; j < kIlp; ++j) y[j] = ok[j] ? __ldg(g.col + b[j]) : 0;
-#pragma unroll
-            for (int j = 0; j < kIlp; ++j) if (ok[j]) p[j] = op.probe(x[j], b[j], y[j]);
-#pragma unroll
-            for (int j = 0; j < kIlp; ++j)
-                if (ok[j]) { cnt.edges++; acc[j] = Op::combine(acc[j], op.val(x[j], b[j], y[j], p[j])); ++b[j]; }
+        for (int j = 0; j < kIlp; ++j) {
+            const bool own = x[j] >= 0 && d0[j] < 32u;
+            const Acc r = warp_seg_rows(op, g, x[j], b[j], own ? d0[j] : 0u, cnt);
+            if (own && (d0[j] > 0u || Op::kFlushEmpty)) op.flush(x[j], r, true, cnt);
         }
-#pragma unroll
-        for (int j = 0; j < kIlp; ++j) if (own[j]) op.flush(x[j], acc[j], true, cnt);
-        // zero-degree items still get their (identity) flush so that owner-side updates happen
-#pragma unroll
-        for (int j = 0; j < kIlp; ++j)
-            if (x[j] >= 0 && d0[j] == 0u && Op::kFlushEmpty) op.flush(x[j], Op::identity(), true, cnt);
     }
     return cnt;
 }
@@ -228,31 +272,11 @@ __device__ __noinline__ LocalCnt lbr_wm(const Src src, const Adj g, Op op) {
         if (x >= 0 && op.skip(x)) x = -1;
         uint32_t b = 0, d = 0;
         if (x >= 0) { b = __ldg(g.off + x); d = __ldg(g.off + x + 1) - b; }
-        if (Op::kFlushEmpty && x >= 0 && d == 0) op.flush(x, Op::identity(), true, cnt);
-        const uint32_t incl = warp_incl_scan(d);
-        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-        const uint32_t excl = incl - d;
-        for (uint32_t k0 = 0; k0 < total; k0 += 64) {
-            int xs[2];
-            uint32_t es[2];
-            bool ok[2];
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                uint32_t k = k0 + 32 * h + lane;
-                unsigned lo = 0, hi = 31;
-#pragma unroll
-                for (int s = 0; s < 5; ++s) {
-                    unsigned mid = (lo + hi) >> 1;
-                    uint32_t v = __shfl_sync(0xffffffffu, incl, mid);
-                    if (v > k) hi = mid; else lo = mid + 1;
-                }
-                xs[h] = __shfl_sync(0xffffffffu, x, lo);
-                uint32_t bb = __shfl_sync(0xffffffffu, b, lo), ex = __shfl_sync(0xffffffffu, excl, lo);
-                es[h] = bb + (k - ex);
-                ok[h] = k < total;
-            }
-            red_edges<Op, 2>(op, g, xs, es, ok, cnt);
-        }
+        // WM: the warp's 32 consecutive rows, warpsize edges at a time, log2(32)-step
+        // search for each edge's row -- reduced per row and flushed by the row's lane
+        const typename Op::Acc r = warp_seg_rows(op, g, x, b, d, cnt);
+        (void)lane;
+        if (x >= 0 && (d > 0 || Op::kFlushEmpty)) op.flush(x, r, true, cnt);
     }
     return cnt;
 }

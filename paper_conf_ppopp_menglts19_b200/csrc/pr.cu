@@ -23,6 +23,8 @@ struct PrArgs {
     double *sum;          // accumulator for edge-parallel pull / push (zero between iterations)
     double *dsum;         // dangling mass D_t, iters+1 entries
     uint32_t *scan;
+    unsigned *heavy_cnt;
+    unsigned *heavy, *hblk;   // tiered pull: heavy rows and their block prefix
     RunCommon rc;
 };
 
@@ -78,6 +80,82 @@ struct PrPushOp {
     __device__ __forceinline__ bool commit(int, uint32_t, int, Tok, Aux, LocalCnt &) const { return false; }
 };
 
+// ---------------------------------------------------------------- B200 tiered pull (TWC)
+// TWC re-tiered for B200: rows < 32 edges are reduced 32 at a time by a
+// warp-segmented scan; rows of 32..kHeavy-1 edges by one warp with 4 loads in flight per lane;
+// rows >= kHeavy edges (R-MAT hubs, up to 163K edges at C3) are cut into kHeavy-edge blocks that
+// every warp of the grid shares (one fp64 atomic per block) and finished after a grid barrier.
+constexpr uint32_t kHeavy = 1024;
+
+struct PrTiers {
+    unsigned *heavy;        // heavy row ids
+    unsigned *hblk;         // exclusive prefix of ceil(d/kHeavy) over heavy rows (+ total)
+    unsigned nheavy;
+};
+
+__device__ __forceinline__ double warp_row_sum(const double *contrib, const int32_t *col, uint32_t b, uint32_t e,
+                                               unsigned long long &edges) {
+    const unsigned lane = lane_id();
+    double s = 0.0;
+    for (uint32_t k0 = b; k0 < e; k0 += 128) {
+        int y[4];
+        double c[4];
+#pragma unroll
+        for (int h = 0; h < 4; ++h) { uint32_t k = k0 + 32 * h + lane; y[h] = k < e ? __ldg(col + k) : -1; }
+#pragma unroll
+        for (int h = 0; h < 4; ++h) c[h] = y[h] >= 0 ? contrib[y[h]] : 0.0;
+#pragma unroll
+        for (int h = 0; h < 4; ++h) { s += c[h]; edges += y[h] >= 0; }
+    }
+    return warp_sum(s);
+}
+
+// phase A: heavy blocks (atomics into sum) + light/medium rows finished in place
+__device__ __noinline__ LocalCnt pr_pull_tiered_a(const PrPullOp op, const Adj g, const PrTiers tiers, int n) {
+    LocalCnt cnt;
+    const unsigned lane = lane_id();
+    const long long NW = gwarps();
+    // grid tier: kHeavy-edge blocks of heavy rows
+    const unsigned nblk = tiers.nheavy ? tiers.hblk[tiers.nheavy] : 0u;
+    for (long long blk = gwarp(); blk < nblk; blk += NW) {
+        // row r: last r with hblk[r] <= blk
+        unsigned lo = 0, hi = tiers.nheavy - 1;
+        while (lo < hi) { unsigned mid = (lo + hi + 1) >> 1; if (tiers.hblk[mid] <= blk) lo = mid; else hi = mid - 1; }
+        const unsigned v = tiers.heavy[lo];
+        const uint32_t rb = __ldg(g.off + v), re = __ldg(g.off + v + 1);
+        const uint32_t b = rb + (uint32_t)(blk - tiers.hblk[lo]) * kHeavy, e = min(re, b + kHeavy);
+        double s = warp_row_sum(op.contrib, g.col, b, e, cnt.edges);
+        if (lane == 0) atomicAdd(op.sum + v, s);
+    }
+    // light and medium rows: a warp takes 32 consecutive vertices
+    for (long long wb = gwarp() * 32; wb < n; wb += NW * 32) {
+        const int x = wb + lane < n ? (int)(wb + lane) : -1;
+        uint32_t b = 0, d = 0;
+        if (x >= 0) { b = __ldg(g.off + x); d = __ldg(g.off + x + 1) - b; }
+        const double r = warp_seg_rows(op, g, x, b, d < 32u ? d : 0u, cnt);
+        if (x >= 0 && d < 32u) op.epi.finish(x, r, cnt.facc);
+        unsigned med = __ballot_sync(0xffffffffu, x >= 0 && d >= 32u && d < kHeavy);
+        while (med) {
+            const int j = __ffs(med) - 1;
+            med &= med - 1;
+            const uint32_t bj = __shfl_sync(0xffffffffu, b, j), dj = __shfl_sync(0xffffffffu, d, j);
+            const double s = warp_row_sum(op.contrib, g.col, bj, bj + dj, cnt.edges);
+            if ((int)lane == j) op.epi.finish(x, s, cnt.facc);
+        }
+    }
+    return cnt;
+}
+
+// phase B (after a grid barrier): finish the heavy rows from their accumulated block sums
+__device__ __forceinline__ void pr_pull_tiered_b(const PrPullOp &op, const PrTiers &tiers, LocalCnt &cnt) {
+    for (long long i = gtid(); i < tiers.nheavy; i += gthreads()) {
+        const unsigned v = tiers.heavy[i];
+        const double s = op.sum[v];
+        op.sum[v] = 0.0;
+        op.epi.finish((int)v, s, cnt.facc);
+    }
+}
+
 __device__ __forceinline__ DevCfg select_pr(const Features &f, const gsw_config &force) {
     DevCfg c = select_traversal(f, force);
     // every vertex and edge is active: pull (atomic-free) with hub-aware TWC unless forced
@@ -125,8 +203,32 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
         if (a.iters == 0) a.out[v] = 1.0 / N;
     }
     for (long long i = gtid(); i <= a.iters; i += gthreads()) a.dsum[i] = 0.0;
+    if (is_book()) *a.heavy_cnt = 0u;
     grid_sync(bar, epoch);
     flush_dangling(dang, a.dsum);
+    // heavy-row table of the tiered pull (rows >= kHeavy in-edges): list, then block prefix
+    q_from_pred((int *)a.heavy, a.heavy_cnt, n,
+                [&](int v) { return __ldg(a.g.in_off + v + 1) - __ldg(a.g.in_off + v) >= kHeavy; });
+    grid_sync(bar, epoch);
+    PrTiers tiers{a.heavy, a.hblk, 0u};
+    tiers.nheavy = cta_read_u32(a.heavy_cnt);
+    if (blockIdx.x == 0) {
+        __shared__ uint32_t sred[kWarps + 1];
+        uint32_t base = 0;
+        for (unsigned t0 = 0; t0 < tiers.nheavy; t0 += kBlock) {
+            unsigned i = t0 + threadIdx.x;
+            uint32_t c = 0;
+            if (i < tiers.nheavy) {
+                unsigned v = tiers.heavy[i];
+                c = (__ldg(a.g.in_off + v + 1) - __ldg(a.g.in_off + v) + kHeavy - 1) / kHeavy;
+            }
+            uint32_t tot;
+            uint32_t ex = block_excl_scan(c, sred, &tot);
+            if (i < tiers.nheavy) tiers.hblk[i] = base + ex;
+            base += tot;
+        }
+        if (threadIdx.x == 0) tiers.hblk[tiers.nheavy] = base;
+    }
     grid_sync(bar, epoch);
 
     Book book;
@@ -156,8 +258,14 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
         if (is_book()) book_expand(book);
         LocalCnt lc;
         bool owner = false;
-        if (c.dir == GSW_PULL) {
-            owner = c.lb == GSW_LB_THREAD || c.lb == GSW_LB_TWC;
+        if (c.dir == GSW_PULL && c.lb == GSW_LB_TWC) {
+            const PrPullOp op{cur, a.sum, epi, true};
+            lc = pr_pull_tiered_a(op, adj_in, tiers, n);
+            grid_sync(bar, epoch);
+            pr_pull_tiered_b(op, tiers, lc);
+            owner = true;
+        } else if (c.dir == GSW_PULL) {
+            owner = c.lb == GSW_LB_THREAD || c.lb == GSW_LB_WM;
             const PrPullOp op{cur, a.sum, epi, owner};
             lc = run_lb_reduce(c.lb, AllSrc{(unsigned)n}, adj_in, op, sm.pull, red, bar, epoch, rc.partial, a.scan);
         } else {
@@ -204,10 +312,14 @@ gsw_status run_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_
     a.sum = (double *)ws.take((size_t)n * 8);
     a.dsum = (double *)ws.take((size_t)(iters + 1) * 8);
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
+    const size_t nh = std::min<size_t>((size_t)n, (size_t)g->g.nnz / kHeavy + 1);
+    a.heavy = (unsigned *)ws.take(nh * 4);
+    a.hblk = (unsigned *)ws.take((nh + 1) * 4);
+    a.heavy_cnt = (unsigned *)ws.take(256);
     LaunchInfo li;
     gsw_status s = prepare_common(g, ws, (const void *)pr_kernel, a.rc, li);
     if (s != GSW_OK) return s;
-    if (!a.out || !a.contrib[1] || !a.sum || !a.dsum || !a.scan) { set_error("workspace too small"); return GSW_ENOMEM; }
+    if (!a.out || !a.contrib[1] || !a.sum || !a.dsum || !a.scan || !a.heavy || !a.hblk || !a.heavy_cnt) { set_error("workspace too small"); return GSW_ENOMEM; }
     void *args[] = {&a};
     s = launch_persistent(g, (const void *)pr_kernel, args, li);
     if (s != GSW_OK) return s;
