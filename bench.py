@@ -156,6 +156,56 @@ def cpu_baseline_sample(g, roots, budget_s=12.0):
             "sample": f"{n} BFS roots on the full C3 graph, single-threaded oracle.bfs, {secs:.1f} s"}
 
 
+def run_extras(gsw, dev, G3, g3, peak):
+    """The other BASELINE.json configs (device time of one autotuned call, best of 3, L2 flushed
+    before each): C3 CC and PageRank (20 iterations, d = 0.85), C2 SSSP, C4 BC (16 sources)."""
+    import torch
+    import gen
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def best(fn):
+        b = None
+        for k in range(3):
+            flush.fill_(k)
+            torch.cuda.synchronize()
+            r = fn()
+            if b is None or r[1]["gpu_ms"] < b[1]["gpu_ms"]:
+                b = r
+        return b[1]
+
+    def rec(value, unit, st):
+        return {"value": value, "unit": unit, "gpu_ms": st["gpu_ms"], "iterations": st["iterations"],
+                "roofline_frac": st["bytes_alg"] / (st["gpu_ms"] * 1e-3) / 1e9 / peak,
+                "achieved_gbs": st["bytes_alg"] / (st["gpu_ms"] * 1e-3) / 1e9}
+
+    out = {}
+    st = best(lambda: G3.cc())
+    out["C3_cc"] = rec(g3.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
+    st = best(lambda: G3.pr(0.85, 20))
+    out["C3_pr"] = rec(20 / (st["gpu_ms"] * 1e-3), "PR iters/s", st)
+    g2 = gen.config_graph("C2")
+    G2 = gsw.Graph(g2.off, g2.col, g2.w, device=dev)
+    st = best(lambda: G2.sssp(0))
+    out["C2_sssp"] = rec(g2.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
+    out["C2_sssp"]["us_per_round"] = st["gpu_ms"] * 1e3 / max(1, st["iterations"])
+    del G2, g2
+    g4 = gen.config_graph("C4")
+    G4 = gsw.Graph(g4.off, g4.col, device=dev)
+    srcs = gen.sources(g4, 16)
+    st = best(lambda: G4.bc(srcs))
+    out["C4_bc"] = rec(16 * g4.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
+    del G4, g4
+    g1 = gen.config_graph("C1")
+    G1 = gsw.Graph(g1.off, g1.col, device=dev)
+    tot_ms, tot_e = 0.0, 0
+    for s in gen.sources(g1, 16):
+        d, st1 = G1.bfs(s)
+        tot_ms += st1["gpu_ms"]
+        tot_e += m_cc(g1.deg, d.cpu().numpy())
+    out["C1_bfs"] = {"value": tot_e / (tot_ms * 1e-3) / 1e9, "unit": "GTEPS", "gpu_ms_per_root": tot_ms / 16}
+    return out
+
+
 def run_gsw(args, ws, rank, local):
     import torch
     import torch.distributed as dist
@@ -191,14 +241,17 @@ def run_gsw(args, ws, rank, local):
     if ws > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    evs, kern_ms, bytes_alg, edges_cc = [], 0.0, 0, 0
+    evs, kern_ms, bytes_alg, edges_cc, g500_bytes = [], 0.0, 0, 0, 0
     with ClockSampler(local) as cs:
         for k in range(args.steps):
             e0, e1, st, s = step(args.warmup + k, True)
             evs.append((e0, e1))
             kern_ms += st["gpu_ms"]
             bytes_alg += st["bytes_alg"]
-            edges_cc += m_cc(deg, out.cpu().numpy())      # outside the [e0, e1] span
+            d = out.cpu().numpy()                             # outside the [e0, e1] span
+            mcc = m_cc(deg, d)
+            edges_cc += mcc
+            g500_bytes += 4 * 2 * mcc + 20 * int((d >= 0).sum())
     torch.cuda.synchronize()
     step_ms = [a.elapsed_time(b) for a, b in evs]
     tot_ms = sum(step_ms)
@@ -212,7 +265,13 @@ def run_gsw(args, ws, rank, local):
     peak, peak_src = hbm_peak()
     achieved = bytes_alg / (kern_ms * 1e-3) / 1e9
     # Graph500-equivalent bytes (full top-down): 4*nnz_cc + 20*N_cc per root (context only)
-    g500 = None
+    g500 = g500_bytes / (kern_ms * 1e-3) / 1e9
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "bfs_c3_traffic.json")
+    if os.path.exists(tf):
+        with open(tf) as f:
+            traffic = json.load(f).get("dram_bytes_per_launch")
+    extra = run_extras(gsw, dev, G, g, peak) if (rank == 0 and not args.quick) else None
 
     # ---- e2e: through the public API from pinned host buffers (graph H2D + BFS + depth D2H)
     e2e = None
@@ -249,13 +308,18 @@ def run_gsw(args, ws, rank, local):
                        "l2": "flushed between steps (256 MiB write outside the timed span)",
                        "parallelism": "replicas" if ws > 1 else "single GPU"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "gsw::bfs_kernel (persistent, 1 launch/step)",
-                         "bytes_model": "SURVEY 8(d) D0 per-level algorithmic bytes of the executed variant"},
+                         "bytes_model": "SURVEY 8(d) D0 per-level algorithmic bytes of the executed variant",
+                         "alg_bytes_per_launch": bytes_alg / args.steps,
+                         "traffic_unit": "DRAM bytes per launch (profiles/bfs_c3_traffic.json, ncu --set full)",
+                         "graph500_equiv": {"achieved": g500, "frac": g500 / peak,
+                                            "bytes_model": "4*nnz_cc + 20*N_cc per root (context)"}},
             "gpu_launches": args.steps,
             "e2e": e2e,
             "clocks": cs.summary(),
             "gen_seconds": gen_s,
+            "extra": extra,
         }
         if not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_baseline_sample(g, roots[:8])
@@ -272,6 +336,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gsw", choices=["gsw", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--quick", action="store_true", help="headline only (skip the other configs)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
