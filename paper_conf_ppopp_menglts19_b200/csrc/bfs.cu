@@ -47,8 +47,7 @@ struct BfsPushOp {
     const uint32_t *off;
     int lvl1;
     int fused;                // 0 standalone, 1 fused -> append to queue, 2 fused -> mark bitmap
-    int *nq;
-    unsigned *nqlen;
+    CtaQueue nq;              // CTA-staged append to the next queue
     unsigned *nfb;
     using Probe = unsigned;
     using Tok = ClaimTok;
@@ -70,8 +69,8 @@ struct BfsPushOp {
             depth[v] = lvl1;
             c.add_vertex(d.y - d.x);
             if (fused == 2) atomicOr(nfb + (v >> 5), 1u << (v & 31));
+            else if (fused == 1) nq.push(v);
         }
-        if (fused == 1) warp_append(nq, nqlen, won, v);
         return false;
     }
 };
@@ -181,8 +180,116 @@ __device__ __noinline__ LocalCnt bfs_pull_words(const unsigned *__restrict__ fb,
     return cnt;
 }
 
+// Pull over a per-warp compacted list of unvisited vertices (the THREAD candidate on the bitmap
+// format, B200 version): a warp compacts the zero bits of 16 visited-map words (512 vertices)
+// into shared memory, then every lane runs kPullCur independent cursors over its list entries;
+// a cursor that finishes (frontier parent found, or row exhausted) immediately refills from the
+// list, so a lane's time is the SUM of its scan lengths spread over kPullCur chains rather than
+// the maximum over a warp.  Each vertex has exactly one owner lane, so its visited / next-frontier
+// bits are set with fire-and-forget atomicOr (no returned value, no dependent round trip).
+constexpr int kPullCur = 4;
+constexpr int kPullWordsPerWarp = 16;
+constexpr int kPullList = kPullWordsPerWarp * 32;
+__device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, unsigned *__restrict__ V,
+                                               int *__restrict__ depth, const uint32_t *__restrict__ in_off,
+                                               const int32_t *__restrict__ in_col,
+                                               const uint32_t *__restrict__ out_off, bool symmetric, int lvl,
+                                               unsigned *__restrict__ nfb, int n, int *lists) {
+    LocalCnt cnt;
+    const int W = (n + 31) >> 5;
+    const unsigned lane = lane_id();
+    int *list = lists + (threadIdx.x >> 5) * (kPullList + kPullWordsPerWarp);
+    unsigned *found_bits = reinterpret_cast<unsigned *>(list + kPullList);
+    for (long long chunk = gwarp(); chunk * kPullWordsPerWarp < W; chunk += gwarps()) {
+        const long long w0 = chunk * kPullWordsPerWarp;
+        unsigned word = 0, orig = ~0u;
+        if (lane < (unsigned)kPullWordsPerWarp && w0 + lane < W) {
+            orig = V[w0 + lane];
+            word = ~orig;                                   // padding bits are set in V
+            found_bits[lane] = 0u;
+        }
+        const unsigned c = __popc(word);
+        const unsigned inc = warp_incl_scan(c);
+        const unsigned total = __shfl_sync(0xffffffffu, inc, 31);
+        unsigned pos = inc - c;
+        while (word) {
+            const int b = __ffs(word) - 1;
+            word &= word - 1;
+            list[pos++] = (int)((w0 + lane) * 32 + b);
+        }
+        __syncwarp();
+        // cursors: v < 0 = empty; st = 0 needs offsets, 1 scanning
+        int v[kPullCur];
+        uint32_t e[kPullCur], end[kPullCur], beg[kPullCur];
+        unsigned next = lane;
+#pragma unroll
+        for (int j = 0; j < kPullCur; ++j) {
+            v[j] = next < total ? list[next] : -1;
+            next += 32;
+        }
+#pragma unroll
+        for (int j = 0; j < kPullCur; ++j) {
+            beg[j] = e[j] = v[j] >= 0 ? __ldg(in_off + v[j]) : 0u;
+            end[j] = v[j] >= 0 ? __ldg(in_off + v[j] + 1) : 0u;
+        }
+        for (;;) {
+            bool any = false;
+#pragma unroll
+            for (int j = 0; j < kPullCur; ++j) any |= v[j] >= 0;
+            if (!any) break;
+            int y[kPullCur];
+            unsigned p[kPullCur];
+#pragma unroll
+            for (int j = 0; j < kPullCur; ++j) y[j] = (v[j] >= 0 && e[j] < end[j]) ? __ldg(in_col + e[j]) : -1;
+#pragma unroll
+            for (int j = 0; j < kPullCur; ++j) p[j] = y[j] >= 0 ? fb[y[j] >> 5] : 0u;
+            int nv[kPullCur];
+#pragma unroll
+            for (int j = 0; j < kPullCur; ++j) {
+                nv[j] = v[j];
+                if (v[j] < 0) continue;
+                bool done = false;
+                if (y[j] >= 0) {
+                    cnt.edges++;
+                    if ((p[j] >> (y[j] & 31)) & 1u) {
+                        const int x = v[j];
+                        depth[x] = lvl + 1;
+                        atomicOr(found_bits + ((x >> 5) - w0), 1u << (x & 31));   // shared memory
+                        cnt.add_vertex(symmetric ? end[j] - beg[j] : __ldg(out_off + x + 1) - __ldg(out_off + x));
+                        done = true;
+                    } else if (++e[j] >= end[j]) {
+                        done = true;
+                    }
+                } else {
+                    done = true;                     // empty row
+                }
+                if (done) { nv[j] = next < total ? list[next] : -1; next += 32; }
+            }
+            // refill: offsets of the newly taken entries
+#pragma unroll
+            for (int j = 0; j < kPullCur; ++j) {
+                if (nv[j] != v[j]) {
+                    v[j] = nv[j];
+                    beg[j] = e[j] = v[j] >= 0 ? __ldg(in_off + v[j]) : 0u;
+                    end[j] = v[j] >= 0 ? __ldg(in_off + v[j] + 1) : 0u;
+                }
+            }
+        }
+        __syncwarp();
+        // the warp owns its chunk's words: one store each for the visited map and AS_{t+1}
+        if (lane < (unsigned)kPullWordsPerWarp && w0 + lane < W) {
+            const unsigned fbits = found_bits[lane];
+            if (fbits) V[w0 + lane] = orig | fbits;
+            if (nfb) nfb[w0 + lane] = fbits;
+        }
+        __syncwarp();
+    }
+    return cnt;
+}
+
 __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
     __shared__ LbSmem sm;
+    __shared__ CtaQStore qs;
     __shared__ uint32_t red[kWarps + 1];
     const RunCommon &rc = a.rc;
     const GridBarrier bar = make_bar(rc);
@@ -205,6 +312,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
         rc.cnt[0].va = 1; rc.cnt[0].ea = dsrc; rc.cnt[0].maxd = dsrc; rc.cnt[0].mind = dsrc; rc.cnt[0].qlen = 1;
         a.q[0][0] = src;
     }
+    cta_queue_reset(qs);
     grid_sync(bar, epoch);
 
     Book book;
@@ -297,8 +405,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
         const bool mark_bitmap = (long long)ea > (long long)(n >> 6);
         const bool next_bitmap = !push || mark_bitmap;
         if (push) {
-            const BfsPushOp op{depth, a.V, a.g.off, t + 1, fused ? (mark_bitmap ? 2 : 1) : 0, a.q[(t + 1) & 1],
-                               &nxt->qlen, a.fb[(t + 1) % 3]};
+            const BfsPushOp op{depth, a.V, a.g.off, t + 1, fused ? (mark_bitmap ? 2 : 1) : 0,
+                               cta_queue(qs, a.q[(t + 1) & 1], &nxt->qlen), a.fb[(t + 1) % 3]};
             if (fused && mark_bitmap) dirty[(t + 1) % 3] = true;
             if (mat == MAT_BITMAP) {
                 lc = run_lb(c.lb, BitmapSrc{fbt, (unsigned)n, 1u}, adj_out, op, sm, red, bar, epoch, rc.partial, a.scan);
@@ -309,8 +417,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
         } else {
             const BfsPullOp op{depth, a.V, a.g.off, c.fmt == GSW_BITMAP ? fbt : nullptr, t, fused, a.fb[(t + 1) % 3]};
             if (c.fmt == GSW_BITMAP && c.lb == GSW_LB_THREAD) {
-                lc = bfs_pull_words(fbt, a.V, depth, a.g.in_off, a.g.in_col, a.g.off, a.g.in_off == a.g.off, t,
-                                    fused ? a.fb[(t + 1) % 3] : nullptr, n);
+                static_assert(sizeof(LbSmem) >= sizeof(int) * (kPullList + kPullWordsPerWarp) * kWarps, "pull lists live in the LB smem");
+                lc = bfs_pull_list(fbt, a.V, depth, a.g.in_off, a.g.in_col, a.g.off, a.g.in_off == a.g.off, t,
+                                   fused ? a.fb[(t + 1) % 3] : nullptr, n, reinterpret_cast<int *>(&sm));
             } else if (c.fmt == GSW_BITMAP) {
                 lc = run_lb(c.lb, BitmapSrc{a.V, (unsigned)n, 0u}, adj_in, op, sm, red, bar, epoch, rc.partial, a.scan);
             } else {
@@ -319,6 +428,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
             }
             if (fused) dirty[(t + 1) % 3] = true;
         }
+        if (push && fused && !mark_bitmap) cta_queue_flush(qs, a.q[(t + 1) & 1], &nxt->qlen);
         flush_counts(lc, nxt);
         grid_sync(bar, epoch);
         mat = fused ? (next_bitmap ? MAT_BITMAP : MAT_QUEUE) : MAT_NONE;
