@@ -4,8 +4,9 @@ PKG := paper_conf_ppopp_menglts19_b200
 CSRC := $(PKG)/csrc
 CU := $(wildcard $(CSRC)/*.cu)
 HDR := $(wildcard $(CSRC)/*.cuh $(CSRC)/*.h) include/gsw.h
+NCCL_INC ?= $(shell python3 -c "import nvidia.nccl, os; print(os.path.join(list(nvidia.nccl.__path__)[0], 'include'))" 2>/dev/null)
 NVFLAGS := -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 \
-           -Xcompiler -fPIC -Iinclude -I$(CSRC) --expt-relaxed-constexpr -Xptxas -v
+           -Xcompiler -fPIC -Iinclude -I$(CSRC) -I$(NCCL_INC) --expt-relaxed-constexpr -Xptxas -v
 LIB := $(PKG)/libgsw.so
 OBJDIR := build/obj
 OBJ := $(patsubst $(CSRC)/%.cu,$(OBJDIR)/%.o,$(CU))
@@ -17,7 +18,7 @@ $(OBJDIR)/%.o: $(CSRC)/%.cu $(HDR)
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> $(OBJDIR)/$*.ptxas.txt || (cat $(OBJDIR)/$*.ptxas.txt; exit 1)
 
 $(LIB): $(OBJ)
-	$(NVCC) -gencode arch=compute_100a,code=sm_100a -shared -o $@ $(OBJ) -lcudart
+	$(NVCC) -gencode arch=compute_100a,code=sm_100a -shared -o $@ $(OBJ) -lcudart -ldl
 
 gen/libgswgen.so: gen/gen.c
 	gcc -O3 -fopenmp -fPIC -shared -o $@ $< -lm

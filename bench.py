@@ -206,7 +206,9 @@ def run_extras(gsw, dev, G3, g3, peak):
     return out
 
 
-def run_gsw(args, ws, rank, local):
+def run_gsw_dist(args, ws, rank, local):
+    """N > 1: the C3 graph 1D vertex-partitioned over N ranks (one per GPU), BFS with per-level
+    NCCL bitmap all-gather + feature all-reduce inside the library (strong scaling: fixed graph)."""
     import torch
     import torch.distributed as dist
     import gen
@@ -214,8 +216,74 @@ def run_gsw(args, ws, rank, local):
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
+    if "RANK" not in os.environ:                       # --force-dist without torchrun
+        os.environ.update(RANK="0", WORLD_SIZE="1", LOCAL_RANK="0", MASTER_ADDR="127.0.0.1",
+                          MASTER_PORT=str(29500 + os.getpid() % 1000))
+    dist.init_process_group("nccl", device_id=dev)
+    g, gen_s = build_graph("C3")
+    deg = g.deg
+    nroots = max(64, args.steps + args.warmup)
+    roots = gen.sources(g, nroots)
+    obj = [gsw.dist_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0)
+    off, col = gsw.owned_rows(g.off, g.col, rank, ws)
+    D = gsw.DistGraph(off, col, g.n, obj[0], ws, rank, device=dev)
+    S = gsw.dist_slice(g.n, ws)
+    out = torch.empty(D.out_len, dtype=torch.int32, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    for k in range(args.warmup):
+        D.bfs(roots[k % nroots], out=out)
+    torch.cuda.synchronize()
+    dist.barrier()
+    tot_ms, edges_cc, bytes_alg, launches = 0.0, 0, 0, 0
+    with ClockSampler(local) as cs:
+        for k in range(args.steps):
+            flush.fill_(k & 0xff)
+            torch.cuda.synchronize()
+            dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(D.stream)
+            _, st = D.bfs(roots[(args.warmup + k) % nroots], out=out)
+            e1.record(D.stream)
+            torch.cuda.synchronize()
+            ms = torch.tensor([e0.elapsed_time(e1)], device=dev)
+            dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+            tot_ms += float(ms.item())
+            bytes_alg += st["bytes_alg"]
+            launches += 3 * st["iterations"] + 4          # init + per level: expand, count-sum (+NCCL)
+            # m_cc from the owned slices (sum over ranks)
+            loc = torch.tensor([int(deg[rank * S:rank * S + D.out_len][out.cpu().numpy() >= 0].sum())], device=dev)
+            dist.all_reduce(loc)
+            edges_cc += int(loc.item()) // 2
+    peak, peak_src = hbm_peak()
+    if rank == 0:
+        line = {
+            "metric": "BFS GTEPS", "value": edges_cc / (tot_ms * 1e-3) / 1e9, "unit": "GTEPS", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": f"C3: BFS on R-MAT scale 22 ef 16, n={g.n}, nnz={g.nnz}, 1D vertex partition "
+                                   f"over {ws} ranks (slice {S}), per-level NCCL bitmap all-gather",
+                       "l2": "flushed between steps", "parallelism": f"1D vertex partition x{ws} (NCCL)"},
+            "roofline": {"bound": "hbm", "achieved": bytes_alg / (tot_ms * 1e-3) / 1e9 / ws, "peak": peak,
+                         "unit": "GB/s", "frac": bytes_alg / (tot_ms * 1e-3) / 1e9 / ws / peak, "traffic": None,
+                         "peak_source": peak_src, "kernel": "gsw k_bfs_push/k_bfs_pull (per level) + NCCL"},
+            "gpu_launches": launches, "clocks": cs.summary(), "gen_seconds": gen_s,
+        }
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def run_gsw(args, ws, rank, local):
+    import torch
+    import torch.distributed as dist
+    import gen
+    import paper_conf_ppopp_menglts19_b200 as gsw
+
+    if ws > 1 or args.force_dist:
+        return run_gsw_dist(args, ws, rank, local)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
     g, gen_s = build_graph("C3")
     deg = g.deg
     nroots = max(64, args.steps + args.warmup)
@@ -337,6 +405,7 @@ def main():
     ap.add_argument("--impl", default="gsw", choices=["gsw", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--quick", action="store_true", help="headline only (skip the other configs)")
+    ap.add_argument("--force-dist", action="store_true", help="run the partitioned NCCL path even at N=1")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

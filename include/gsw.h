@@ -157,6 +157,39 @@ gsw_status gsw_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_
 gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc,
                   gsw_run_stats *stats);
 
+/* ---------------------------------------------------------------------------------------------
+ * Multi-GPU: 1D vertex partition (the paper itself is single-GPU).  Rank r of p owns
+ * the vertex slice [r*S, min(n,(r+1)*S)) with S = gsw_dist_slice(n, p) (a multiple of 64, equal
+ * for every rank as NCCL collectives need equal counts).  Every write lands on an owned vertex, so
+ * no cross-GPU atomics are needed.  Per BFS level a rank expands into its owned slice of the next
+ * frontier bitmap (pull: owned rows = in-edges of owned vertices; push: the column slice "global
+ * source -> owned targets" built at create time), then an in-place ncclAllGather of the bitmap
+ * slices (n/8 bytes total) and an ncclAllReduce of the 16-byte feature counts give every rank the
+ * same frontier and the same selector decision.  PageRank all-gathers the fp64 contributions and
+ * all-reduces the dangling mass each iteration.  NCCL is loaded at run time (dlopen); without it
+ * the NCCL calls return GSW_ENCCL.  Supported on distributed handles: gsw_bfs, gsw_pr (others
+ * return GSW_EUNSUPPORTED).  Outputs of distributed handles cover the OWNED slice only.
+ * ------------------------------------------------------------------------------------------- */
+/* Slice size S for n vertices over p ranks. */
+int64_t gsw_dist_slice(int64_t n, int32_t nranks);
+/* Fill 128 bytes with a new ncclUniqueId (call on one rank, broadcast the bytes to the others). */
+gsw_status gsw_dist_unique_id(void *id128);
+/* Workspace bytes for a partition of n_global vertices with nnz_owned adjacency entries. */
+gsw_status gsw_dist_workspace_size(int64_t n_global, int64_t nnz_owned, int32_t nranks, size_t *bytes);
+/* NCCL mode (one process per GPU).  owned: the rows of the owned slice -- owned->n = number of
+ * owned vertices, row_offsets start at 0, col_indices are GLOBAL ids (symmetric graph).
+ * Collective over all ranks (same call order on every rank).  Errors: GSW_EINVAL (slice size
+ * mismatch), GSW_ENCCL (communicator creation failed). */
+gsw_status gsw_graph_create_dist(const gsw_csr *owned, int64_t n_global, const void *nccl_id128,
+                                 int32_t nranks, int32_t rank, void *workspace, size_t ws_bytes,
+                                 void *cuda_stream, gsw_graph *out);
+/* Loopback mode: `nparts` virtual ranks of the full symmetric graph on THIS GPU, exchanging
+ * through device memory in stream order (the same partitioned kernels as NCCL mode; used to test
+ * the partitioned path on one GPU).  Outputs cover all n vertices. */
+gsw_status gsw_dist_loopback_workspace_size(int64_t n, int64_t nnz, int32_t nparts, size_t *bytes);
+gsw_status gsw_graph_create_partitioned(const gsw_csr *csr, int32_t nparts, void *workspace,
+                                        size_t ws_bytes, void *cuda_stream, gsw_graph *out);
+
 /* Thread-local message for the last non-OK status of this thread. */
 const char *gsw_last_error(void);
 /* Library version string. */

@@ -151,7 +151,7 @@ class Graph:
     def _out(self, out, dtype):
         import torch
         if out is None:
-            return torch.empty(self.n, dtype=dtype, device=self.device)
+            return torch.empty(getattr(self, "out_len", self.n), dtype=dtype, device=self.device)
         return out
 
     def bfs(self, source: int, out=None, records: int = 0):
@@ -192,3 +192,100 @@ class Graph:
         check(_lib.load().gsw_bc(self._h, src.ctypes.data if src.size else None, int(src.size), out.data_ptr(),
                                  ctypes.byref(st)), "gsw_bc")
         return out, _stats_dict(st, recs)
+
+
+# ------------------------------------------------------------------------------------------------
+# Multi-GPU: 1D vertex partition (include/gsw.h "Multi-GPU").  BFS and PageRank run on these
+# handles; outputs cover the owned slice (NCCL mode) or all vertices (loopback mode).
+
+def dist_slice(n: int, nranks: int) -> int:
+    """Slice size S: rank r owns vertices [r*S, min(n, (r+1)*S))."""
+    return int(_lib.load().gsw_dist_slice(int(n), int(nranks)))
+
+
+def dist_unique_id() -> bytes:
+    """A fresh 128-byte ncclUniqueId (create on one rank, broadcast to the others)."""
+    buf = ctypes.create_string_buffer(128)
+    check(_lib.load().gsw_dist_unique_id(buf), "gsw_dist_unique_id")
+    return buf.raw
+
+
+class _Handle(Graph):
+    """Shared methods of the partitioned handles (bfs, pr, force_config come from Graph)."""
+
+    def __init__(self):   # noqa: D401 -- constructed by the subclasses
+        pass
+
+
+class DistGraph(_Handle):
+    """NCCL mode: this process owns rows [rank*S, rank*S + n_owned) of an n_global-vertex
+    symmetric graph (global column ids).  Collective: every rank constructs it in the same order."""
+
+    def __init__(self, owned_offsets, owned_cols, n_global: int, nccl_id: bytes, nranks: int, rank: int,
+                 device: str | int = "cuda", stream=None):
+        import torch
+        lib = _lib.load()
+        self.device = torch.device(device)
+        off = _as(owned_offsets, np.int64, torch.int64)
+        col = _as(owned_cols, np.int32, torch.int32)
+        self.n = int(n_global)
+        self.out_len = int(off.shape[0]) - 1
+        self.nnz = int(col.shape[0])
+        self.rank, self.nranks = int(rank), int(nranks)
+        with torch.cuda.device(self.device):
+            self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+            po, ko, _ = _ptr_of(off)
+            pc, kc, _ = _ptr_of(col) if self.nnz else (None, None, False)
+            csr = _lib.gsw_csr(self.out_len, self.nnz, po, pc, None)
+            nbytes = ctypes.c_size_t()
+            check(lib.gsw_dist_workspace_size(self.n, self.nnz, self.nranks, ctypes.byref(nbytes)),
+                  "gsw_dist_workspace_size")
+            self.workspace = torch.empty(nbytes.value, dtype=torch.uint8, device=self.device)
+            idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
+            h = ctypes.c_void_p()
+            check(lib.gsw_graph_create_dist(ctypes.byref(csr), self.n, idbuf, self.nranks, self.rank,
+                                            self.workspace.data_ptr(), nbytes.value, self.stream.cuda_stream,
+                                            ctypes.byref(h)), "gsw_graph_create_dist")
+            self._h = h
+            del ko, kc
+
+
+class PartitionedGraph(_Handle):
+    """Loopback mode: `nparts` virtual ranks of the full graph on this GPU, running the same
+    partitioned kernels as DistGraph with the exchange done in device memory."""
+
+    def __init__(self, row_offsets, col_indices, nparts: int, device: str | int = "cuda", stream=None):
+        import torch
+        lib = _lib.load()
+        self.device = torch.device(device)
+        off = _as(row_offsets, np.int64, torch.int64)
+        col = _as(col_indices, np.int32, torch.int32)
+        self.n = int(off.shape[0]) - 1
+        self.out_len = self.n
+        self.nnz = int(col.shape[0])
+        self.nparts = int(nparts)
+        with torch.cuda.device(self.device):
+            self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+            po, ko, _ = _ptr_of(off)
+            pc, kc, _ = _ptr_of(col) if self.nnz else (None, None, False)
+            csr = _lib.gsw_csr(self.n, self.nnz, po, pc, None)
+            nbytes = ctypes.c_size_t()
+            check(lib.gsw_dist_loopback_workspace_size(self.n, self.nnz, self.nparts, ctypes.byref(nbytes)),
+                  "gsw_dist_loopback_workspace_size")
+            self.workspace = torch.empty(nbytes.value, dtype=torch.uint8, device=self.device)
+            h = ctypes.c_void_p()
+            check(lib.gsw_graph_create_partitioned(ctypes.byref(csr), self.nparts, self.workspace.data_ptr(),
+                                                   nbytes.value, self.stream.cuda_stream, ctypes.byref(h)),
+                  "gsw_graph_create_partitioned")
+            self._h = h
+            del ko, kc
+
+
+def owned_rows(row_offsets, col_indices, rank: int, nranks: int):
+    """Rows [rank*S, min(n, (rank+1)*S)) of a CSR as (offsets rebased to 0, global columns)."""
+    off = np.asarray(row_offsets, dtype=np.int64)
+    n = off.shape[0] - 1
+    S = dist_slice(n, nranks)
+    vb, ve = min(n, rank * S), min(n, (rank + 1) * S)
+    loc = off[vb:ve + 1] - off[vb]
+    return loc, np.asarray(col_indices)[off[vb]:off[ve]]

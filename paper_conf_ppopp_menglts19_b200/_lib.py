@@ -71,6 +71,16 @@ SIGNATURES = {
     "gsw_cc": (ctypes.c_int, [_P, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_pr": (ctypes.c_int, [_P, ctypes.c_double, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_bc": (ctypes.c_int, [_P, _P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
+    "gsw_dist_slice": (ctypes.c_int64, [ctypes.c_int64, ctypes.c_int32]),
+    "gsw_dist_unique_id": (ctypes.c_int, [_P]),
+    "gsw_dist_workspace_size": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32,
+                                               ctypes.POINTER(ctypes.c_size_t)]),
+    "gsw_graph_create_dist": (ctypes.c_int, [ctypes.POINTER(gsw_csr), ctypes.c_int64, _P, ctypes.c_int32,
+                                             ctypes.c_int32, _P, ctypes.c_size_t, _P, ctypes.POINTER(_P)]),
+    "gsw_dist_loopback_workspace_size": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32,
+                                                        ctypes.POINTER(ctypes.c_size_t)]),
+    "gsw_graph_create_partitioned": (ctypes.c_int, [ctypes.POINTER(gsw_csr), ctypes.c_int32, _P, ctypes.c_size_t,
+                                                    _P, ctypes.POINTER(_P)]),
     "gsw_last_error": (ctypes.c_char_p, []),
     "gsw_version": (ctypes.c_char_p, []),
 }

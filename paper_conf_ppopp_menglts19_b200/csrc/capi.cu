@@ -23,6 +23,20 @@ gsw_status load_csr(gsw_graph g, const gsw_csr *c, Workspace &ws, uint32_t **off
                     int64_t *staging);
 gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp);
 gsw_status validate_graph(gsw_graph g);
+// dist.cu
+int64_t dist_slice(int64_t n, int32_t p);
+gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int32_t nranks, int32_t rank,
+                       bool loopback, void *workspace, size_t ws_bytes, void *stream, gsw_graph *out);
+void dist_destroy(DistState *d);
+gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stats *st);
+gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out, gsw_run_stats *st);
+size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, bool own_copy);
+gsw_status dist_unique_id(void *id128);
+
+static gsw_status no_dist(gsw_graph g, const char *what) {
+    if (g->dist) { set_error(std::string(what) + ": not supported on a distributed handle"); return GSW_EUNSUPPORTED; }
+    return GSW_OK;
+}
 
 static gsw_status check_csr(const gsw_csr *c, const char *what) {
     if (!c) { set_error(std::string(what) + " is NULL"); return GSW_EINVAL; }
@@ -127,12 +141,14 @@ gsw_status gsw_graph_destroy(gsw_graph g) {
     if (!g) return GSW_OK;
     if (g->ev0) cudaEventDestroy(g->ev0);
     if (g->ev1) cudaEventDestroy(g->ev1);
+    dist_destroy(g->dist);
     delete g;
     return GSW_OK;
 }
 
 gsw_status gsw_graph_validate(gsw_graph g) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (gsw_status s = no_dist(g, "gsw_graph_validate")) return s;
     return validate_graph(g);
 }
 
@@ -159,27 +175,61 @@ gsw_status gsw_force_config(gsw_graph g, const gsw_config *cfg) {
 
 gsw_status gsw_bfs(gsw_graph g, int32_t source, int32_t *depth, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (g->dist) return dist_bfs(g, source, depth, stats);
     return run_bfs(g, source, depth, stats);
 }
 
 gsw_status gsw_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (gsw_status s = no_dist(g, "gsw_sssp")) return s;
     return run_sssp(g, source, dist, stats);
 }
 
 gsw_status gsw_cc(gsw_graph g, int32_t *label, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (gsw_status s = no_dist(g, "gsw_cc")) return s;
     return run_cc(g, label, stats);
 }
 
 gsw_status gsw_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (g->dist) return dist_pr(g, damping, iters, rank, stats);
     return run_pr(g, damping, iters, rank, stats);
 }
 
 gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (gsw_status s = no_dist(g, "gsw_bc")) return s;
     return run_bc(g, sources, nsrc, bc, stats);
+}
+
+int64_t gsw_dist_slice(int64_t n, int32_t nranks) { return (n > 0 && nranks > 0) ? dist_slice(n, nranks) : 0; }
+
+gsw_status gsw_dist_unique_id(void *id128) { return dist_unique_id(id128); }
+
+gsw_status gsw_dist_workspace_size(int64_t n_global, int64_t nnz_owned, int32_t nranks, size_t *bytes) {
+    if (!bytes || n_global <= 0 || nnz_owned < 0 || nranks < 1) { set_error("gsw_dist_workspace_size: bad arguments"); return GSW_EINVAL; }
+    *bytes = dist_workspace(n_global, nnz_owned, nranks, 1, true);
+    return GSW_OK;
+}
+
+gsw_status gsw_dist_loopback_workspace_size(int64_t n, int64_t nnz, int32_t nparts, size_t *bytes) {
+    if (!bytes || n <= 0 || nnz < 0 || nparts < 1) { set_error("gsw_dist_loopback_workspace_size: bad arguments"); return GSW_EINVAL; }
+    *bytes = dist_workspace(n, nnz, nparts, nparts, false);
+    return GSW_OK;
+}
+
+gsw_status gsw_graph_create_dist(const gsw_csr *owned, int64_t n_global, const void *nccl_id128, int32_t nranks,
+                                 int32_t rank, void *workspace, size_t ws_bytes, void *cuda_stream, gsw_graph *out) {
+    if (!out) { set_error("out is NULL"); return GSW_EINVAL; }
+    if (nranks > 1 && !nccl_id128) { set_error("nccl_id128 is NULL"); return GSW_EINVAL; }
+    return dist_create(owned, n_global, nccl_id128, nranks, rank, false, workspace, ws_bytes, cuda_stream, out);
+}
+
+gsw_status gsw_graph_create_partitioned(const gsw_csr *csr, int32_t nparts, void *workspace, size_t ws_bytes,
+                                        void *cuda_stream, gsw_graph *out) {
+    if (!out || !csr) { set_error("null argument"); return GSW_EINVAL; }
+    return dist_create(csr, csr->n, nullptr, nparts, 0, true, workspace, ws_bytes, cuda_stream, out);
 }
 
 }  // extern "C"

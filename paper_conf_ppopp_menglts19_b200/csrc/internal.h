@@ -48,7 +48,12 @@ struct Workspace {
 
 }  // namespace gsw
 
+namespace gsw {
+struct DistState;
+}
+
 struct gsw_graph_s {
+    gsw::DistState *dist = nullptr;   // multi-GPU / partitioned handle (dist.cu), else nullptr
     gsw::DevGraph g{};
     gsw::Attrs attrs{};
     bool symmetric = true;
