@@ -207,9 +207,13 @@ __device__ __noinline__ LocalCnt lb_wm(const Src src, const Adj g, Op op) {
     LocalCnt cnt;
     const unsigned sz = src.size();
     const unsigned lane = lane_id();
-    for (long long wb = gwarp() * 32; wb < sz; wb += gwarps() * 32) {
+    // items per warp: up to warpsize; fewer when the active set cannot fill every warp
+    // of the grid, so that small frontiers are spread over all SMs (one edge per lane)
+    const long long NW = gwarps();
+    const unsigned ipw = (unsigned)max(1LL, min(32LL, ((long long)sz + NW - 1) / NW));
+    for (long long wb = gwarp() * ipw; wb < sz; wb += NW * ipw) {
         long long i = wb + lane;
-        int x = i < sz ? src.get((unsigned)i) : -1;
+        int x = (lane < ipw && i < sz) ? src.get((unsigned)i) : -1;
         if (x >= 0 && op.skip(x)) x = -1;
         uint32_t b = 0, d = 0;
         if (x >= 0) { b = __ldg(g.off + x); d = __ldg(g.off + x + 1) - b; }

@@ -39,6 +39,7 @@ __device__ __forceinline__ int pick(int forced, int chosen) { return forced != G
 // split is  pull <=> Ea * kPullAlpha > Eia  and  Va * kPullBeta > N   (reading R6).
 constexpr float kPullAlpha = 16.f;
 constexpr float kPullBeta = 1024.f;
+constexpr long long kTwcMinActive = 148LL * 4 * kBlock * 4;   // items that fill every TWC tile once
 
 __device__ __forceinline__ int traversal_direction(const Features &f) {
     return ((float)f.Ea * kPullAlpha > (float)f.Eia && (float)f.Va * kPullBeta > f.N) ? GSW_PULL : GSW_PUSH;
@@ -51,10 +52,12 @@ __device__ __forceinline__ DevCfg select_traversal(const Features &f, const gsw_
     // P3 load balance: "TWC has the lowest overhead", "CM and WM perform better with irregular
     // workloads", "when the workload contains a hub vertex ... STRICT is the best".
     // Pull with early exit scans ~1-2 edges per vertex, so the per-thread mapping wins on B200.
+    // On B200 TWC's tiles (blockDim x 4 items per CTA) only pay once the active set fills the
+    // grid; below that WM with adaptive items per warp spreads the edges over every SM.
     int lb;
     if (c.dir == GSW_PULL) lb = GSW_LB_THREAD;
-    else if (f.Ea <= 8192 && f.maxd <= 1024u) lb = GSW_LB_WM;               // tiny, latency-bound
     else if (f.maxd > 1024u || cd > 64.f) lb = GSW_LB_STRICT;                // hub in workload
+    else if (f.Va < kTwcMinActive) lb = GSW_LB_WM;                           // latency-bound
     else lb = GSW_LB_TWC;                                                    // regular degrees
     c.lb = pick(force.load_balance, lb);
     // P2 format: "bitmap is more friendly to dense workloads, the unsorted queue is more friendly

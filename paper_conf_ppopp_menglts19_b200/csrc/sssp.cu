@@ -66,10 +66,9 @@ struct SsspPushOp {
     const uint32_t *w;
     const uint32_t *off;
     SsClassify cl;
-    int *nq;              // next near queue (fused, few claims) or nullptr (bitmap marking)
-    unsigned *nqlen;
-    int *fq;
-    unsigned *fqlen;
+    bool use_q;           // next near set as a queue (fused, few claims) or bitmap marking only
+    CtaQueue nq;          // CTA-staged appends (common.cuh)
+    CtaQueue fq;
     using Probe = uint2;  // (dist[u] + w(u,v), dist[v])
     using Tok = SsTok;
     using Aux = SsAux;
@@ -97,10 +96,14 @@ struct SsspPushOp {
     __device__ __forceinline__ bool commit(int, uint32_t, int v, Tok, Aux a, LocalCnt &c) const {
         const unsigned bit = 1u << (v & 31);
         const bool nw = !(a.nclaim & bit), fw = !(a.fclaim & bit);
-        if (nw) c.add_vertex(a.d1 - a.d0);
-        if (nq) warp_append(nq, nqlen, nw, v);
-        if (fw) c.aux++;
-        warp_append(fq, fqlen, fw, v);
+        if (nw) {
+            c.add_vertex(a.d1 - a.d0);
+            if (use_q) nq.push(v);
+        }
+        if (fw) {
+            c.aux++;
+            fq.push(v);
+        }
         return false;
     }
 };
@@ -112,8 +115,7 @@ struct SsspPullOp {
     const unsigned *nbt;      // near set N_t
     const uint32_t *off;      // out-offsets
     SsClassify cl;
-    int *fq;
-    unsigned *fqlen;
+    CtaQueue fq;
     using Probe = uint2;      // (near word of u, dist[u])
     using Acc = unsigned long long;
     static constexpr bool kFlushEmpty = false;
@@ -137,7 +139,7 @@ struct SsspPullOp {
             if (!(atomicOr(cl.nnb + (v >> 5), bit) & bit)) c.add_vertex(__ldg(off + v + 1) - __ldg(off + v));
         } else if (!(atomicOr(cl.farbit + (v >> 5), bit) & bit)) {
             c.aux++;
-            fq[atomicAdd(fqlen, 1u)] = v;
+            fq.push(v);
         }
     }
 };
@@ -156,6 +158,7 @@ union SsSmem {
 __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
     __shared__ SsSmem sm;
     __shared__ uint32_t red[kWarps + 1];
+    __shared__ CtaQStore qs0, qs1;        // staged appends: near queue, far queue
     const RunCommon &rc = a.rc;
     const GridBarrier bar = make_bar(rc);
     unsigned epoch = 0;
@@ -177,6 +180,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
         a.flen[0] = 0u; a.flen[1] = 0u;
         for (int i = 0; i < 2; ++i) { a.split[i] = SplitCnt{0ull, 0ull, 0u, 0u, 0xffffffffu, 0u}; }
     }
+    cta_queue_reset(qs0);
+    cta_queue_reset(qs1);
     grid_sync(bar, epoch);
 
     Book book;
@@ -216,20 +221,22 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
             LocalCnt lc;
             unsigned lmin = 0xffffffffu;
             int *qa = a.q[t & 1];
-            for (long long base = gwarp() * 32; base < L; base += gwarps() * 32) {
-                long long i = base + lane_id();
-                int v = i < L ? a.fq[fsrc][i] : -1;
-                unsigned dv = v >= 0 ? dist[v] : 0xffffffffu;
-                bool to_near = v >= 0 && (unsigned long long)dv < theta;
-                bool keep = v >= 0 && !to_near;
-                if (to_near) {
+            const CtaQueue qn = cta_queue(qs0, qa, &sp->qlen), qk = cta_queue(qs1, a.fq[fdst], a.flen + fdst);
+            for (long long i = gtid(); i < L; i += gthreads()) {
+                const int v = a.fq[fsrc][i];
+                const unsigned dv = dist[v];
+                if ((unsigned long long)dv < theta) {
                     atomicAnd(a.farbit + (v >> 5), ~(1u << (v & 31)));
                     lc.add_vertex(__ldg(a.g.off + v + 1) - __ldg(a.g.off + v));
+                    qn.push(v);
+                } else {
+                    qk.push(v);
+                    lc.aux++;
+                    lmin = min(lmin, dv);
                 }
-                warp_append(qa, &sp->qlen, to_near, v);
-                warp_append(a.fq[fdst], a.flen + fdst, keep, v);
-                if (keep) { lc.aux++; lmin = min(lmin, dv); }
             }
+            cta_queue_flush(qs0, qa, &sp->qlen);
+            cta_queue_flush(qs1, a.fq[fdst], a.flen + fdst);
             // per-CTA reduction into the split counters
             {
                 unsigned long long va = block_sum(lc.va, (unsigned long long *)sm.push.cm.excl);
@@ -332,8 +339,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
         const bool use_q = push && fused && (long long)cv.ea <= (long long)(n >> 6);
         LocalCnt lc;
         if (push) {
-            const SsspPushOp op{dist, a.g.w, a.g.off, cl, use_q ? a.q[(t + 1) & 1] : nullptr, &nxt->qlen,
-                                a.fq[fcur], a.flen + fcur};
+            const SsspPushOp op{dist, a.g.w, a.g.off, cl, use_q, cta_queue(qs0, a.q[(t + 1) & 1], &nxt->qlen),
+                                cta_queue(qs1, a.fq[fcur], a.flen + fcur)};
             if (mat == SM_BITMAP) {
                 lc = run_lb(c.lb, BitmapSrc{nbt, (unsigned)n, 1u}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
             } else {
@@ -341,11 +348,13 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
                 lc = run_lb(c.lb, QueueSrc{qa, ql}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
             }
         } else {
-            const SsspPullOp op{dist, a.g.in_w, nbt, a.g.off, cl, a.fq[fcur], a.flen + fcur};
+            const SsspPullOp op{dist, a.g.in_w, nbt, a.g.off, cl, cta_queue(qs1, a.fq[fcur], a.flen + fcur)};
             lc = run_lb_reduce(c.lb, AllSrc{(unsigned)n}, adj_in, op, sm.pull, red, bar, epoch, rc.partial, a.scan);
         }
         dirty[(t + 1) % 3] = true;
         if (fused) {
+            cta_queue_flush(qs0, a.q[(t + 1) & 1], &nxt->qlen);
+            cta_queue_flush(qs1, a.fq[fcur], a.flen + fcur);
             flush_counts(lc, nxt);
             grid_sync(bar, epoch);
             mat = use_q ? SM_QUEUE : SM_BITMAP;
@@ -354,6 +363,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
             LocalCnt ec;
             ec.edges = lc.edges;
             grid_sync(bar, epoch);
+            const CtaQueue qf = cta_queue(qs1, a.fq[fcur], a.flen + fcur);
             for (long long w = gwarp(); w < W; w += gwarps()) {
                 const unsigned m = a.chg[w];
                 const int v = (int)(w * 32 + lane_id());
@@ -369,8 +379,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
                 const unsigned nm = __ballot_sync(0xffffffffu, near);
                 if (lane_id() == 0) { nnb[w] = nm; a.chg[w] = 0u; }
                 if (far) ec.aux++;
-                warp_append(a.fq[fcur], a.flen + fcur, far, v);
+                if (far) qf.push(v);
             }
+            cta_queue_flush(qs1, a.fq[fcur], a.flen + fcur);
             flush_counts(ec, nxt);
             grid_sync(bar, epoch);
             mat = SM_BITMAP;
