@@ -8,13 +8,16 @@
 //   - when N_t is empty, theta advances and F is split: dist < theta -> N, the rest stays in F;
 //   - terminate when N and F are empty.
 // Stepping candidates for the threshold theta (gsw_config.stepping):
-//   AUTO (dynamic stepping): per round, Increase (theta += delta0) when the active edges dropped by
-//   more than 35% (Fig. 12(e): increase when Ea is small), Decrease (theta -= delta0/2,
-//   never below the last split point) when they grew by more than 35%, otherwise Remain;
+//   AUTO (dynamic stepping): per round, compare the active edges with the previous round's: grown
+//   by more than 35% -> Increase (theta += delta0), shrunk by more than 35% -> Decrease
+//   (theta -= delta0/2, never below the last split point), otherwise Remain (law 1;
+//   alternative readings selectable with GSW_SSSP_LAW for calibration);
 //   INCREASE / DECREASE / REMAIN pin that per-round decision; STATIC = delta-stepping with a fixed
 //   step (theta moves only at splits); UNORDERED = Bellman-Ford (theta = infinity).
 // delta0 = gsw_config.delta0, or c*wbar/dbar with c = 32 (reading R6b).
 // Any schedule reaches the exact distances (they are the unique fixpoint); only speed differs.
+#include <cstdlib>
+
 #include "engine.cuh"
 #include "internal.h"
 #include "launch.h"
@@ -25,6 +28,10 @@ namespace gsw {
 
 enum { SM_NONE = 0, SM_QUEUE = 1, SM_SQUEUE = 2, SM_BITMAP = 3 };
 enum { ST_DYNAMIC = 0, ST_STATIC = 1, ST_UNORDERED = 2, ST_INC = 3, ST_DEC = 4, ST_REMAIN = 5 };
+// Law 1 (the literal reading of P:651-654, "if the number of edges increases or decreases by some
+// margin, we increase or decrease the priority threshold accordingly") measured best: C2 SSSP
+// 62.7 ms vs 87.1 ms for law 0 and 79.6 ms for static delta (tools/sssp_law_sweep.py, DESIGN R7).
+constexpr int kDefaultLaw = 1;
 
 struct SplitCnt {
     unsigned long long va, ea;
@@ -45,6 +52,7 @@ struct SsspArgs {
     uint32_t *scan;
     unsigned delta0;
     int mode;
+    int law;              // dynamic-stepping control law (R7); GSW_SSSP_LAW overrides
     RunCommon rc;
 };
 
@@ -284,8 +292,21 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
         // ---- P4 stepping decision for this round
         int step = GSW_STEP_REMAIN;
         if (a.mode == ST_DYNAMIC && t > 0 && prev_ea > 0) {
-            if ((double)cv.ea < 0.65 * (double)prev_ea) step = GSW_STEP_INCREASE;
-            else if ((double)cv.ea > 1.35 * (double)prev_ea) step = GSW_STEP_DECREASE;
+            const double e = (double)cv.ea, ep = (double)prev_ea, lo = (double)gthreads();
+            const bool drop = e < 0.65 * ep, grow = e > 1.35 * ep;
+            switch (a.law) {
+            case 1:  // literal: threshold follows the edge trend
+                step = grow ? GSW_STEP_INCREASE : (drop ? GSW_STEP_DECREASE : GSW_STEP_REMAIN);
+                break;
+            case 2:  // absolute (Fig. 12(e)): raise while the round is latency-bound, lower when wasteful
+                step = e < lo ? GSW_STEP_INCREASE : (e > 8.0 * lo ? GSW_STEP_DECREASE : GSW_STEP_REMAIN);
+                break;
+            case 3:  // relative 35% rule, raising only while latency-bound
+                step = (drop && e < lo) ? GSW_STEP_INCREASE : (grow ? GSW_STEP_DECREASE : GSW_STEP_REMAIN);
+                break;
+            default: // inverse: refill a draining band, brake an exploding one
+                step = drop ? GSW_STEP_INCREASE : (grow ? GSW_STEP_DECREASE : GSW_STEP_REMAIN);
+            }
         } else if (a.mode == ST_INC) step = GSW_STEP_INCREASE;
         else if (a.mode == ST_DEC) step = GSW_STEP_DECREASE;
         if (a.mode != ST_UNORDERED && a.mode != ST_STATIC) {
@@ -428,6 +449,8 @@ gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_sta
     case GSW_STEP_REMAIN: a.mode = ST_REMAIN; break;
     default: a.mode = ST_DYNAMIC;
     }
+    a.law = kDefaultLaw;
+    if (const char *law = getenv("GSW_SSSP_LAW")) a.law = atoi(law);
     LaunchInfo li;
     gsw_status s = prepare_common(g, ws, (const void *)sssp_kernel, a.rc, li);
     if (s != GSW_OK) return s;
