@@ -23,6 +23,7 @@ struct CcArgs {
     int *q;               // active-set queue (push in queue formats)
     uint32_t *scan;
     long long iso_count;
+    unsigned *heavy, *hblk, *heavy_cnt;   // tiered pull (lb_reduce.cuh lbr_tiered)
     RunCommon rc;
 };
 
@@ -65,18 +66,17 @@ struct CcPullOp {
     const uint32_t *off;         // out-offsets (degree of a changed vertex)
     bool fused;
     unsigned *nfb;
-    using Probe = uint2;         // (active-set word of u, label[u])
+    // The min over ALL in-neighbours equals the min over the active ones combined with label[v]
+    // (inactive labels were already propagated; min is idempotent), so pull gathers labels only:
+    // one random load per edge instead of two (the active-set probe).
+    using Probe = unsigned;      // label[u]
     using Acc = unsigned long long;
     static constexpr bool kFlushEmpty = false;
     static __device__ __forceinline__ Acc identity() { return 0x7fffffffull; }
     static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a < b ? a : b; }
     __device__ __forceinline__ bool skip(int) const { return false; }
-    __device__ __forceinline__ Probe probe(int, uint32_t, int u) const {
-        return make_uint2(fb[u >> 5], (unsigned)label[u]);
-    }
-    __device__ __forceinline__ Acc val(int, uint32_t, int u, Probe p) const {
-        return ((p.x >> (u & 31)) & 1u) ? (Acc)p.y : identity();
-    }
+    __device__ __forceinline__ Probe probe(int, uint32_t, int u) const { return (unsigned)label[u]; }
+    __device__ __forceinline__ Acc val(int, uint32_t, int, Probe p) const { return (Acc)p; }
     __device__ __forceinline__ void flush(int v, Acc m, bool exclusive, LocalCnt &c) const {
         if (m == identity()) return;
         int mi = (int)m;
@@ -131,7 +131,14 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) cc_kernel(CcArgs a) {
         rc.cnt[0].va = (unsigned long long)(n - a.iso_count);
         rc.cnt[0].ea = a.g.nnz;
         rc.cnt[0].maxd = 0; rc.cnt[0].mind = 0;
+        *a.heavy_cnt = 0u;
     }
+    grid_sync(bar, epoch);
+    Tiers tiers{a.heavy, a.hblk, 0u};
+    tiered_build_p1(adj_in, n, tiers, a.heavy_cnt);
+    grid_sync(bar, epoch);
+    tiers.nheavy = cta_read_u32(a.heavy_cnt);
+    tiered_build_p2(adj_in, tiers, red);
     grid_sync(bar, epoch);
 
     Book book;
@@ -192,8 +199,11 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) cc_kernel(CcArgs a) {
                 lc = run_lb(c.lb, QueueSrc{a.q, qlen}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
         } else {
             const CcPullOp op{a.label, fbt, a.g.off, fused, mark};
-            lc = run_lb_reduce(c.lb, BitmapSrc{a.iso, (unsigned)n, 0u}, adj_in, op, sm.pull, red, bar, epoch,
-                               rc.partial, a.scan);
+            if (c.lb == GSW_LB_TWC)
+                lc = lbr_tiered(op, adj_in, tiers, n);          // B200 TWC: warp-seg / warp / grid tiers
+            else
+                lc = run_lb_reduce(c.lb, BitmapSrc{a.iso, (unsigned)n, 0u}, adj_in, op, sm.pull, red, bar, epoch,
+                                   rc.partial, a.scan);
         }
         dirty[(t + 1) % 3] = true;
         if (fused) {
@@ -233,10 +243,14 @@ gsw_status run_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     a.q = (int *)ws.take((size_t)n * 4);
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
     a.iso_count = g->attrs.isolated;
+    const size_t nh = std::min<size_t>((size_t)n, (size_t)g->g.nnz / kHeavy + 1);
+    a.heavy = (unsigned *)ws.take(nh * 4);
+    a.hblk = (unsigned *)ws.take((nh + 1) * 4);
+    a.heavy_cnt = (unsigned *)ws.take(256);
     LaunchInfo li;
     gsw_status s = prepare_common(g, ws, (const void *)cc_kernel, a.rc, li);
     if (s != GSW_OK) return s;
-    if (!a.label || !a.chg || !a.fb[2] || !a.q || !a.scan) { set_error("workspace too small"); return GSW_ENOMEM; }
+    if (!a.label || !a.chg || !a.fb[2] || !a.q || !a.scan || !a.heavy || !a.hblk || !a.heavy_cnt) { set_error("workspace too small"); return GSW_ENOMEM; }
     void *args[] = {&a};
     s = launch_persistent(g, (const void *)cc_kernel, args, li);
     if (s != GSW_OK) return s;

@@ -14,6 +14,7 @@
 //   thread tier and WM reduce short rows with a warp-segmented scan); CM and STRICT split rows
 //   across threads and flush partials (STRICT merges runs of the same row first).
 #pragma once
+#include "engine.cuh"
 #include "lb.cuh"
 
 namespace gsw {
@@ -433,6 +434,108 @@ __device__ __forceinline__ LocalCnt run_lb_reduce(int lb, const Src &src, const 
         return lbr_strict(src, adj, op, scan, total, &sm.strict);
     }
     }
+}
+
+}  // namespace gsw
+
+// ------------------------------------------------------------------ B200 tiered reduction (TWC)
+// TWC re-tiered for B200 for reductions over a STATIC item set (every vertex, or every
+// non-isolated vertex): rows < 32 edges -> warp-segmented scan (32 rows per warp); 32..kHeavy-1 ->
+// one warp per row with 4 loads in flight per lane; >= kHeavy -> kHeavy-edge blocks shared by all
+// warps of the grid, each flushed as a partial (exclusive = false).  Ops whose partial flush
+// accumulates into a side buffer finish those rows after a grid barrier (tiered_finish).  The
+// heavy-row table is built once per run (tiered_build, two phases).
+namespace gsw {
+
+constexpr uint32_t kHeavy = 1024;
+
+struct Tiers {
+    unsigned *heavy;        // heavy row ids
+    unsigned *hblk;         // exclusive prefix of ceil(d/kHeavy) over heavy rows, hblk[nheavy] = total
+    unsigned nheavy;
+};
+
+// phase 1 (all CTAs): list heavy rows (in-degree >= kHeavy) with warp-aggregated appends
+__device__ __forceinline__ void tiered_build_p1(const Adj g, int n, Tiers t, unsigned *count) {
+    q_from_pred((int *)t.heavy, count, n, [&](int v) { return __ldg(g.off + v + 1) - __ldg(g.off + v) >= kHeavy; });
+}
+// phase 2 (after a grid barrier; CTA 0 scans, the others return): block prefix
+__device__ __forceinline__ void tiered_build_p2(const Adj g, Tiers t, uint32_t *red) {
+    if (blockIdx.x != 0) return;
+    uint32_t base = 0;
+    for (unsigned t0 = 0; t0 < t.nheavy; t0 += kBlock) {
+        const unsigned i = t0 + threadIdx.x;
+        uint32_t c = 0;
+        if (i < t.nheavy) {
+            const unsigned v = t.heavy[i];
+            c = (__ldg(g.off + v + 1) - __ldg(g.off + v) + kHeavy - 1) / kHeavy;
+        }
+        uint32_t tot;
+        const uint32_t ex = block_excl_scan(c, red, &tot);
+        if (i < t.nheavy) t.hblk[i] = base + ex;
+        base += tot;
+    }
+    if (threadIdx.x == 0) t.hblk[t.nheavy] = base;
+}
+
+// one warp reduces the edges [b, e) of row x (4 loads in flight per lane)
+template <class Op>
+__device__ __forceinline__ typename Op::Acc warp_row_reduce(const Op &op, const Adj &g, int x, uint32_t b, uint32_t e,
+                                                            unsigned long long &edges) {
+    using Acc = typename Op::Acc;
+    const unsigned lane = lane_id();
+    Acc a = Op::identity();
+    for (uint32_t k0 = b; k0 < e; k0 += 128) {
+        int y[4];
+        typename Op::Probe p[4];
+#pragma unroll
+        for (int h = 0; h < 4; ++h) { const uint32_t k = k0 + 32 * h + lane; y[h] = k < e ? __ldg(g.col + k) : -1; }
+#pragma unroll
+        for (int h = 0; h < 4; ++h) if (y[h] >= 0) p[h] = op.probe(x, k0 + 32 * h + lane, y[h]);
+#pragma unroll
+        for (int h = 0; h < 4; ++h)
+            if (y[h] >= 0) { a = Op::combine(a, op.val(x, k0 + 32 * h + lane, y[h], p[h])); edges++; }
+    }
+    return warp_combine<Op>(a);
+}
+
+// items: vertices v in [0, n) with !skip(v) (isolated rows reduce to the identity)
+template <class Op>
+__device__ __noinline__ LocalCnt lbr_tiered(const Op op, const Adj g, const Tiers tiers, int n) {
+    LocalCnt cnt;
+    const unsigned lane = lane_id();
+    const long long NW = gwarps();
+    // grid tier
+    const unsigned nblk = tiers.nheavy ? tiers.hblk[tiers.nheavy] : 0u;
+    for (long long blk = gwarp(); blk < nblk; blk += NW) {
+        unsigned lo = 0, hi = tiers.nheavy - 1;
+        while (lo < hi) { const unsigned mid = (lo + hi + 1) >> 1; if (tiers.hblk[mid] <= blk) lo = mid; else hi = mid - 1; }
+        const int v = (int)tiers.heavy[lo];
+        if (op.skip(v)) continue;
+        const uint32_t rb = __ldg(g.off + v), re = __ldg(g.off + v + 1);
+        const uint32_t b = rb + (uint32_t)(blk - tiers.hblk[lo]) * kHeavy, e = min(re, b + kHeavy);
+        const typename Op::Acc s = warp_row_reduce(op, g, v, b, e, cnt.edges);
+        if (lane == 0) op.flush(v, s, false, cnt);
+    }
+    // light and medium rows: a warp takes 32 consecutive vertices
+    for (long long wb = gwarp() * 32; wb < n; wb += NW * 32) {
+        int x = wb + lane < n ? (int)(wb + lane) : -1;
+        if (x >= 0 && op.skip(x)) x = -1;
+        uint32_t b = 0, d = 0;
+        if (x >= 0) { b = __ldg(g.off + x); d = __ldg(g.off + x + 1) - b; }
+        const typename Op::Acc r = warp_seg_rows(op, g, x, b, d < 32u ? d : 0u, cnt);
+        if (x >= 0 && d < 32u && (d > 0u || Op::kFlushEmpty)) op.flush(x, r, true, cnt);
+        unsigned med = __ballot_sync(0xffffffffu, x >= 0 && d >= 32u && d < kHeavy);
+        while (med) {
+            const int j = __ffs(med) - 1;
+            med &= med - 1;
+            const int xj = __shfl_sync(0xffffffffu, x, j);
+            const uint32_t bj = __shfl_sync(0xffffffffu, b, j), dj = __shfl_sync(0xffffffffu, d, j);
+            const typename Op::Acc s = warp_row_reduce(op, g, xj, bj, bj + dj, cnt.edges);
+            if ((int)lane == j) op.flush(x, s, true, cnt);
+        }
+    }
+    return cnt;
 }
 
 }  // namespace gsw

@@ -81,18 +81,9 @@ struct PrPushOp {
 };
 
 // ---------------------------------------------------------------- B200 tiered pull (TWC)
-// TWC re-tiered for B200: rows < 32 edges are reduced 32 at a time by a
-// warp-segmented scan; rows of 32..kHeavy-1 edges by one warp with 4 loads in flight per lane;
-// rows >= kHeavy edges (R-MAT hubs, up to 163K edges at C3) are cut into kHeavy-edge blocks that
-// every warp of the grid shares (one fp64 atomic per block) and finished after a grid barrier.
-constexpr uint32_t kHeavy = 1024;
-
-struct PrTiers {
-    unsigned *heavy;        // heavy row ids
-    unsigned *hblk;         // exclusive prefix of ceil(d/kHeavy) over heavy rows (+ total)
-    unsigned nheavy;
-};
-
+// lb_reduce.cuh lbr_tiered: rows < 32 warp-segmented, 32..1023 one warp per row, >= 1024 cut into
+// 1024-edge blocks shared by the whole grid; their partial sums land in `sum` (fp64 atomics) and are
+// finished after a grid barrier (phase B below).
 __device__ __forceinline__ double warp_row_sum(const double *contrib, const int32_t *col, uint32_t b, uint32_t e,
                                                unsigned long long &edges) {
     const unsigned lane = lane_id();
@@ -111,7 +102,7 @@ __device__ __forceinline__ double warp_row_sum(const double *contrib, const int3
 }
 
 // phase A: heavy blocks (atomics into sum) + light/medium rows finished in place
-__device__ __noinline__ LocalCnt pr_pull_tiered_a(const PrPullOp op, const Adj g, const PrTiers tiers, int n) {
+__device__ __noinline__ LocalCnt pr_pull_tiered_a(const PrPullOp op, const Adj g, const Tiers tiers, int n) {
     LocalCnt cnt;
     const unsigned lane = lane_id();
     const long long NW = gwarps();
@@ -147,7 +138,7 @@ __device__ __noinline__ LocalCnt pr_pull_tiered_a(const PrPullOp op, const Adj g
 }
 
 // phase B (after a grid barrier): finish the heavy rows from their accumulated block sums
-__device__ __forceinline__ void pr_pull_tiered_b(const PrPullOp &op, const PrTiers &tiers, LocalCnt &cnt) {
+__device__ __forceinline__ void pr_pull_tiered_b(const PrPullOp &op, const Tiers &tiers, LocalCnt &cnt) {
     for (long long i = gtid(); i < tiers.nheavy; i += gthreads()) {
         const unsigned v = tiers.heavy[i];
         const double s = op.sum[v];
@@ -207,28 +198,11 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
     grid_sync(bar, epoch);
     flush_dangling(dang, a.dsum);
     // heavy-row table of the tiered pull (rows >= kHeavy in-edges): list, then block prefix
-    q_from_pred((int *)a.heavy, a.heavy_cnt, n,
-                [&](int v) { return __ldg(a.g.in_off + v + 1) - __ldg(a.g.in_off + v) >= kHeavy; });
+    Tiers tiers{a.heavy, a.hblk, 0u};
+    tiered_build_p1(adj_in, n, tiers, a.heavy_cnt);
     grid_sync(bar, epoch);
-    PrTiers tiers{a.heavy, a.hblk, 0u};
     tiers.nheavy = cta_read_u32(a.heavy_cnt);
-    if (blockIdx.x == 0) {
-        __shared__ uint32_t sred[kWarps + 1];
-        uint32_t base = 0;
-        for (unsigned t0 = 0; t0 < tiers.nheavy; t0 += kBlock) {
-            unsigned i = t0 + threadIdx.x;
-            uint32_t c = 0;
-            if (i < tiers.nheavy) {
-                unsigned v = tiers.heavy[i];
-                c = (__ldg(a.g.in_off + v + 1) - __ldg(a.g.in_off + v) + kHeavy - 1) / kHeavy;
-            }
-            uint32_t tot;
-            uint32_t ex = block_excl_scan(c, sred, &tot);
-            if (i < tiers.nheavy) tiers.hblk[i] = base + ex;
-            base += tot;
-        }
-        if (threadIdx.x == 0) tiers.hblk[tiers.nheavy] = base;
-    }
+    tiered_build_p2(adj_in, tiers, red);
     grid_sync(bar, epoch);
 
     Book book;
