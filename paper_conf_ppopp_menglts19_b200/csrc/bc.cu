@@ -34,6 +34,7 @@ struct BcArgs {
     unsigned *lvl_off;    // level boundaries in S (per source, reused)
     uint32_t *scan;
     unsigned *err;        // sigma overflow flag
+    unsigned *heavy[2], *hblk[2], *heavy_cnt;   // tiered reductions: [0] in-edges, [1] out-edges
     RunCommon rc;
 };
 
@@ -46,8 +47,7 @@ struct BcPushOp {
     unsigned *V;
     const uint32_t *off;
     int lvl1;
-    int *S;
-    unsigned *slen;
+    CtaQueue S;
     struct Tok { int old; unsigned su_lo, su_hi; };
     using Probe = BcProbe;
     using Aux = uint2;
@@ -70,7 +70,7 @@ struct BcPushOp {
             c.add_vertex(d.y - d.x);
             atomicOr(V + (v >> 5), 1u << (v & 31));
         }
-        warp_append(S, slen, won, v);
+        if (won) S.push(v);
         return false;
     }
 };
@@ -82,14 +82,19 @@ struct BcPullOp {
     unsigned *V;
     const uint32_t *off;
     int lvl;
-    int *S;
-    unsigned *slen;
+    CtaQueue S;
     using Probe = BcProbe;
     using Acc = unsigned long long;
     static constexpr bool kFlushEmpty = false;
     static __device__ __forceinline__ Acc identity() { return 0ull; }
     static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a + b; }
-    __device__ __forceinline__ bool skip(int v) const { return test_bit_relaxed(V, v); }
+    // skip vertices settled BEFORE this level only: a vertex claimed during this phase (depth
+    // l+1) must keep accumulating sigma from the rest of its parents (hub rows are split across
+    // warps by the tiered mapping)
+    __device__ __forceinline__ bool skip(int v) const {
+        const int d = depth[v];
+        return d >= 0 && d <= lvl;
+    }
     __device__ __forceinline__ Probe probe(int, uint32_t, int u) const {
         unsigned long long su = sigma[u];
         return BcProbe{depth[u], (unsigned)su, (unsigned)(su >> 32)};
@@ -105,7 +110,7 @@ struct BcPullOp {
         if (won) {
             atomicOr(V + (v >> 5), 1u << (v & 31));
             c.add_vertex(__ldg(off + v + 1) - __ldg(off + v));
-            S[atomicAdd(slen, 1u)] = v;
+            S.push(v);
         }
     }
 };
@@ -119,12 +124,13 @@ struct BcBackOp {
     double *dacc;
     int lvl;
     bool owner;
+    bool by_level;        // items are all vertices; only those on level lvl take part
     using Probe = double;
     using Acc = double;
     static constexpr bool kFlushEmpty = true;
     static __device__ __forceinline__ Acc identity() { return 0.0; }
     static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a + b; }
-    __device__ __forceinline__ bool skip(int) const { return false; }
+    __device__ __forceinline__ bool skip(int v) const { return by_level && depth[v] != lvl; }
     __device__ __forceinline__ Probe probe(int, uint32_t, int w) const {
         const int dw = depth[w];
         const double ow = omega[w];                // issued together with depth[w]
@@ -151,6 +157,7 @@ union BcSmem {
 __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
     __shared__ BcSmem sm;
     __shared__ uint32_t red[kWarps + 1];
+    __shared__ CtaQStore qs;              // staged appends to the BFS stack S
     const RunCommon &rc = a.rc;
     const GridBarrier bar = make_bar(rc);
     unsigned epoch = 0;
@@ -158,6 +165,23 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
     const Adj adj_out{a.g.off, a.g.col}, adj_in{a.g.in_off, a.g.in_col};
 
     for (long long v = gtid(); v < n; v += gthreads()) a.bc[v] = 0.0;
+    if (is_book()) { a.heavy_cnt[0] = 0u; a.heavy_cnt[32] = 0u; }
+    cta_queue_reset(qs);
+    grid_sync(bar, epoch);
+    // heavy-row tables of the tiered reductions (forward pull: in-edges, backward: out-edges)
+    const bool sym = a.g.in_off == a.g.off;
+    Tiers tin{a.heavy[0], a.hblk[0], 0u}, tout{a.heavy[1], a.hblk[1], 0u};
+    tiered_build_p1(adj_in, n, tin, a.heavy_cnt);
+    if (!sym) tiered_build_p1(adj_out, n, tout, a.heavy_cnt + 32);
+    grid_sync(bar, epoch);
+    tin.nheavy = cta_read_u32(a.heavy_cnt);
+    tiered_build_p2(adj_in, tin, red);
+    if (sym) tout = tin;
+    else {
+        tout.nheavy = cta_read_u32(a.heavy_cnt + 32);
+        tiered_build_p2(adj_out, tout, red);
+    }
+    grid_sync(bar, epoch);
     Book book;
     Features f = rc.base;
     int t = 0;                          // global iteration counter (records)
@@ -210,15 +234,20 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
             if (is_book()) book_expand(book);
             LocalCnt lc;
             // next level is appended at S[send ...); its counter lives in the next slot's qlen
+            const CtaQueue sq = cta_queue(qs, a.S + send, &nxt->qlen);
             if (c.dir == GSW_PUSH) {
-                const BcPushOp op{a.depth, a.sigma, a.V, a.g.off, lvl + 1, a.S + send, &nxt->qlen};
+                const BcPushOp op{a.depth, a.sigma, a.V, a.g.off, lvl + 1, sq};
                 lc = run_lb(c.lb, QueueSrc{a.S + lbeg, (unsigned)cv.va}, adj_out, op, sm.push, red, bar, epoch,
                             rc.partial, a.scan);
             } else {
-                const BcPullOp op{a.depth, a.sigma, a.V, a.g.off, lvl, a.S + send, &nxt->qlen};
-                lc = run_lb_reduce(c.lb, BitmapSrc{a.V, (unsigned)n, 0u}, adj_in, op, sm.pull, red, bar, epoch,
-                                   rc.partial, a.scan);
+                const BcPullOp op{a.depth, a.sigma, a.V, a.g.off, lvl, sq};
+                if (c.lb == GSW_LB_TWC)
+                    lc = lbr_tiered(op, adj_in, tin, n);      // B200 TWC (skip = visited)
+                else
+                    lc = run_lb_reduce(c.lb, BitmapSrc{a.V, (unsigned)n, 0u}, adj_in, op, sm.pull, red, bar, epoch,
+                                       rc.partial, a.scan);
             }
+            cta_queue_flush(qs, a.S + send, &nxt->qlen);
             flush_counts(lc, nxt);
             grid_sync(bar, epoch);
             // the next level's size is its Va (read at the top of the next iteration)
@@ -251,9 +280,24 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
             }
             const int lb = rc.force.load_balance ? rc.force.load_balance : GSW_LB_TWC;
             const bool owner = lb == GSW_LB_THREAD || lb == GSW_LB_TWC || lb == GSW_LB_WM;
-            const BcBackOp op{a.depth, a.sigma, a.omega, a.bc, a.dacc, lvl, owner};
-            LocalCnt lc = run_lb_reduce(lb, QueueSrc{a.S + lo, hi - lo}, adj_out, op, sm.pull, red, bar, epoch,
-                                        rc.partial, a.scan);
+            LocalCnt lc;
+            if (lb == GSW_LB_TWC) {
+                // B200 TWC over every vertex of the level (skip others); hub rows are reduced by the
+                // grid tier into dacc and finished after a barrier
+                const BcBackOp op{a.depth, a.sigma, a.omega, a.bc, a.dacc, lvl, true, true};
+                lc = lbr_tiered(op, adj_out, tout, n);
+                grid_sync(bar, epoch);
+                for (long long i = gtid(); i < tout.nheavy; i += gthreads()) {
+                    const int v = (int)tout.heavy[i];
+                    if (a.depth[v] != lvl) continue;
+                    const double s = a.dacc[v];
+                    a.dacc[v] = 0.0;
+                    op.finish(v, s);
+                }
+            } else {
+            const BcBackOp op{a.depth, a.sigma, a.omega, a.bc, a.dacc, lvl, owner, false};
+            lc = run_lb_reduce(lb, QueueSrc{a.S + lo, hi - lo}, adj_out, op, sm.pull, red, bar, epoch,
+                               rc.partial, a.scan);
             if (!owner) {
                 grid_sync(bar, epoch);
                 for (long long i = gtid(); i < hi - lo; i += gthreads()) {
@@ -262,6 +306,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
                     a.dacc[v] = 0.0;
                     op.finish(v, s);
                 }
+            }
             }
             flush_counts(lc, rc.cnt + ((t + 1) % 3));
             grid_sync(bar, epoch);
@@ -306,12 +351,19 @@ gsw_status run_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc_
     a.lvl_off = (unsigned *)ws.take((size_t)kMaxHist * 4);
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
     a.err = (unsigned *)ws.take(256);
+    const size_t nh = std::min<size_t>((size_t)n, (size_t)g->g.nnz / kHeavy + 1);
+    for (int i = 0; i < 2; ++i) {
+        a.heavy[i] = (unsigned *)ws.take(nh * 4);
+        a.hblk[i] = (unsigned *)ws.take((nh + 1) * 4);
+    }
+    a.heavy_cnt = (unsigned *)ws.take(256);
     int *dsrc = (int *)ws.take((size_t)std::max(nsrc, 1) * 4);
     a.sources = dsrc;
     LaunchInfo li;
     gsw_status s = prepare_common(g, ws, (const void *)bc_kernel, a.rc, li);
     if (s != GSW_OK) return s;
-    if (!a.bc || !a.depth || !a.sigma || !a.omega || !a.dacc || !a.V || !a.S || !a.lvl_off || !a.scan || !a.err || !dsrc) {
+    if (!a.bc || !a.depth || !a.sigma || !a.omega || !a.dacc || !a.V || !a.S || !a.lvl_off || !a.scan || !a.err || !dsrc ||
+        !a.heavy[1] || !a.hblk[1] || !a.heavy_cnt) {
         set_error("workspace too small");
         return GSW_ENOMEM;
     }
