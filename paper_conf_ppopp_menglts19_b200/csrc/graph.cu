@@ -59,8 +59,21 @@ __global__ void k_attrs(const uint32_t *off, int n, AttrAcc *acc) {
     }
 }
 
-__global__ void k_degree_hist(const uint32_t *off, int n, unsigned long long *hist) {
-    for (long long v = gtid(); v < n; v += gthreads()) atomicAdd(&hist[off[v + 1] - off[v]], 1ull);
+// degree histogram: small degrees (the hot bins of power-law graphs) are counted in a per-CTA
+// shared-memory histogram and merged once; large degrees go straight to global atomics
+constexpr int kHistSmem = 2048;
+__global__ void k_degree_hist(const uint32_t *off, int n, unsigned long long *hist, unsigned nbins) {
+    __shared__ unsigned sh[kHistSmem];
+    for (int i = threadIdx.x; i < kHistSmem; i += blockDim.x) sh[i] = 0u;
+    __syncthreads();
+    for (long long v = gtid(); v < n; v += gthreads()) {
+        const unsigned d = off[v + 1] - off[v];
+        if (d < (unsigned)kHistSmem) atomicAdd(&sh[d], 1u);
+        else atomicAdd(&hist[d], 1ull);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < kHistSmem && i < (int)nbins; i += blockDim.x)
+        if (sh[i]) atomicAdd(&hist[i], (unsigned long long)sh[i]);
 }
 
 __global__ void k_maxw(const uint32_t *w, long long nnz, AttrAcc *acc) {
@@ -163,7 +176,7 @@ gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp) {
     size_t nb = (size_t)h.maxd + 1;
     unsigned long long *hist = (unsigned long long *)((char *)tmp + 256);
     GSW_CUDA(cudaMemsetAsync(hist, 0, nb * 8, g->stream));
-    k_degree_hist<<<grid_for(n, g->sms), kBlock, 0, g->stream>>>(G.off, n, hist);
+    k_degree_hist<<<grid_for(n, g->sms), kBlock, 0, g->stream>>>(G.off, n, hist, (unsigned)nb);
     GSW_CUDA(cudaGetLastError());
     std::vector<unsigned long long> hh(nb);
     GSW_CUDA(cudaMemcpyAsync(hh.data(), hist, nb * 8, cudaMemcpyDeviceToHost, g->stream));
