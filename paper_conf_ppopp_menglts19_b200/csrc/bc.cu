@@ -24,7 +24,8 @@ struct BcArgs {
     const unsigned *iso;
     const int *sources;   // device copy
     int nsrc;
-    double *bc;
+    double *bc;           // internal order
+    double *out;          // caller order (relabeled graphs), else nullptr
     int *depth;
     unsigned long long *sigma;
     double *omega;        // (1 + delta) / sigma
@@ -186,7 +187,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
     Features f = rc.base;
     int t = 0;                          // global iteration counter (records)
     for (int k = 0; k < a.nsrc; ++k) {
-        const int src = a.sources[k];
+        const int src = map_in(a.g.inv, a.sources[k]);
         // ---- per-source init
         for (long long v = gtid(); v < n; v += gthreads()) {
             a.depth[v] = v == src ? 0 : -1;
@@ -325,6 +326,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
             if (a.sigma[v] >> 63) atomicOr(a.err, 1u);
         grid_sync(bar, epoch);
     }
+    if (a.out) gather_out(a.out, a.bc, a.g.inv, n);
     if (is_book()) book_finish(book, rc, t);
 }
 
@@ -341,7 +343,9 @@ gsw_status run_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc_
     a.g = g->g;
     a.iso = g->iso;
     a.nsrc = nsrc;
-    a.bc = dev_out ? bc_out : (double *)ws.take((size_t)n * 8);
+    const bool relabeled = g->g.inv != nullptr;
+    a.bc = (dev_out && !relabeled) ? bc_out : (double *)ws.take((size_t)n * 8);
+    a.out = relabeled ? (dev_out ? bc_out : (double *)ws.take((size_t)n * 8)) : nullptr;
     a.depth = (int *)ws.take((size_t)n * 4);
     a.sigma = (unsigned long long *)ws.take((size_t)n * 8);
     a.omega = (double *)ws.take((size_t)n * 8);
@@ -372,7 +376,8 @@ gsw_status run_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc_
     void *args[] = {&a};
     s = launch_persistent(g, (const void *)bc_kernel, args, li);
     if (s != GSW_OK) return s;
-    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(bc_out, a.bc, (size_t)n * 8, cudaMemcpyDeviceToHost, g->stream));
+    if (!dev_out)
+        GSW_CUDA(cudaMemcpyAsync(bc_out, relabeled ? a.out : a.bc, (size_t)n * 8, cudaMemcpyDeviceToHost, g->stream));
     s = finish_run(g, a.rc, li, st);
     if (s != GSW_OK) return s;
     unsigned herr = 0;

@@ -22,8 +22,9 @@ enum { MAT_NONE = 0, MAT_QUEUE = 1, MAT_SQUEUE = 2, MAT_BITMAP = 3 };
 struct BfsArgs {
     DevGraph g;
     const unsigned *iso;
-    int src;
-    int *depth;
+    int src;              // caller id
+    int *depth;           // internal order
+    int *out;             // caller order (relabeled graphs), else nullptr
     unsigned *V;          // visited map (isolated + padding bits pre-set)
     unsigned *fb[3];      // frontier bitmaps, ring of 3
     int *q[2];            // active-set queues, double buffered
@@ -294,7 +295,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
     const RunCommon &rc = a.rc;
     const GridBarrier bar = make_bar(rc);
     unsigned epoch = 0;
-    const int n = a.g.n, W = (n + 31) >> 5, src = a.src;
+    const int n = a.g.n, W = (n + 31) >> 5, src = map_in(a.g.inv, a.src);
     int *depth = a.depth;
     const Adj adj_out{a.g.off, a.g.col}, adj_in{a.g.in_off, a.g.in_col};
 
@@ -436,6 +437,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
         prev_va = (long long)va;
         prev_via = Via;
     }
+    if (a.out) gather_out(a.out, depth, a.g.inv, n);
     if (is_book()) book_finish(book, rc, t);
 }
 
@@ -449,7 +451,9 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     a.g = g->g;
     a.iso = g->iso;
     a.src = source;
-    a.depth = dev_out ? depth_out : (int *)ws.take((size_t)n * 4);
+    const bool relabeled = g->g.inv != nullptr;
+    a.depth = (dev_out && !relabeled) ? depth_out : (int *)ws.take((size_t)n * 4);
+    a.out = relabeled ? (dev_out ? depth_out : (int *)ws.take((size_t)n * 4)) : nullptr;
     a.V = (unsigned *)ws.take((size_t)W * 4);
     for (int i = 0; i < 3; ++i) a.fb[i] = (unsigned *)ws.take((size_t)W * 4);
     for (int i = 0; i < 2; ++i) a.q[i] = (int *)ws.take((size_t)n * 4);
@@ -463,7 +467,8 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     void *args[] = {&a};
     s = launch_persistent(g, (const void *)bfs_kernel, args, li);
     if (s != GSW_OK) return s;
-    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(depth_out, a.depth, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
+    if (!dev_out)
+        GSW_CUDA(cudaMemcpyAsync(depth_out, relabeled ? a.out : a.depth, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
     return finish_run(g, a.rc, li, st);
 }
 

@@ -1,6 +1,7 @@
 // capi.cu -- the extern "C" boundary declared in include/gsw.h: argument validation, error
 // plumbing, handle lifetime.  Every compute step runs in the kernels of the other .cu files.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -23,6 +24,7 @@ gsw_status load_csr(gsw_graph g, const gsw_csr *c, Workspace &ws, uint32_t **off
                     int64_t *staging);
 gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp);
 gsw_status validate_graph(gsw_graph g);
+gsw_status relabel_graph(gsw_graph g, uint32_t *perm, uint32_t *inv, char *tmp, size_t tmp_bytes);
 // dist.cu
 int64_t dist_slice(int64_t n, int32_t p);
 gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int32_t nranks, int32_t rank,
@@ -63,7 +65,7 @@ const char *gsw_version(void) { return "gsw-b200 0.1 (sm_100a)"; }
 gsw_status gsw_workspace_size(int64_t n, int64_t nnz, int32_t has_weights, int32_t has_csc, size_t *bytes) {
     if (!bytes || n <= 0 || nnz < 0) { set_error("gsw_workspace_size: bad arguments"); return GSW_EINVAL; }
     if (nnz >= (int64_t(1) << 32) || n >= (int64_t(1) << 31) - 64) { set_error("graph too large"); return GSW_EOVERFLOW; }
-    *bytes = graph_bytes(n, nnz, has_weights, has_csc) + scratch_bytes_for(n, nnz) + 4096;
+    *bytes = graph_bytes(n, nnz, has_weights, has_csc) + scratch_bytes_for(n, nnz, has_weights) + 4096;
     return GSW_OK;
 }
 
@@ -107,7 +109,7 @@ gsw_status gsw_graph_create(const gsw_csr *csr, const gsw_csr *csc, void *worksp
     if (e != cudaSuccess) { delete g; return cuda_fail(e, "gsw_graph_create setup"); }
     Workspace ws{g->ws, ws_bytes, 0};
     size_t gb = graph_bytes(csr->n, csr->nnz, csr->weights != nullptr, csc != nullptr);
-    Workspace gws{g->ws, gb + 1024, 0};
+    Workspace gws{g->ws, gb + 1024, 0};   // graph region (CSR/CSC, isolated bitmap, perm/inv)
     g->scratch = g->ws + ((gb + 1024 + 255) & ~size_t(255));
     g->scratch_bytes = ws_bytes - ((gb + 1024 + 255) & ~size_t(255));
     int64_t *staging = (int64_t *)g->scratch;
@@ -130,7 +132,13 @@ gsw_status gsw_graph_create(const gsw_csr *csr, const gsw_csr *csc, void *worksp
         g->symmetric = true;
     }
     g->iso = (unsigned *)gws.take((size_t)((csr->n + 31) / 32) * 4);
-    if (!g->iso) { gsw_graph_destroy(g); set_error("workspace too small"); return GSW_ENOMEM; }
+    uint32_t *perm = (uint32_t *)gws.take((size_t)csr->n * 4), *inv = (uint32_t *)gws.take((size_t)csr->n * 4);
+    if (!g->iso || !perm || !inv) { gsw_graph_destroy(g); set_error("workspace too small"); return GSW_ENOMEM; }
+    // degree-ordered relabeling (graph.cu); GSW_NO_RELABEL=1 keeps caller order (A/B measurements)
+    const char *nr = getenv("GSW_NO_RELABEL");
+    if (!(nr && nr[0] == '1') && csr->nnz < (int64_t(1) << 31)) {
+        if ((s = relabel_graph(g, perm, inv, g->scratch, g->scratch_bytes)) != GSW_OK) { gsw_graph_destroy(g); return s; }
+    }
     void *tmp = (char *)g->scratch + (((csr->n + 1) * 16 + 4096 + 255) & ~int64_t(255));
     if ((s = compute_attrs(g, g->iso, tmp)) != GSW_OK) { gsw_graph_destroy(g); return s; }
     *out = g;

@@ -17,7 +17,8 @@ namespace gsw {
 struct CcArgs {
     DevGraph g;
     const unsigned *iso;
-    int *label;
+    int *label;           // internal order, values are caller ids
+    int *out;             // caller order (relabeled graphs), else nullptr
     unsigned *chg;        // per-vertex "label changed" status flags (standalone filter)
     unsigned *fb[3];      // active-set bitmaps, ring of 3
     int *q;               // active-set queue (push in queue formats)
@@ -119,7 +120,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) cc_kernel(CcArgs a) {
     const Adj adj_out{a.g.off, a.g.col}, adj_in{a.g.in_off, a.g.in_col};
 
     // ---- init: label = id, AS_0 = every non-isolated vertex
-    for (long long v = gtid(); v < n; v += gthreads()) a.label[v] = (int)v;
+    // labels are CALLER ids so that the fixpoint is the minimum caller id of each component
+    for (long long v = gtid(); v < n; v += gthreads()) a.label[v] = a.g.perm ? (int)a.g.perm[v] : (int)v;
     for (long long w = gtid(); w < W; w += gthreads()) {
         unsigned valid = (w == W - 1 && (n & 31)) ? ((1u << (n & 31)) - 1u) : ~0u;
         a.fb[0][w] = ~a.iso[w] & valid;
@@ -226,6 +228,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) cc_kernel(CcArgs a) {
         prev_dir = c.dir;
         prev_va = cv.va;
     }
+    if (a.out) gather_out(a.out, a.label, a.g.inv, n);
     if (is_book()) book_finish(book, rc, t);
 }
 
@@ -237,7 +240,9 @@ gsw_status run_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     CcArgs a{};
     a.g = g->g;
     a.iso = g->iso;
-    a.label = dev_out ? label_out : (int *)ws.take((size_t)n * 4);
+    const bool relabeled = g->g.inv != nullptr;
+    a.label = (dev_out && !relabeled) ? label_out : (int *)ws.take((size_t)n * 4);
+    a.out = relabeled ? (dev_out ? label_out : (int *)ws.take((size_t)n * 4)) : nullptr;
     a.chg = (unsigned *)ws.take((size_t)W * 4);
     for (int i = 0; i < 3; ++i) a.fb[i] = (unsigned *)ws.take((size_t)W * 4);
     a.q = (int *)ws.take((size_t)n * 4);
@@ -254,7 +259,8 @@ gsw_status run_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     void *args[] = {&a};
     s = launch_persistent(g, (const void *)cc_kernel, args, li);
     if (s != GSW_OK) return s;
-    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(label_out, a.label, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
+    if (!dev_out)
+        GSW_CUDA(cudaMemcpyAsync(label_out, relabeled ? a.out : a.label, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
     return finish_run(g, a.rc, li, st);
 }
 

@@ -87,6 +87,14 @@ __device__ __forceinline__ void write_record(const RunCommon &rc, int t, const D
     }
 }
 
+// ------------------------------------------------------------------ caller-order output
+// internal ids are degree-ordered (graph.cu relabel): out[j] = in[inv[j]] for caller ids j
+template <class T>
+__device__ __forceinline__ void gather_out(T *out, const T *in, const uint32_t *inv, int n) {
+    for (long long j = gtid(); j < n; j += gthreads()) out[j] = in[inv[j]];
+}
+__device__ __forceinline__ int map_in(const uint32_t *inv, int v) { return inv ? (int)inv[v] : v; }
+
 // ------------------------------------------------------------------ active-set builders
 // bitmap from a per-vertex predicate: one warp per 32-vertex word, ballot, one store
 template <class Pred>

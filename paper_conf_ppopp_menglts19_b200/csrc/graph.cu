@@ -4,6 +4,10 @@
 #include <cstring>
 #include <vector>
 
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
+#include <cub/device/device_segmented_sort.cuh>
+
 #include "common.cuh"
 #include "internal.h"
 
@@ -92,6 +96,30 @@ __global__ void k_validate(const uint32_t *off, const int32_t *col, int n, long 
         if (col[e] < 0 || col[e] >= n) atomicOr(bad, 2u);
 }
 
+// ---- degree-ordered relabeling
+__global__ void k_deg_iota(const uint32_t *off, int n, uint32_t *deg, uint32_t *ids) {
+    for (long long v = gtid(); v < n; v += gthreads()) { deg[v] = off[v + 1] - off[v]; ids[v] = (uint32_t)v; }
+}
+__global__ void k_invert(const uint32_t *perm, int n, uint32_t *inv) {
+    for (long long i = gtid(); i < n; i += gthreads()) inv[perm[i]] = (uint32_t)i;
+}
+// new row i = old row perm[i], columns renamed through inv; one warp per row
+__global__ void k_permute_rows(const uint32_t *noff, const uint32_t *off, const int32_t *col, const uint32_t *w,
+                               const uint32_t *perm, const uint32_t *inv, int n, int32_t *ncol, uint32_t *nw) {
+    for (long long i = gwarp(); i < n; i += gwarps()) {
+        const uint32_t o = perm[i];
+        const uint32_t b = off[o], e = off[o + 1], nb = noff[i];
+        for (uint32_t k = b + lane_id(); k < e; k += 32) {
+            ncol[nb + (k - b)] = (int32_t)inv[col[k]];
+            if (w) nw[nb + (k - b)] = w[k];
+        }
+    }
+}
+__global__ void k_set_u32(uint32_t *p, uint32_t v) { *p = v; }
+__global__ void k_perm_deg(const uint32_t *off, const uint32_t *perm, int n, uint32_t *degp) {
+    for (long long i = gtid(); i < n; i += gthreads()) { const uint32_t o = perm[i]; degp[i] = off[o + 1] - off[o]; }
+}
+
 inline int grid_for(long long work, int sms) {
     long long b = (work + kBlock - 1) / kBlock;
     long long cap = (long long)sms * 8;
@@ -107,17 +135,19 @@ size_t graph_bytes(int64_t n, int64_t nnz, int has_w, int has_csc) {
     add((n + 1) * 4); add(nnz * 4); if (has_w) add(nnz * 4);
     if (has_csc) { add((n + 1) * 4); add(nnz * 4); if (has_w) add(nnz * 4); }
     add(W * 4);  // isolated bitmap
+    add(n * 4); add(n * 4);  // relabeling: perm, inv
     return b;
 }
 
 // Per-run scratch: the maximum over algorithms.
-size_t scratch_bytes_for(int64_t n, int64_t nnz) {
-    (void)nnz;
+size_t relabel_temp_bytes(int64_t n, int64_t nnz, int has_w);
+size_t scratch_bytes_for(int64_t n, int64_t nnz, int has_w) {
     size_t W = (size_t)((n + 31) / 32);
     size_t per_v = 64;                         // BC: depth 4 + sigma 8 + delta 8 + stack 4 + bc 8 + queues
     size_t b = per_v * (size_t)(n + 64) + 16 * W * 4;
     b += (size_t)(n + 1) * 8;                  // i64 offset staging at ingest / scan arrays
     b += 8u << 20;                             // control blocks, per-CTA partials, history, records
+    if (nnz < (int64_t(1) << 31)) b = std::max(b, relabel_temp_bytes(n, nnz, has_w));   // ingest temp
     return b;
 }
 
@@ -204,6 +234,79 @@ gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp) {
     A.maxw = h.maxw;
     A.wbar = G.nnz ? (double)h.wsum / (double)G.nnz : 0.0;
     A.isolated = (int64_t)h.iso;
+    return GSW_OK;
+}
+
+// ---------------------------------------------------------------- degree-ordered relabeling
+// Internal vertex ids are assigned by descending degree (stable: ties keep caller order) and every
+// row is sorted ascending in the new ids.  Hubs then share a few cache lines in every per-vertex
+// array (frontier bits, labels, PR contributions) and come first in each adjacency row, which
+// helps the early-exit pull.  Outputs are gathered back to caller ids by each kernel.
+static size_t al256(size_t x) { return (x + 255) & ~size_t(255); }
+
+size_t relabel_temp_bytes(int64_t n, int64_t nnz, int has_w) {
+    size_t t1 = 0, t2 = 0, t3 = 0;
+    cub::DeviceRadixSort::SortPairsDescending(nullptr, t1, (uint32_t *)nullptr, (uint32_t *)nullptr,
+                                              (uint32_t *)nullptr, (uint32_t *)nullptr, (int)n);
+    cub::DeviceScan::InclusiveSum(nullptr, t2, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)n);
+    if (has_w)
+        cub::DeviceSegmentedSort::SortPairs(nullptr, t3, (int32_t *)nullptr, (int32_t *)nullptr, (uint32_t *)nullptr,
+                                            (uint32_t *)nullptr, (int)nnz, (int)n, (uint32_t *)nullptr,
+                                            (uint32_t *)nullptr);
+    else
+        cub::DeviceSegmentedSort::SortKeys(nullptr, t3, (int32_t *)nullptr, (int32_t *)nullptr, (int)nnz, (int)n,
+                                           (uint32_t *)nullptr, (uint32_t *)nullptr);
+    size_t t = std::max(t1, std::max(t2, t3));
+    return al256(t) + 3 * al256((size_t)n * 4) + al256((size_t)(n + 1) * 4) + al256((size_t)std::max<int64_t>(nnz, 1) * 4) * (has_w ? 2 : 1) + 4096;
+}
+
+static gsw_status relabel_csr(gsw_graph g, uint32_t *off, int32_t *col, uint32_t *w, const uint32_t *perm,
+                              const uint32_t *inv, uint32_t *degp, uint32_t *noff, int32_t *colT, uint32_t *wT,
+                              void *cub_tmp, size_t cub_bytes) {
+    const int n = g->g.n;
+    const int64_t nnz = g->g.nnz;
+    cudaStream_t s = g->stream;
+    k_perm_deg<<<grid_for(n, g->sms), kBlock, 0, s>>>(off, perm, n, degp);
+    size_t cb = cub_bytes;
+    GSW_CUDA(cub::DeviceScan::InclusiveSum(cub_tmp, cb, degp, noff + 1, n, s));
+    k_set_u32<<<1, 1, 0, s>>>(noff, 0u);
+    k_permute_rows<<<grid_for((long long)n * 32, g->sms), kBlock, 0, s>>>(noff, off, col, w, perm, inv, n, colT, wT);
+    GSW_CUDA(cudaGetLastError());
+    GSW_CUDA(cudaMemcpyAsync(off, noff, (size_t)(n + 1) * 4, cudaMemcpyDeviceToDevice, s));
+    cb = cub_bytes;
+    if (w) GSW_CUDA(cub::DeviceSegmentedSort::SortPairs(cub_tmp, cb, colT, col, wT, w, (int)nnz, n, noff, noff + 1, s));
+    else GSW_CUDA(cub::DeviceSegmentedSort::SortKeys(cub_tmp, cb, colT, col, (int)nnz, n, noff, noff + 1, s));
+    return GSW_OK;
+}
+
+gsw_status relabel_graph(gsw_graph g, uint32_t *perm, uint32_t *inv, char *tmp, size_t tmp_bytes) {
+    const int n = g->g.n;
+    const int64_t nnz = g->g.nnz;
+    const int has_w = g->g.w != nullptr;
+    if (tmp_bytes < relabel_temp_bytes(n, nnz, has_w)) { set_error("relabel: scratch too small"); return GSW_ENOMEM; }
+    Workspace t{tmp, tmp_bytes, 0};
+    uint32_t *deg = (uint32_t *)t.take((size_t)n * 4), *ids = (uint32_t *)t.take((size_t)n * 4);
+    uint32_t *degs = (uint32_t *)t.take((size_t)n * 4), *noff = (uint32_t *)t.take((size_t)(n + 1) * 4);
+    int32_t *colT = (int32_t *)t.take((size_t)std::max<int64_t>(nnz, 1) * 4);
+    uint32_t *wT = has_w ? (uint32_t *)t.take((size_t)std::max<int64_t>(nnz, 1) * 4) : nullptr;
+    size_t cub_bytes = tmp_bytes - t.used - 512;
+    void *cub_tmp = t.take(cub_bytes);
+    cudaStream_t s = g->stream;
+    k_deg_iota<<<grid_for(n, g->sms), kBlock, 0, s>>>(g->g.off, n, deg, ids);
+    size_t cb = cub_bytes;
+    GSW_CUDA(cub::DeviceRadixSort::SortPairsDescending(cub_tmp, cb, deg, degs, ids, perm, n, 0, 32, s));
+    k_invert<<<grid_for(n, g->sms), kBlock, 0, s>>>(perm, n, inv);
+    GSW_CUDA(cudaGetLastError());
+    gsw_status st = relabel_csr(g, (uint32_t *)g->g.off, (int32_t *)g->g.col, (uint32_t *)g->g.w, perm, inv, degs,
+                                noff, colT, wT, cub_tmp, cub_bytes);
+    if (st != GSW_OK) return st;
+    if (!g->symmetric) {
+        st = relabel_csr(g, (uint32_t *)g->g.in_off, (int32_t *)g->g.in_col, (uint32_t *)g->g.in_w, perm, inv, degs,
+                         noff, colT, wT, cub_tmp, cub_bytes);
+        if (st != GSW_OK) return st;
+    }
+    g->g.perm = perm;
+    g->g.inv = inv;
     return GSW_OK;
 }
 

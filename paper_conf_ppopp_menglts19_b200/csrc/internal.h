@@ -20,6 +20,10 @@ struct DevGraph {
     const uint32_t *in_off;   // n+1  (in-edges, pull)
     const int32_t *in_col;
     const uint32_t *in_w;
+    // degree-ordered relabeling (graph.cu): internal id i is caller id perm[i]; inv[caller] = i.
+    // nullptr when the graph is kept in caller order.
+    const uint32_t *perm;
+    const uint32_t *inv;
 };
 
 // Dataset attributes (Table 1), computed once at load.
@@ -81,7 +85,7 @@ gsw_status cuda_fail(cudaError_t e, const char *what);
     } while (0)
 
 // scratch bytes for a graph of n vertices (max over algorithms), see DESIGN.md "HBM layout"
-size_t scratch_bytes_for(int64_t n, int64_t nnz);
+size_t scratch_bytes_for(int64_t n, int64_t nnz, int has_w);
 
 // 1 if p is device (or managed) memory, 0 if host, -1 on error
 int is_device_ptr(const void *p);

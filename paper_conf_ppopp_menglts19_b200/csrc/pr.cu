@@ -31,6 +31,7 @@ struct PrArgs {
 // epilogue shared by owner flushes and the accumulator pass
 struct PrEpi {
     const uint32_t *off;
+    const uint32_t *perm;   // relabeled graphs: out is in caller order
     double *out;
     double *cnext;
     double base, d;
@@ -38,7 +39,7 @@ struct PrEpi {
     __device__ __forceinline__ void finish(int v, double s, double &dang) const {
         double p = base + d * s;
         uint32_t dg = __ldg(off + v + 1) - __ldg(off + v);
-        if (last) out[v] = p;
+        if (last) out[perm ? perm[v] : v] = p;
         cnext[v] = dg ? p / (double)dg : 0.0;
         if (!dg) dang += p;
     }
@@ -191,7 +192,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
         a.contrib[0][v] = dg ? (1.0 / N) / (double)dg : 0.0;
         a.sum[v] = 0.0;
         if (!dg) dang += 1.0 / N;
-        if (a.iters == 0) a.out[v] = 1.0 / N;
+        if (a.iters == 0) a.out[v] = 1.0 / N;         // uniform: order-free
     }
     for (long long i = gtid(); i <= a.iters; i += gthreads()) a.dsum[i] = 0.0;
     if (is_book()) *a.heavy_cnt = 0u;
@@ -227,7 +228,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
         if (threadIdx.x == 0) sD = *(volatile const double *)(a.dsum + t);
         __syncthreads();
         const double D = sD;
-        const PrEpi epi{a.g.off, a.out, a.contrib[(t + 1) & 1], (1.0 - d) / N + d * D / N, d, t == a.iters - 1};
+        const PrEpi epi{a.g.off, a.g.perm, a.out, a.contrib[(t + 1) & 1], (1.0 - d) / N + d * D / N, d, t == a.iters - 1};
         const double *cur = a.contrib[t & 1];
         if (is_book()) book_expand(book);
         LocalCnt lc;

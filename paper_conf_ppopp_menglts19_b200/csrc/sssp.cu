@@ -40,8 +40,9 @@ struct SplitCnt {
 
 struct SsspArgs {
     DevGraph g;
-    int src;
-    unsigned *dist;
+    int src;              // caller id
+    unsigned *dist;       // internal order
+    unsigned *out;        // caller order (relabeled graphs), else nullptr
     unsigned *nb[3];      // near-set bitmaps (ring of 3); also the claim map of the next near set
     int *q[2];            // near queues
     unsigned *chg;        // "improved this round" status flags (standalone filter)
@@ -170,7 +171,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
     const RunCommon &rc = a.rc;
     const GridBarrier bar = make_bar(rc);
     unsigned epoch = 0;
-    const int n = a.g.n, W = (n + 31) >> 5, src = a.src;
+    const int n = a.g.n, W = (n + 31) >> 5, src = map_in(a.g.inv, a.src);
     const Adj adj_out{a.g.off, a.g.col}, adj_in{a.g.in_off, a.g.in_col};
     unsigned *dist = a.dist;
 
@@ -410,6 +411,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
         prev_dir = c.dir;
         prev_va = cv.va;
     }
+    if (a.out) gather_out(a.out, dist, a.g.inv, n);
     if (is_book()) book_finish(book, rc, t);
 }
 
@@ -427,7 +429,9 @@ gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_sta
     SsspArgs a{};
     a.g = g->g;
     a.src = source;
-    a.dist = dev_out ? dist_out : (unsigned *)ws.take((size_t)n * 4);
+    const bool relabeled = g->g.inv != nullptr;
+    a.dist = (dev_out && !relabeled) ? dist_out : (unsigned *)ws.take((size_t)n * 4);
+    a.out = relabeled ? (dev_out ? dist_out : (unsigned *)ws.take((size_t)n * 4)) : nullptr;
     for (int i = 0; i < 3; ++i) a.nb[i] = (unsigned *)ws.take((size_t)W * 4);
     for (int i = 0; i < 2; ++i) a.q[i] = (int *)ws.take((size_t)n * 4);
     for (int i = 0; i < 2; ++i) a.fq[i] = (int *)ws.take((size_t)n * 4);
@@ -461,7 +465,8 @@ gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_sta
     void *args[] = {&a};
     s = launch_persistent(g, (const void *)sssp_kernel, args, li);
     if (s != GSW_OK) return s;
-    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(dist_out, a.dist, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
+    if (!dev_out)
+        GSW_CUDA(cudaMemcpyAsync(dist_out, relabeled ? a.out : a.dist, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
     return finish_run(g, a.rc, li, st);
 }
 
