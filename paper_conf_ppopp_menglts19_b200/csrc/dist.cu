@@ -555,7 +555,7 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
         if (Va == 0) break;
         if (t > 0) { Via -= Va; Eia -= Ea; }
         // same direction split as the single-GPU selector (select.cuh, R6)
-        int dir = ((double)Ea * 16.0 > (double)Eia && (double)Va * 1024.0 > (double)d->n) ? GSW_PULL : GSW_PUSH;
+        int dir = ((double)Ea * 16.0 > (double)Eia && (double)Va * 2048.0 > (double)d->n) ? GSW_PULL : GSW_PUSH;
         if (g->forced.direction != GSW_AUTO) dir = g->forced.direction;
         unsigned *fb = d->FB[t & 1], *nfb = d->FB[(t + 1) & 1];
         GSW_CUDA(cudaMemsetAsync(nfb, 0, FBW * 4, s));

@@ -431,6 +431,72 @@ __device__ __noinline__ LocalCnt lb_strict(const Src src, const Adj g, Op op, co
 
 namespace gsw {
 
+// STRICT for small active sets (<= kStrictTile items, e.g. a few hubs): every CTA scans the item
+// degrees itself in shared memory (no grid-wide scan, no grid barriers) and the diagonals per
+// thread shrink so that the edges spread over every thread of the grid (one edge per thread when
+// the frontier is tiny but the edges are many).
+template <class Src, class Op>
+__device__ __noinline__ LocalCnt lb_strict_small(const Src src, const Adj g, Op op, StrictSmem *sm) {
+    LocalCnt cnt;
+    __shared__ uint32_t red[kWarps + 1];
+    const unsigned sz = src.size();
+    uint32_t base = 0;
+    for (unsigned t0 = 0; t0 < sz; t0 += kBlock) {
+        const unsigned i = t0 + threadIdx.x;
+        int x = i < sz ? src.get(i) : -1;
+        if (x >= 0 && op.skip(x)) x = -1;
+        const uint32_t b = x >= 0 ? __ldg(g.off + x) : 0u;
+        const uint32_t d = x >= 0 ? __ldg(g.off + x + 1) - b : 0u;
+        uint32_t tot;
+        const uint32_t ex = block_excl_scan(d, red, &tot);
+        if (i < sz) { sm->scan[i] = base + ex; sm->x[i] = x; sm->beg[i] = b; }
+        base += tot;
+    }
+    const uint32_t total = base;
+    if (threadIdx.x == 0) sm->scan[sz] = total;
+    __syncthreads();
+    const unsigned long long D = (unsigned long long)sz + total;
+    const unsigned long long per = ((unsigned long long)gridDim.x * kBlock);
+    const unsigned vt = (unsigned)max(1ull, min((unsigned long long)kStrictVT, (D + per - 1) / per));
+    const unsigned long long tile = (unsigned long long)kBlock * vt;
+    const unsigned long long ntiles = (D + tile - 1) / tile;
+    for (unsigned long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const unsigned long long dd0 = min(D, t * tile + (unsigned long long)threadIdx.x * vt);
+        const unsigned long long dd1 = min(D, dd0 + vt);
+        // items consumed at dd0: merge path over the whole (shared-memory) scan
+        long long lo = dd0 > total ? (long long)(dd0 - total) : 0;
+        long long hi = (long long)min((unsigned long long)sz, dd0);
+        while (lo < hi) {
+            const long long mid = (lo + hi) >> 1;
+            if ((unsigned long long)sm->scan[mid + 1] <= dd0 - 1 - (unsigned long long)mid) lo = mid + 1; else hi = mid;
+        }
+        long long ii = lo;
+        unsigned long long k = dd0 - (unsigned long long)ii;
+        int xs[kStrictVT];
+        uint32_t es[kStrictVT];
+        bool ok[kStrictVT], stop[kStrictVT];
+#pragma unroll
+        for (int s = 0; s < kStrictVT; ++s) {
+            ok[s] = false; xs[s] = -1; es[s] = 0;
+            const unsigned long long dd = dd0 + s;
+            if (dd < dd1) {
+                if (ii < (long long)sz && (unsigned long long)sm->scan[ii + 1] <= k) {
+                    ++ii;
+                } else {
+                    const int x = sm->x[ii];
+                    xs[s] = x;
+                    es[s] = sm->beg[ii] + (uint32_t)(k - sm->scan[ii]);
+                    ok[s] = x >= 0 && !(Op::kEarlyExit && op.skip(x));
+                    ++k;
+                }
+            }
+        }
+        edge_batch<kStrictVT>(op, g, xs, es, ok, stop, cnt);
+    }
+    __syncthreads();
+    return cnt;
+}
+
 union LbSmem {
     TwcSmem twc;
     CmSmem cm;
@@ -449,6 +515,7 @@ __device__ __forceinline__ LocalCnt run_lb(int lb, const Src &src, const Adj &ad
     case GSW_LB_WM: return lb_wm(src, adj, op);
     case GSW_LB_CM: return lb_cm(src, adj, op, &sm.cm);
     default: {
+        if (src.size() <= (unsigned)kStrictTile) return lb_strict_small(src, adj, op, &sm.strict);
         strict_scan_p1(src, adj, partial, red);
         grid_sync(bar, epoch);
         uint32_t total = strict_scan_p2(src, adj, partial, scan, red);

@@ -38,7 +38,7 @@ __device__ __forceinline__ int pick(int forced, int chosen) { return forced != G
 // ~1/3600, and pulling a tiny frontier costs a full scan of the visited map, so the calibrated
 // split is  pull <=> Ea * kPullAlpha > Eia  and  Va * kPullBeta > N   (reading R6).
 constexpr float kPullAlpha = 16.f;
-constexpr float kPullBeta = 1024.f;
+constexpr float kPullBeta = 2048.f;
 constexpr long long kTwcMinActive = 148LL * 4 * kBlock * 4;   // items that fill every TWC tile once
 
 __device__ __forceinline__ int traversal_direction(const Features &f) {

@@ -68,7 +68,7 @@ def test_features_match_oracle_per_level(gsw):
         # direction split on Ea/Eia with the B200-calibrated constants (select.cuh,
         # DESIGN.md reading R6), reproduced exactly
         for r in rec:
-            pull = r["Ea"] * 16.0 > r["Eia"] and r["Va"] * 1024.0 > g.n
+            pull = r["Ea"] * 16.0 > r["Eia"] and r["Va"] * 2048.0 > g.n
             assert r["direction"] == (gsw.PULL if pull else gsw.PUSH)
 
 
