@@ -150,7 +150,8 @@ __device__ __forceinline__ void pr_pull_tiered_b(const PrPullOp &op, const Tiers
 
 __device__ __forceinline__ DevCfg select_pr(const Features &f, const gsw_config &force) {
     DevCfg c = select_traversal(f, force);
-    // every vertex and edge is active: pull (atomic-free) with hub-aware TWC unless forced
+    // every vertex and edge is active: pull (atomic-free); the AUTO choice (pull + STRICT) is
+    // dispatched to pr_stream.cu by run_pr, so this kernel only runs forced combinations
     if (force.load_balance == GSW_AUTO) c.lb = GSW_LB_TWC;
     c.fmt = GSW_BITMAP;
     c.fused = GSW_FUSED;
@@ -270,11 +271,22 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
     }
 }
 
+gsw_status run_pr_stream(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st);
+
 gsw_status run_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st) {
     const int n = g->g.n;
     if (!rank) { set_error("gsw_pr: rank is NULL"); return GSW_EINVAL; }
     if (iters < 0 || iters > kMaxHist - 2) { set_error("gsw_pr: iters out of range"); return GSW_EINVAL; }
     if (!(damping >= 0.0 && damping <= 1.0)) { set_error("gsw_pr: damping must be in [0,1]"); return GSW_EINVAL; }
+    // Every iteration of PR has the same features (Va = N, Ea = nnz), so select_pr's decision is the
+    // same for all of them and is taken here once: pull + STRICT runs the edge-tiled stream kernel
+    // (pr_stream.cu); every other forced combination runs pr_kernel below.
+    {
+        const gsw_config &fc = g->forced;
+        const int dir = fc.direction != GSW_AUTO ? fc.direction : GSW_PULL;
+        const int lb = fc.load_balance != GSW_AUTO ? fc.load_balance : GSW_LB_STRICT;
+        if (dir == GSW_PULL && lb == GSW_LB_STRICT) return run_pr_stream(g, damping, iters, rank, st);
+    }
     Workspace ws{g->scratch, g->scratch_bytes, 0};
     const bool dev_out = is_device_ptr(rank) == 1;
     PrArgs a{};
