@@ -91,9 +91,11 @@ __device__ __forceinline__ double block_sum_1024(double v, double *sh) {
 
 __device__ __forceinline__ void load_cols(const int32_t *in_col, uint32_t e0, uint32_t nnz, int (&c)[kEpt]) {
     if (e0 + kEpt <= nnz) {
-        const int4 x = ld_stream4(reinterpret_cast<const int4 *>(in_col + e0));
-        const int4 y = ld_stream4(reinterpret_cast<const int4 *>(in_col + e0 + 4));
-        c[0] = x.x; c[1] = x.y; c[2] = x.z; c[3] = x.w; c[4] = y.x; c[5] = y.y; c[6] = y.z; c[7] = y.w;
+#pragma unroll
+        for (int h = 0; h < kEpt / 4; ++h) {
+            const int4 x = ld_stream4(reinterpret_cast<const int4 *>(in_col + e0 + 4 * h));
+            c[4 * h] = x.x; c[4 * h + 1] = x.y; c[4 * h + 2] = x.z; c[4 * h + 3] = x.w;
+        }
     } else {
 #pragma unroll
         for (int j = 0; j < kEpt; ++j) c[j] = e0 + j < nnz ? __ldg(in_col + e0 + j) : 0;
@@ -234,6 +236,23 @@ __global__ void __launch_bounds__(kSBlock, 1) pr_stream_kernel(PrsArgs a) {
                 load_cols(in_col, qn * kWt + lane * kEpt, nnz, cols);
                 nlo = a.wt_row[qn]; nhi = a.wt_row[qn + 1];
             }
+            const uint32_t ts = q * (uint32_t)kWt, te = min(ts + (uint32_t)kWt, nnz);
+            if (lo == hi) {
+                // the whole tile lies in row lo (hub rows): a warp sum, no row walk
+                const uint32_t e0 = ts + lane * kEpt;
+                double acc = 0.0;
+#pragma unroll
+                for (int j = 0; j < kEpt; ++j) acc += e0 + j < te ? (double)val[j] : 0.0;
+                acc = warp_sum(acc);
+                const uint32_t rb = __shfl_sync(0xffffffffu, pre_off, 0), re = __shfl_sync(0xffffffffu, pre_off, 1);
+                if (lane == 0) {
+                    if (rb < ts || re > te) atomicAdd(a.sum + lo, acc);      // finished in phase B
+                    else finish((int)lo, acc, a.sym ? re - rb : deg_out((int)lo));
+                }
+                lo = nlo; hi = nhi;
+                if (qn < a.nwt) pre_off = lo + lane <= hi + 1 ? __ldg(in_off + lo + lane) : 0u;
+                continue;
+            }
             // row offsets of this tile (rows lo .. hi+1) into the warp's buffer
             const unsigned cnt = hi - lo + 2;
             const uint32_t *so;
@@ -246,7 +265,6 @@ __global__ void __launch_bounds__(kSBlock, 1) pr_stream_kernel(PrsArgs a) {
                 so = in_off + lo;
             }
             __syncwarp();
-            const uint32_t ts = q * (uint32_t)kWt, te = min(ts + (uint32_t)kWt, nnz);
             const uint32_t e0 = ts + lane * kEpt;
             const int m = e0 < te ? (int)min((uint32_t)kEpt, te - e0) : 0;
             int ckey = -2 - (int)lane;           // carry key (global row) or a unique breaker
