@@ -181,9 +181,12 @@ __device__ __noinline__ LocalCnt bfs_pull_words(const unsigned *__restrict__ fb,
     return cnt;
 }
 
-// Pull over a per-warp compacted list of unvisited vertices (the THREAD candidate on the bitmap
-// format, B200 version): a warp compacts the zero bits of 16 visited-map words (512 vertices)
-// into shared memory, then every lane runs kPullCur independent cursors over its list entries;
+// Pull over the unvisited vertices of 16 visited-map words per warp (the THREAD candidate on the
+// bitmap format, B200 version).  Pass 1: every unvisited vertex probes its first in-neighbour
+// through the coalesced in_first array (after relabeling, the highest-degree neighbour -- the
+// likeliest frontier member), which settles most vertices of the big middle level without the
+// random col access.  Pass 2: the misses are compacted into shared memory and every lane runs
+// kPullCur independent cursors over them, from their second edge;
 // a cursor that finishes (frontier parent found, or row exhausted) immediately refills from the
 // list, so a lane's time is the SUM of its scan lengths spread over kPullCur chains rather than
 // the maximum over a warp.  Each vertex has exactly one owner lane, so its visited / next-frontier
@@ -193,7 +196,7 @@ constexpr int kPullWordsPerWarp = 16;
 constexpr int kPullList = kPullWordsPerWarp * 32;
 __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, unsigned *__restrict__ V,
                                                int *__restrict__ depth, const uint32_t *__restrict__ in_off,
-                                               const int32_t *__restrict__ in_col,
+                                               const int32_t *__restrict__ in_col, const int32_t *__restrict__ in_first,
                                                const uint32_t *__restrict__ out_off, bool symmetric, int lvl,
                                                unsigned *__restrict__ nfb, int n, int *lists) {
     LocalCnt cnt;
@@ -209,17 +212,49 @@ __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, 
             word = ~orig;                                   // padding bits are set in V
             found_bits[lane] = 0u;
         }
-        const unsigned c = __popc(word);
-        const unsigned inc = warp_incl_scan(c);
-        const unsigned total = __shfl_sync(0xffffffffu, inc, 31);
-        unsigned pos = inc - c;
-        while (word) {
-            const int b = __ffs(word) - 1;
-            word &= word - 1;
-            list[pos++] = (int)((w0 + lane) * 32 + b);
+        // pass 1: probe the first in-neighbour (the highest-degree one) of every unvisited vertex,
+        // coalesced through in_first, 4 words in flight; a miss with more edges joins the list
+        unsigned total = 0;                                  // warp-uniform list length
+        unsigned nz = __ballot_sync(0xffffffffu, word != 0u);  // words with unvisited vertices
+#pragma unroll 1
+        while (nz) {
+            int y[4], vv[4], kk[4];
+            uint32_t b[4], en[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                kk[j] = nz ? __ffs(nz) - 1 : -1;              // warp-uniform
+                nz &= nz - 1u;
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const unsigned wm = __shfl_sync(0xffffffffu, word, kk[j] < 0 ? 0 : kk[j]);
+                vv[j] = (int)((w0 + kk[j]) * 32 + lane);
+                const bool act = kk[j] >= 0 && ((wm >> lane) & 1u);   // padding bits are set in V: vv < n
+                y[j] = act ? __ldg(in_first + vv[j]) : -2;
+                b[j] = act ? __ldg(in_off + vv[j]) : 0u;
+                en[j] = act ? __ldg(in_off + vv[j] + 1) : 0u;
+            }
+            unsigned p[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) p[j] = y[j] >= 0 ? fb[y[j] >> 5] : 0u;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const bool hit = y[j] >= 0 && ((p[j] >> (y[j] & 31)) & 1u);
+                if (y[j] >= 0) cnt.edges++;
+                if (hit) {
+                    depth[vv[j]] = lvl + 1;
+                    cnt.add_vertex(symmetric ? en[j] - b[j] : __ldg(out_off + vv[j] + 1) - __ldg(out_off + vv[j]));
+                }
+                const unsigned hm = __ballot_sync(0xffffffffu, hit);
+                if (lane == 0 && kk[j] >= 0) found_bits[kk[j]] = hm;
+                const bool miss = y[j] >= 0 && !hit && en[j] - b[j] > 1u;
+                const unsigned mm = __ballot_sync(0xffffffffu, miss);
+                if (miss) list[total + __popc(mm & lanemask_lt())] = vv[j];
+                total += __popc(mm);
+            }
         }
         __syncwarp();
-        // cursors: v < 0 = empty; st = 0 needs offsets, 1 scanning
+        // pass 2: cursors over the misses, from their second edge
         int v[kPullCur];
         uint32_t e[kPullCur], end[kPullCur], beg[kPullCur];
         unsigned next = lane;
@@ -230,7 +265,8 @@ __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, 
         }
 #pragma unroll
         for (int j = 0; j < kPullCur; ++j) {
-            beg[j] = e[j] = v[j] >= 0 ? __ldg(in_off + v[j]) : 0u;
+            beg[j] = v[j] >= 0 ? __ldg(in_off + v[j]) : 0u;
+            e[j] = beg[j] + 1;
             end[j] = v[j] >= 0 ? __ldg(in_off + v[j] + 1) : 0u;
         }
         for (;;) {
@@ -271,7 +307,8 @@ __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, 
             for (int j = 0; j < kPullCur; ++j) {
                 if (nv[j] != v[j]) {
                     v[j] = nv[j];
-                    beg[j] = e[j] = v[j] >= 0 ? __ldg(in_off + v[j]) : 0u;
+                    beg[j] = v[j] >= 0 ? __ldg(in_off + v[j]) : 0u;
+                    e[j] = beg[j] + 1;
                     end[j] = v[j] >= 0 ? __ldg(in_off + v[j] + 1) : 0u;
                 }
             }
@@ -419,7 +456,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
             const BfsPullOp op{depth, a.V, a.g.off, c.fmt == GSW_BITMAP ? fbt : nullptr, t, fused, a.fb[(t + 1) % 3]};
             if (c.fmt == GSW_BITMAP && c.lb == GSW_LB_THREAD) {
                 static_assert(sizeof(LbSmem) >= sizeof(int) * (kPullList + kPullWordsPerWarp) * kWarps, "pull lists live in the LB smem");
-                lc = bfs_pull_list(fbt, a.V, depth, a.g.in_off, a.g.in_col, a.g.off, a.g.in_off == a.g.off, t,
+                lc = bfs_pull_list(fbt, a.V, depth, a.g.in_off, a.g.in_col, a.g.in_first, a.g.off, a.g.in_off == a.g.off, t,
                                    fused ? a.fb[(t + 1) % 3] : nullptr, n, reinterpret_cast<int *>(&sm));
             } else if (c.fmt == GSW_BITMAP) {
                 lc = run_lb(c.lb, BitmapSrc{a.V, (unsigned)n, 0u}, adj_in, op, sm, red, bar, epoch, rc.partial, a.scan);

@@ -25,6 +25,7 @@ gsw_status load_csr(gsw_graph g, const gsw_csr *c, Workspace &ws, uint32_t **off
 gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp);
 gsw_status validate_graph(gsw_graph g);
 gsw_status relabel_graph(gsw_graph g, uint32_t *perm, uint32_t *inv, char *tmp, size_t tmp_bytes);
+gsw_status build_first_nbr(gsw_graph g, int32_t *first);
 // dist.cu
 int64_t dist_slice(int64_t n, int32_t p);
 gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int32_t nranks, int32_t rank,
@@ -139,6 +140,9 @@ gsw_status gsw_graph_create(const gsw_csr *csr, const gsw_csr *csc, void *worksp
     if (!(nr && nr[0] == '1') && csr->nnz < (int64_t(1) << 31)) {
         if ((s = relabel_graph(g, perm, inv, g->scratch, g->scratch_bytes)) != GSW_OK) { gsw_graph_destroy(g); return s; }
     }
+    int32_t *first = (int32_t *)gws.take((size_t)csr->n * 4 + 4);
+    if (!first) { gsw_graph_destroy(g); set_error("workspace too small"); return GSW_ENOMEM; }
+    if ((s = build_first_nbr(g, first)) != GSW_OK) { gsw_graph_destroy(g); return s; }
     void *tmp = (char *)g->scratch + (((csr->n + 1) * 16 + 4096 + 255) & ~int64_t(255));
     if ((s = compute_attrs(g, g->iso, tmp)) != GSW_OK) { gsw_graph_destroy(g); return s; }
     *out = g;

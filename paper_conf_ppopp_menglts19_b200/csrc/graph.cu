@@ -96,6 +96,12 @@ __global__ void k_validate(const uint32_t *off, const int32_t *col, int n, long 
         if (col[e] < 0 || col[e] >= n) atomicOr(bad, 2u);
 }
 
+__global__ void k_first_nbr(const uint32_t *off, const int32_t *col, int n, int32_t *first) {
+    for (long long v = gtid(); v < n; v += gthreads()) {
+        const uint32_t b = off[v];
+        first[v] = off[v + 1] > b ? col[b] : -1;
+    }
+}
 // ---- degree-ordered relabeling
 __global__ void k_deg_iota(const uint32_t *off, int n, uint32_t *deg, uint32_t *ids) {
     for (long long v = gtid(); v < n; v += gthreads()) { deg[v] = off[v + 1] - off[v]; ids[v] = (uint32_t)v; }
@@ -136,6 +142,7 @@ size_t graph_bytes(int64_t n, int64_t nnz, int has_w, int has_csc) {
     if (has_csc) { add((n + 1) * 4); add(nnz * 4); if (has_w) add(nnz * 4); }
     add(W * 4);  // isolated bitmap
     add(n * 4); add(n * 4);  // relabeling: perm, inv
+    add(n * 4);              // first in-neighbour
     return b;
 }
 
@@ -324,6 +331,13 @@ gsw_status validate_graph(gsw_graph g) {
     GSW_CUDA(cudaStreamSynchronize(g->stream));
     if (hb & 1u) { set_error("row offsets are not monotone"); return GSW_EINVAL; }
     if (hb & 2u) { set_error("column index out of range"); return GSW_EINVAL; }
+    return GSW_OK;
+}
+
+gsw_status build_first_nbr(gsw_graph g, int32_t *first) {
+    k_first_nbr<<<grid_for(g->g.n, g->sms), kBlock, 0, g->stream>>>(g->g.in_off, g->g.in_col, g->g.n, first);
+    GSW_CUDA(cudaGetLastError());
+    g->g.in_first = first;
     return GSW_OK;
 }
 

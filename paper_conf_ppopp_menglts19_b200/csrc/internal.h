@@ -20,6 +20,9 @@ struct DevGraph {
     const uint32_t *in_off;   // n+1  (in-edges, pull)
     const int32_t *in_col;
     const uint32_t *in_w;
+    // in_first[v] = in_col[in_off[v]] (-1 for empty rows): the first in-neighbour, i.e. the
+    // highest-degree one after relabeling, read coalesced by the pull's first probe (graph.cu)
+    const int32_t *in_first;
     // degree-ordered relabeling (graph.cu): internal id i is caller id perm[i]; inv[caller] = i.
     // nullptr when the graph is kept in caller order.
     const uint32_t *perm;

@@ -15,7 +15,8 @@ D = {v: k for k, v in gsw.DIRECTIONS.items()}
 L = {v: k for k, v in gsw.LOAD_BALANCES.items()}
 F = {v: k for k, v in gsw.FORMATS.items()}
 U = {v: k for k, v in gsw.FUSIONS.items()}
-for force in [dict(), dict(direction="push"), dict(direction="pull")]:
+forces = [dict()] if (len(sys.argv) > 3 and sys.argv[3] == 'auto') else [dict(), dict(direction="push"), dict(direction="pull")]
+for force in forces:
     G.force_config(**force)
     for s in roots:
         best = None
