@@ -6,7 +6,7 @@ BFS on the C3 graph (Graph500 R-MAT scale 22, edge factor 16, symmetrised), root
 SURVEY Q12 source stream.  One step = one autotuned gsw_bfs call (features -> selector -> Filter
 -> Expand per level, all inside one persistent kernel) from the next root.
 
-  python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--workload bfs|...]
+  python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--workload C3|C5]
 
 Prints ONE JSON line on rank 0.  GTEPS = sum over steps of m_cc / device time, with m_cc = the
 undirected edges with both endpoints reached.  L2 is flushed (256 MiB write) between
@@ -153,7 +153,7 @@ def cpu_baseline_sample(g, roots, budget_s=12.0):
         if secs > budget_s:
             break
     return {"value": edges / secs / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
-            "sample": f"{n} BFS roots on the full C3 graph, single-threaded oracle.bfs, {secs:.1f} s"}
+            "sample": f"{n} BFS roots on the full {g.name} graph, single-threaded oracle.bfs, {secs:.1f} s"}
 
 
 def run_extras(gsw, dev, G3, g3, peak):
@@ -284,7 +284,7 @@ def run_gsw(args, ws, rank, local):
         return run_gsw_dist(args, ws, rank, local)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    g, gen_s = build_graph("C3")
+    g, gen_s = build_graph(args.workload)
     deg = g.deg
     nroots = max(64, args.steps + args.warmup)
     roots = gen.sources(g, nroots)
@@ -339,7 +339,7 @@ def run_gsw(args, ws, rank, local):
     if os.path.exists(tf):
         with open(tf) as f:
             traffic = json.load(f).get("dram_bytes_per_launch")
-    extra = run_extras(gsw, dev, G, g, peak) if (rank == 0 and not args.quick) else None
+    extra = run_extras(gsw, dev, G, g, peak) if (rank == 0 and not args.quick and args.workload == "C3") else None
 
     # ---- e2e: through the public API from pinned host buffers (graph H2D + BFS + depth D2H)
     e2e = None
@@ -349,7 +349,7 @@ def run_gsw(args, ws, rank, local):
         host_out = torch.empty(g.n, dtype=torch.int32).pin_memory()
         del G
         torch.cuda.synchronize()
-        ke = min(args.steps, 8)
+        ke = min(args.steps, 8 if args.workload == "C3" else 2)
         e2e_ms, e2e_edges = 0.0, 0
         for k in range(ke + 1):
             s = roots[k % nroots]
@@ -371,7 +371,8 @@ def run_gsw(args, ws, rank, local):
             "metric": "BFS GTEPS", "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": "C3: BFS on R-MAT scale 22 ef 16 (Graph500 a,b,c=.57,.19,.19), "
+            "config": {"workload": f"{args.workload}: BFS on R-MAT scale {22 if args.workload == 'C3' else 26} ef 16 "
+                                   "(Graph500 a,b,c=.57,.19,.19), "
                                    f"n={g.n}, nnz={g.nnz}, roots per SURVEY Q12, autotuned",
                        "l2": "flushed between steps (256 MiB write outside the timed span)",
                        "parallelism": "replicas" if ws > 1 else "single GPU"},
@@ -390,7 +391,7 @@ def run_gsw(args, ws, rank, local):
             "extra": extra,
         }
         if not args.no_cpu_baseline:
-            line["cpu_baseline"] = cpu_baseline_sample(g, roots[:8])
+            line["cpu_baseline"] = cpu_baseline_sample(g, roots[:8 if args.workload == "C3" else 1])
         print(json.dumps(line), flush=True)
     if ws > 1:
         dist.barrier()
@@ -405,6 +406,8 @@ def main():
     ap.add_argument("--impl", default="gsw", choices=["gsw", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--quick", action="store_true", help="headline only (skip the other configs)")
+    ap.add_argument("--workload", default="C3", choices=["C3", "C5"],
+                    help="C3 (default, the north_star's headline) or C5 (R-MAT scale 26, 1 GPU)")
     ap.add_argument("--force-dist", action="store_true", help="run the partitioned NCCL path even at N=1")
     args = ap.parse_args()
     if args.warmup < 3:

@@ -91,6 +91,8 @@ typedef struct {
     int64_t edges;                /* adjacency entries read by this iteration's Expand          */
     uint32_t theta;               /* SSSP priority threshold in force (0 for other algorithms) */
     float filter_us, expand_us;   /* device time of the Filter and Expand phases (%globaltimer)*/
+    int32_t ctas;                 /* CTAs that executed the iteration: the persistent grid, or 1
+                                     in the CTA-resident tier for tiny active sets */
 } gsw_iter_record;
 
 typedef struct {

@@ -46,7 +46,7 @@ class gsw_iter_record(ctypes.Structure):
                 ("load_balance", ctypes.c_int32), ("stepping", ctypes.c_int32), ("fusion", ctypes.c_int32),
                 ("Va", ctypes.c_int64), ("Ea", ctypes.c_int64), ("Via", ctypes.c_int64),
                 ("Eia", ctypes.c_int64), ("edges", ctypes.c_int64), ("theta", ctypes.c_uint32),
-                ("filter_us", ctypes.c_float), ("expand_us", ctypes.c_float)]
+                ("filter_us", ctypes.c_float), ("expand_us", ctypes.c_float), ("ctas", ctypes.c_int32)]
 
 
 class gsw_run_stats(ctypes.Structure):

@@ -325,8 +325,238 @@ __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, 
     return cnt;
 }
 
-__global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
-    __shared__ LbSmem sm;
+// ---------------------------------------------------------------- CTA-resident tier (solo)
+// On road-like graphs and in the first/last levels of scale-free ones the active set is a few
+// hundred vertices: one grid-wide iteration then costs ~8-13 us of barrier and dependent L2/HBM
+// round trips (queue -> offsets -> columns -> probe -> claim -> degree -> counters -> barrier),
+// almost none of it work.  While the selector keeps choosing fused push and the level stays
+// below (solo_v vertices, solo_e edges), CTA 0 runs the levels alone with the frontier, its
+// offsets, degrees and degree scan in shared memory; the other CTAs park at one grid barrier.
+// Per level the dependent global chain is two round trips: the column loads, then the claim
+// (atomicOr on the visited map) issued together with a speculative load of the target's offsets,
+// so a winner enters the next frontier with its row already known.  The edges of a level are
+// split evenly over the 256 threads by a merge-path search on the degree scan.  The selector
+// still runs every level on the same features and the records mark these iterations ctas = 1.
+constexpr int kSQ = 768;       // solo frontier capacity (vertices of one level); sized so that
+                               // SoloSmem fits inside LbSmem (the kernel's smem, hence its L1 share, is unchanged)
+constexpr int kSoloK = 4;      // edges in flight per thread
+struct SoloSmem {
+    int q[2][kSQ];
+    uint32_t beg[2][kSQ];
+    uint32_t scan[2][kSQ + 1];     // degrees, then their exclusive scan
+    unsigned qn[2];
+    unsigned long long ea;
+    unsigned maxd, mind;
+    int go;
+    uint32_t red[kWarps + 1];
+    unsigned long long book_raw[(sizeof(Book) + 7) / 8];   // CTA 0 / thread 0's Book during the episode
+    long long prev_va;
+};
+union BfsSmem {
+    LbSmem lb;
+    SoloSmem solo;
+};
+static_assert(sizeof(SoloSmem) <= sizeof(LbSmem), "the solo tier must not grow the kernel's shared memory");
+
+// Runs levels t, t+1, ... on the calling CTA (CTA 0) until the selector or the size limits end
+// the episode; returns with AS_t (t = first level NOT run) in a.q[t & 1], its counters in
+// rc.cnt[t % 3] and the loop state in rc.pub.  Called by all threads of CTA 0.
+// Everything is passed by value (the kernel's bookkeeping travels through ss.book / ss.prev_va):
+// taking the address of the kernel's locals would pin them to local memory for the whole run.
+__device__ __noinline__ void bfs_solo(const BfsArgs &a, SoloSmem &ss, int t, long long Via, long long Eia,
+                                      const Features fbase, unsigned qn0) {
+    float4 hist = make_float4(0.f, 0.f, 0.f, 0.f);   // history features of the next level (thread 0)
+    Book &book = *reinterpret_cast<Book *>(ss.book_raw);   // thread 0 only
+    long long &prev_va = ss.prev_va;                  // thread 0 only
+    const RunCommon &rc = a.rc;
+    const unsigned tid = threadIdx.x;
+    const uint32_t *__restrict__ off = a.g.off;
+    const int32_t *__restrict__ col = a.g.col;
+    unsigned *V = a.V;
+    int *depth = a.depth;
+    const long long sv = rc.solo_v < (long long)kSQ ? rc.solo_v : (long long)kSQ, se = rc.solo_e;
+    // AS_t0 from the grid's queue (qn0 <= kSQ), with its offsets
+    for (unsigned i0 = tid; i0 < qn0; i0 += kBlock * 4) {
+        int u[4];
+        uint32_t b[4], e[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) u[k] = i0 + k * kBlock < qn0 ? a.q[t & 1][i0 + k * kBlock] : -1;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            b[k] = u[k] >= 0 ? __ldg(off + u[k]) : 0u;
+            e[k] = u[k] >= 0 ? __ldg(off + u[k] + 1) : 0u;
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            if (u[k] < 0) continue;
+            const unsigned i = i0 + k * kBlock;
+            ss.q[0][i] = u[k]; ss.beg[0][i] = b[k]; ss.scan[0][i] = e[k] - b[k];
+        }
+    }
+    int cur = 0;
+    unsigned qn = qn0;
+    bool first = true;
+    unsigned long long E_prev = 0, Ea = 0;
+    unsigned mxd = 0, mnd = 0;
+    for (;;) {
+        // (A) features of AS_t: degrees are in shared memory (spilled entries: global queue)
+        if (tid == 0) { ss.ea = 0ull; ss.maxd = 0u; ss.mind = 0xffffffffu; }
+        __syncthreads();
+        {
+            const int *gq = a.q[t & 1];
+            unsigned long long lea = 0;
+            unsigned lmx = 0, lmn = 0xffffffffu;
+            for (unsigned i = tid; i < qn; i += kBlock) {
+                unsigned d;
+                if (i < (unsigned)kSQ) d = ss.scan[cur][i];
+                else { const int u = gq[i]; d = __ldg(off + u + 1) - __ldg(off + u); }
+                lea += d;
+                lmx = d > lmx ? d : lmx;
+                lmn = d < lmn ? d : lmn;
+            }
+            lea = warp_sum(lea);
+            lmx = warp_max(lmx);
+            lmn = warp_min(lmn);
+            if (lane_id() == 0 && lea) {
+                atomicAdd(&ss.ea, lea);
+                atomicMax(&ss.maxd, lmx);
+                atomicMin(&ss.mind, lmn);
+            }
+        }
+        __syncthreads();
+        Ea = ss.ea; mxd = ss.maxd; mnd = ss.mind;
+        // (B) the selector on AS_t's features: continue solo only for fused push on a small set
+        if (tid == 0) {
+            int go = first ? 1 : 0;
+            if (!first && qn > 0) {
+                Features f = fbase;
+                f.Va = (long long)qn; f.Ea = (long long)Ea; f.Via = Via - (long long)qn; f.Eia = Eia - (long long)Ea;
+                f.maxd = mxd; f.mind = mnd; f.iter = t;
+                f.tf = hist.x; f.te = hist.y; f.Tf = hist.z; f.Te = hist.w;
+                DevCfg c = select_traversal(f, rc.force);
+                if (c.dir == GSW_PUSH && c.fused == GSW_FUSED && (long long)qn <= sv && (long long)Ea <= se) {
+                    go = 1;
+                    c.fmt = GSW_QUEUE;
+                    book.bytes += 12ull * (unsigned long long)prev_va + 4ull * E_prev + 8ull * qn;
+                    book.edges += E_prev;
+                    if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)E_prev;
+                    // history carried to iteration t+1 (book_start's lag-2 protocol, kept in registers)
+                    hist = book_start(book, rc, t, rc.cnt + ((t + 1) % 3));
+                    write_record(rc, t, c, f, 0u);
+                    reset_cnt(rc.cnt + ((t + 2) % 3));
+                }
+            }
+            if (first) {       // the main loop's book_start(t) wrote the history of t+1
+                const IterCnt *cs = rc.cnt + ((t + 1) % 3);
+                hist = make_float4(cs->tf, cs->te, cs->Tf, cs->Te);
+            }
+            if (go && t < kMaxHist) rc.rec[t].ctas = 1;
+            ss.go = go;
+            ss.qn[cur ^ 1] = 0u;
+        }
+        __syncthreads();
+        if (!ss.go) break;
+        if (!first) { Via -= (long long)qn; Eia -= (long long)Ea; }
+        // (C) exclusive scan of the degrees (consecutive entries per thread)
+        {
+            const unsigned per = (qn + kBlock - 1) / kBlock, i0 = tid * per;
+            uint32_t loc = 0;
+            for (unsigned k = 0; k < per; ++k)
+                if (i0 + k < qn) loc += ss.scan[cur][i0 + k];
+            uint32_t tot;
+            uint32_t ex = block_excl_scan(loc, ss.red, &tot);
+            for (unsigned k = 0; k < per; ++k) {
+                if (i0 + k < qn) { const uint32_t d = ss.scan[cur][i0 + k]; ss.scan[cur][i0 + k] = ex; ex += d; }
+            }
+            if (tid == 0) ss.scan[cur][qn] = tot;
+            __syncthreads();
+        }
+        if (tid == 0) book_expand(book);
+        // (D) Expand: thread tid takes edges [lo, hi) of the level.  Round trip 1: columns;
+        // round trip 2: claim (atomicOr on V) + the target's offsets, loaded speculatively
+        {
+            const unsigned E = (unsigned)Ea;
+            const int nx = cur ^ 1;
+            int *gqn = a.q[(t + 1) & 1];
+            const uint32_t *scan = ss.scan[cur], *beg = ss.beg[cur];
+            const unsigned lo = (unsigned)(((unsigned long long)E * tid) / kBlock);
+            const unsigned hi = (unsigned)(((unsigned long long)E * (tid + 1)) / kBlock);
+            // every lane of a warp runs the warp's maximum number of batches, so the claim
+            // commits can be warp-aggregated (one shared atomic per warp and batch)
+            const unsigned mine = hi > lo ? (hi - lo + kSoloK - 1) / kSoloK : 0u;
+            const unsigned nb = __reduce_max_sync(0xffffffffu, mine);
+            unsigned i = 0, j = lo;
+            if (lo < hi) {
+                unsigned L = 0, R = qn;
+                while (R - L > 1) {
+                    const unsigned m = (L + R) >> 1;
+                    if (scan[m] <= lo) L = m; else R = m;
+                }
+                i = L;
+            }
+            for (unsigned bt = 0; bt < nb; ++bt) {
+                int v[kSoloK];
+#pragma unroll
+                for (int k = 0; k < kSoloK; ++k) {
+                    v[k] = -1;
+                    if (j < hi) {
+                        while (scan[i + 1] <= j) ++i;
+                        v[k] = __ldg(col + beg[i] + (j - scan[i]));
+                        ++j;
+                    }
+                }
+                unsigned old[kSoloK];
+                uint32_t vb[kSoloK], ve[kSoloK];
+#pragma unroll
+                for (int k = 0; k < kSoloK; ++k) {
+                    old[k] = v[k] >= 0 ? atomicOr(V + (v[k] >> 5), 1u << (v[k] & 31)) : 0xffffffffu;
+                    vb[k] = v[k] >= 0 ? __ldg(off + v[k]) : 0u;
+                    ve[k] = v[k] >= 0 ? __ldg(off + v[k] + 1) : 0u;
+                }
+#pragma unroll
+                for (int k = 0; k < kSoloK; ++k) {
+                    const bool won = v[k] >= 0 && !((old[k] >> (v[k] & 31)) & 1u);
+                    const unsigned m = __ballot_sync(0xffffffffu, won);
+                    if (!m) continue;
+                    unsigned base = 0;
+                    if (lane_id() == (unsigned)(__ffs(m) - 1)) base = atomicAdd(&ss.qn[nx], (unsigned)__popc(m));
+                    base = __shfl_sync(0xffffffffu, base, __ffs(m) - 1);
+                    if (won) {
+                        depth[v[k]] = t + 1;
+                        const unsigned p = base + __popc(m & lanemask_lt());
+                        if (p < (unsigned)kSQ) { ss.q[nx][p] = v[k]; ss.beg[nx][p] = vb[k]; ss.scan[nx][p] = ve[k] - vb[k]; }
+                        else gqn[p] = v[k];
+                    }
+                }
+            }
+            __syncthreads();
+            E_prev = E;
+            if (tid == 0) prev_va = (long long)qn;
+            qn = ss.qn[nx];
+            cur = nx;
+            ++t;
+            first = false;
+        }
+    }
+    // hand AS_t to the grid: the queue (smem part; the spill is already in place), its counters
+    // in slot t % 3 (plus the edges of level t-1, accounted by the main loop), the loop state
+    {
+        int *gq = a.q[t & 1];
+        const unsigned m = qn < (unsigned)kSQ ? qn : (unsigned)kSQ;
+        for (unsigned i = tid; i < m; i += kBlock) gq[i] = ss.q[cur][i];
+        if (tid == 0) {
+            IterCnt *c = rc.cnt + (t % 3);
+            c->va = qn; c->ea = Ea; c->maxd = mxd; c->mind = mnd; c->qlen = qn; c->edges = E_prev;
+            TeamPub p{};
+            p.t = t; p.Via = Via; p.Eia = Eia;
+            *rc.pub = p;
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(const __grid_constant__ BfsArgs a) {
+    __shared__ BfsSmem bsm;
+    LbSmem &sm = bsm.lb;
     __shared__ CtaQStore qs;
     __shared__ uint32_t red[kWarps + 1];
     const RunCommon &rc = a.rc;
@@ -354,6 +584,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
     grid_sync(bar, epoch);
 
     Book book;
+    const bool solo_allowed = rc.solo_e > 0 && rc.force.direction == GSW_AUTO && rc.force.format == GSW_AUTO &&
+                              rc.force.load_balance == GSW_AUTO && rc.force.fusion == GSW_AUTO;
+    bool last_small = false;
     long long Via = (long long)n - 1, Eia = (long long)a.g.nnz - dsrc;
     int mat = MAT_SQUEUE;
     bool dirty[3] = {false, false, false};
@@ -383,6 +616,34 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(BfsArgs a) {
         const DevCfg c = select_traversal(f, rc.force);
         write_record(rc, t, c, f, 0u);
         if (is_book()) reset_cnt(rc.cnt + ((t + 2) % 3));
+        // CTA-resident tier: CTA 0 runs the levels alone while the frontier stays tiny
+        // (entered only after two consecutive small levels: a one-level episode costs more in
+        // park/wake and hand-back than it saves, measured on C1/C3)
+        const bool small = (long long)ea <= rc.solo_e && (long long)va <= rc.solo_v && va <= (unsigned long long)kSQ;
+        const bool solo = solo_allowed && small && last_small && c.dir == GSW_PUSH && c.fused == GSW_FUSED &&
+                          (mat == MAT_QUEUE || mat == MAT_SQUEUE);
+        last_small = small;
+        if (solo) {
+            if (blockIdx.x == 0) {
+                if (threadIdx.x == 0) { *reinterpret_cast<Book *>(bsm.solo.book_raw) = book; bsm.solo.prev_va = prev_va; }
+                bfs_solo(a, bsm.solo, t, Via, Eia, f, cv.qlen);
+                if (threadIdx.x == 0) { book = *reinterpret_cast<const Book *>(bsm.solo.book_raw); prev_va = bsm.solo.prev_va; }
+                prev_dir = GSW_PUSH;
+                grid_sync(bar, epoch);
+            } else {
+                grid_park(bar, epoch);
+            }
+            TeamPub p;
+            pub_read(rc.pub, p);
+            t = (int)p.t; Via = p.Via; Eia = p.Eia;
+            mat = MAT_QUEUE;
+            if (dirty[0] || dirty[1] || dirty[2]) {          // the grid's next Filter expects clean maps
+                for (int i = 0; i < 3; ++i) if (dirty[i]) { clear_words(a.fb[i], W); dirty[i] = false; }
+                grid_sync(bar, epoch);
+            }
+            --t;
+            continue;
+        }
         const int b2 = (t + 2) % 3;
         if (dirty[b2]) { clear_words(a.fb[b2], W); dirty[b2] = false; }
 

@@ -89,6 +89,34 @@ __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch)
     __syncthreads();
 }
 
+// Grid barrier for CTAs parked while CTA 0 runs a solo episode (engine.cuh):
+// same protocol as grid_sync, but the wait sleeps between polls so the parked CTAs do not steal
+// issue slots from CTA 0's SM or keep invalidating its L1 with acquire loads.
+__device__ __forceinline__ void grid_park(const GridBarrier &b, unsigned &epoch) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned target = epoch + 1;
+        unsigned prev;
+        asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(prev) : "l"(b.arrive) : "memory");
+        if (prev == target * gridDim.x - 1) {
+            st_release(b.gen, target);
+        } else {
+            uint64_t t0 = globaltimer();
+            unsigned spins = 0;
+            while (ld_acquire(b.gen) < target) {
+                __nanosleep(200);
+                if (((++spins) & 255u) == 0 && globaltimer() - t0 > kBarrierTimeoutNs) {
+                    atomicExch(b.err, 0xBA5u);
+                    __trap();
+                }
+            }
+        }
+        __threadfence();
+    }
+    epoch += 1;
+    __syncthreads();
+}
+
 // ------------------------------------------------------------------ warp / block reductions
 template <typename T>
 __device__ __forceinline__ T warp_sum(T v) {

@@ -11,6 +11,12 @@
 namespace gsw {
 
 constexpr int kMaxHist = 1 << 16;   // iterations with stored history / records
+// CTA-resident (solo) tier thresholds: an iteration runs on CTA 0 alone when its active set has
+// at most kSoloV vertices and kSoloE edges (and the selector picked fused push on a queue).
+// Calibrated on B200 (tools/solo_sweep.py, tools/round_stats.py): a solo
+// level costs ~2.7 us at 1 vertex and ~9 us at 300 vertices, a grid level ~13 us.
+constexpr long long kSoloE = 2048;
+constexpr long long kSoloV = 512;
 
 struct Hist {
     float tf, te, Tf, Te;
@@ -33,7 +39,27 @@ struct RunCommon {
     uint32_t *partial;       // gridDim entries (+1)
     gsw_config force;
     Features base;           // dataset attributes (runtime fields filled per iteration)
+    struct TeamPub *pub;     // loop state handed from CTA 0 to the parked CTAs (solo tier)
+    long long solo_e, solo_v;  // solo-tier thresholds on Ea / Va (0 disables the tier)
 };
+
+// Loop state CTA 0 hands to the parked CTAs when a solo episode ends:
+// written by thread 0 of CTA 0 before the releasing grid barrier, read after it.
+struct alignas(16) TeamPub {
+    long long t, Via, Eia;
+    unsigned long long va, ea;
+    int mat, dirty, done, qlen;
+    int dir, fmt, lb, step, fused, pad;
+    unsigned long long aux[8];   // algorithm-specific (SSSP: theta, floor, |F|, ...)
+};
+__device__ __forceinline__ void pub_read(const TeamPub *g, TeamPub &out) {
+    __shared__ TeamPub s;
+    __syncthreads();
+    if (threadIdx.x == 0) s = *g;   // plain loads after the barrier's acquire (L1 invalidated)
+    __syncthreads();
+    out = s;
+    __syncthreads();
+}
 
 __device__ __forceinline__ GridBarrier make_bar(const RunCommon &rc) {
     return GridBarrier{&rc.ctl->arrive, &rc.ctl->gen, &rc.ctl->err};
@@ -51,17 +77,20 @@ __device__ __forceinline__ bool is_book() { return blockIdx.x == 0 && threadIdx.
 // Start of iteration t (CTA 0 / thread 0): close the timing of iteration t-1 (Filter = start ->
 // expand stamp, Expand = expand stamp -> now) and publish it as history features through the
 // counter slot `carry` that every CTA reads at iteration t+1 (lag 2, identical in all CTAs).
-__device__ __forceinline__ void book_start(Book &b, const RunCommon &rc, int t, IterCnt *carry) {
+__device__ __forceinline__ float4 book_start(Book &b, const RunCommon &rc, int t, IterCnt *carry) {
     uint64_t now = globaltimer();
+    float4 h = make_float4(0.f, 0.f, 0.f, 0.f);
     if (t >= 1) {
         float tf = (float)(b.t_expand - b.t_start) * 1e-3f;
         float te = (float)(now - b.t_expand) * 1e-3f;
         b.sum_tf += tf; b.sum_te += te;
-        carry->tf = tf; carry->te = te; carry->Tf = b.sum_tf / (float)t; carry->Te = b.sum_te / (float)t;
+        h = make_float4(tf, te, b.sum_tf / (float)t, b.sum_te / (float)t);
+        carry->tf = h.x; carry->te = h.y; carry->Tf = h.z; carry->Te = h.w;
         if (t - 1 < kMaxHist) { rc.rec[t - 1].filter_us = tf; rc.rec[t - 1].expand_us = te; }
     }
     b.t_start = now;
     b.t_expand = now;
+    return h;   // the history features iteration t+1 will read from `carry`
 }
 __device__ __forceinline__ void book_expand(Book &b) { b.t_expand = globaltimer(); }
 __device__ __forceinline__ void book_finish(const Book &b, const RunCommon &rc, int iters) {
@@ -83,15 +112,40 @@ __device__ __forceinline__ void write_record(const RunCommon &rc, int t, const D
         r.edges = 0;
         r.theta = theta;
         r.filter_us = 0.f; r.expand_us = 0.f;
+        r.ctas = (int32_t)gridDim.x;
         rc.rec[t] = r;
     }
 }
 
 // ------------------------------------------------------------------ caller-order output
 // internal ids are degree-ordered (graph.cu relabel): out[j] = in[inv[j]] for caller ids j
+// Batched: each thread issues kG index loads, then kG value loads, then kG stores, so one
+// dependent (inv -> in) round trip covers kG elements (the plain loop was latency-bound: ~28
+// serial round trips per thread at C3, ~25 us).
 template <class T>
-__device__ __forceinline__ void gather_out(T *out, const T *in, const uint32_t *inv, int n) {
-    for (long long j = gtid(); j < n; j += gthreads()) out[j] = in[inv[j]];
+__device__ __forceinline__ void gather_out(T *__restrict__ out, const T *__restrict__ in,
+                                           const uint32_t *__restrict__ inv, int n) {
+    constexpr int kG = 8;
+    const long long T0 = gtid(), NT = gthreads();
+    for (long long base = T0; base < n; base += kG * NT) {
+        uint32_t ix[kG];
+        T val[kG];
+#pragma unroll
+        for (int k = 0; k < kG; ++k) {
+            const long long j = base + k * NT;
+            ix[k] = j < n ? __ldg(inv + j) : 0u;
+        }
+#pragma unroll
+        for (int k = 0; k < kG; ++k) {
+            const long long j = base + k * NT;
+            if (j < n) val[k] = in[ix[k]];
+        }
+#pragma unroll
+        for (int k = 0; k < kG; ++k) {
+            const long long j = base + k * NT;
+            if (j < n) out[j] = val[k];
+        }
+    }
 }
 __device__ __forceinline__ int map_in(const uint32_t *inv, int v) { return inv ? (int)inv[v] : v; }
 

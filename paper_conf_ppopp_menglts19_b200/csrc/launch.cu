@@ -1,5 +1,6 @@
 // launch.cu -- persistent cooperative launch + run bookkeeping shared by all algorithms.
 #include <algorithm>
+#include <cstdlib>
 #include <map>
 #include <mutex>
 
@@ -19,8 +20,18 @@ static int blocks_per_sm(const void *kernel) {
         nb = 1;
     }
     nb = std::max(1, std::min(nb, kMinBlocks));
+    // optional shared-memory carveout hint (percent), for L1-vs-smem A/B measurements
+    if (const char *c = std::getenv("GSW_CARVEOUT")) {
+        if (cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, std::atoi(c)) != cudaSuccess)
+            cudaGetLastError();
+    }
     cache[kernel] = nb;
     return nb;
+}
+
+static long long env_ll(const char *name, long long dflt) {
+    const char *v = std::getenv(name);
+    return (v && *v) ? std::atoll(v) : dflt;
 }
 
 gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li) {
@@ -30,7 +41,8 @@ gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCom
     rc.hist = (Hist *)ws.take(sizeof(Hist) * kMaxHist);
     rc.rec = (gsw_iter_record *)ws.take(sizeof(gsw_iter_record) * kMaxHist);
     rc.partial = (uint32_t *)ws.take(sizeof(uint32_t) * (li.grid + 1));
-    if (!rc.ctl || !rc.cnt || !rc.hist || !rc.rec || !rc.partial) {
+    rc.pub = (TeamPub *)ws.take(sizeof(TeamPub));
+    if (!rc.ctl || !rc.cnt || !rc.hist || !rc.rec || !rc.partial || !rc.pub) {
         set_error("workspace too small for the run's control blocks");
         return GSW_ENOMEM;
     }
@@ -40,6 +52,9 @@ gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCom
     f.N = (float)A.N; f.M = (float)A.M; f.dbar = (float)A.dbar; f.sd = (float)A.sd; f.rd = (float)A.rd;
     f.gini = (float)A.gini; f.her = (float)A.her;
     rc.base = f;
+    // solo tier (CTA 0 alone for tiny active sets); GSW_SOLO_E / GSW_SOLO_V override (calibration)
+    rc.solo_e = env_ll("GSW_SOLO_E", kSoloE);
+    rc.solo_v = env_ll("GSW_SOLO_V", kSoloV);
     GSW_CUDA(cudaMemsetAsync(rc.ctl, 0, sizeof(Ctl), g->stream));
     return GSW_OK;
 }

@@ -123,3 +123,35 @@ def test_c3_full_size(gsw):
     for s in gen.sources(g, 2):
         d, st = _bfs(G, s, records=64)
         assert np.array_equal(d, oracle.bfs(g, s))
+
+
+@pytest.mark.parametrize("solo", [("0", "0"), ("8192", "4096"), ("64", "16"), ("1000000", "1000000")])
+def test_solo_tier_thresholds(gsw, monkeypatch, solo):
+    """CTA-resident tier: identical depths and per-level features whether the
+    tier is off, on, switching every few levels (tiny thresholds) or always on; the records say
+    which iterations ran on one CTA."""
+    monkeypatch.setenv("GSW_SOLO_E", solo[0])
+    monkeypatch.setenv("GSW_SOLO_V", solo[1])
+    for g in (gen.grid(61, 47), gen.rmat(13, seed=5), gen.from_edges(300, [(i, i + 1) for i in range(299)])):
+        G = gsw.Graph(g.off, g.col)
+        for s in gen.sources(g, 3, seed=4):
+            d, st = _bfs(G, s, records=4096)
+            assert np.array_equal(d, oracle.bfs(g, s)), (solo, g.name, s)
+            Va, Ea, Via, Eia = oracle.bfs_features(g, s)
+            assert [r["Va"] for r in st["records"]] == Va.tolist()
+            assert [r["Ea"] for r in st["records"]] == Ea.tolist()
+            assert [r["Via"] for r in st["records"]] == Via.tolist()
+            ctas = [r["ctas"] for r in st["records"]]
+            if solo[0] == "0":
+                assert all(c > 1 for c in ctas)
+            elif g.name.startswith("grid"):
+                assert any(c == 1 for c in ctas)
+
+
+def test_solo_tier_on_c2_grid(gsw):
+    """C2-shaped road grid: the autotuned BFS runs most levels on one CTA and stays bit-exact."""
+    g = gen.grid(2048)
+    G = gsw.Graph(g.off, g.col)
+    d, st = _bfs(G, 0, records=8192)
+    assert np.array_equal(d, oracle.bfs(g, 0))
+    assert sum(r["ctas"] == 1 for r in st["records"]) > 800     # the two corners of the diamond

@@ -38,12 +38,14 @@ JOBS = {
 
 def variants(algo):
     yield None
-    if algo in ("bfs", "cc", "sssp"):
+    if algo == "sssp":
+        # a forced SSSP variant pins the per-round stepping decision too (P4 candidates
+        # Increase / Decrease / Remain, plus static delta-stepping and Bellman-Ford)
+        for v in itertools.product(DIRS, FMTS, LBS, FUS, STEPS):
+            yield dict(direction=v[0], format=v[1], load_balance=v[2], fusion=v[3], stepping=v[4])
+    elif algo in ("bfs", "cc"):
         for v in itertools.product(DIRS, FMTS, LBS, FUS):
             yield dict(direction=v[0], format=v[1], load_balance=v[2], fusion=v[3])
-        if algo == "sssp":
-            for s in STEPS:
-                yield dict(stepping=s)
     else:
         for v in itertools.product(DIRS, LBS):
             yield dict(direction=v[0], load_balance=v[1])
@@ -54,6 +56,7 @@ def main():
     ap.add_argument("--json", default=None)
     ap.add_argument("--only", default=",".join(["C3:bfs", "C1:bfs", "C2:sssp", "C3:cc"]))
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--sssp-reps", type=int, default=1)
     ap.add_argument("--budget-ms", type=float, default=3000.0,
                     help="skip the remaining reps/roots of a variant slower than this")
     a = ap.parse_args()
@@ -84,7 +87,7 @@ def main():
             tot = 0.0
             for s in roots:
                 ms = []
-                for r in range(a.reps):
+                for r in range(a.sssp_reps if algo == "sssp" else a.reps):
                     flush.fill_(r)
                     torch.cuda.synchronize()
                     if algo == "bfs":

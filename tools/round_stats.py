@@ -22,3 +22,12 @@ for q in (10, 50, 90, 99):
 big = np.argsort(-(f + e))[:5]
 for i in big:
     print("  slow round", i, r[i])
+ct = np.array([x.get("ctas", 0) for x in r])
+for name, m in (("solo (ctas=1)", ct == 1), ("grid", ct != 1)):
+    if m.any():
+        print(f"  {name}: rounds={m.sum()} filter_us mean={f[m].mean():.2f} expand_us mean={e[m].mean():.2f} "
+              f"Va mean={va[m].mean():.0f} edges mean={ed[m].mean():.0f}")
+        for lo, hi in ((0, 16), (16, 128), (128, 512), (512, 1024), (1024, 1 << 30)):
+            mm = m & (va >= lo) & (va < hi)
+            if mm.any():
+                print(f"     Va in [{lo},{hi}): n={mm.sum()} us/round={(f[mm] + e[mm]).mean():.2f}")
