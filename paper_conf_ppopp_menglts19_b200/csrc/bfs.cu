@@ -10,6 +10,9 @@
 // Status (Fig. 11 filter): Active = depth==t, Inactive = depth<0 (not in the visited map),
 // Fixed = visited earlier.  compAtomic = atomicExch in the paper is applied only to
 // Inactive targets (reading R3): an atomicOr test-and-set on the visited bitmap.
+#include <cstdlib>
+#include <cstring>
+
 #include "engine.cuh"
 #include "internal.h"
 #include "launch.h"
@@ -783,6 +786,8 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     LaunchInfo li;
     gsw_status s = prepare_common(g, ws, (const void *)bfs_kernel, a.rc, li);
     if (s != GSW_OK) return s;
+    // BFS selector: hand-set rules (default) or the learned trees (GSW_SELECTOR=trees)
+    if (const char *sel = std::getenv("GSW_SELECTOR")) a.rc.base.selector = std::strcmp(sel, "trees") == 0 ? 1 : 0;
     if (!a.depth || !a.V || !a.fb[2] || !a.q[1] || !a.iq || !a.scan) { set_error("workspace too small"); return GSW_ENOMEM; }
     void *args[] = {&a};
     s = launch_persistent(g, (const void *)bfs_kernel, args, li);

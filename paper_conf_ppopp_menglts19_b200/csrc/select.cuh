@@ -5,6 +5,8 @@
 // fusion.  Those trees are not printed and the corpus is out of scope, so the trees
 // below are shallow hand-set if-else rules that encode the paper's stated findings (each rule
 // cites the sentence it follows) with thresholds calibrated on B200.
+// select_trees.cuh holds CART trees learned the paper's way on a synthetic brute-force corpus
+// (tools/selector_corpus.py + tools/train_selector.py); GSW_SELECTOR=trees uses them for BFS.
 // Every CTA evaluates the selector redundantly on identical inputs, so all CTAs agree on the
 // configuration without an extra barrier.
 #pragma once
@@ -22,6 +24,7 @@ struct Features {
     // historical information, lagged by one iteration (reading R9)
     float tf, te, Tf, Te;
     int iter;
+    int selector;   // 0: the hand-set rules below; 1: the learned trees (select_trees.cuh, GSW_SELECTOR=trees)
 };
 
 struct DevCfg {
@@ -29,6 +32,10 @@ struct DevCfg {
 };
 
 __device__ __forceinline__ int pick(int forced, int chosen) { return forced != GSW_AUTO ? forced : chosen; }
+
+}  // namespace gsw
+#include "select_trees.cuh"
+namespace gsw {
 
 // BFS-like traversal (BFS, BC forward): active = frontier, inactive = unvisited.
 // Direction split (P1).  The paper's stated finding is "the pull mode is preferable ... when the
@@ -47,6 +54,15 @@ __device__ __forceinline__ int traversal_direction(const Features &f) {
 
 __device__ __forceinline__ DevCfg select_traversal(const Features &f, const gsw_config &force) {
     DevCfg c;
+    if (f.selector == 1) {
+        // learned CART trees (R13b), in the paper's order
+        c.dir = pick(force.direction, tree_direction(f));
+        c.lb = pick(force.load_balance, tree_lb(f, c.dir));
+        c.fmt = pick(force.format, tree_format(f, c.dir, c.lb));
+        c.fused = pick(force.fusion, tree_fusion(f, c.dir, c.lb, c.fmt));
+        c.step = GSW_STEP_REMAIN;
+        return c;
+    }
     c.dir = pick(force.direction, traversal_direction(f));
     float cd = f.Va > 0 ? (float)f.Ea / (float)f.Va : 0.f;
     // P3 load balance: "TWC has the lowest overhead", "CM and WM perform better with irregular

@@ -155,3 +155,16 @@ def test_solo_tier_on_c2_grid(gsw):
     d, st = _bfs(G, 0, records=8192)
     assert np.array_equal(d, oracle.bfs(g, 0))
     assert sum(r["ctas"] == 1 for r in st["records"]) > 800     # the two corners of the diamond
+
+
+def test_learned_selector_parity(gsw, monkeypatch):
+    """GSW_SELECTOR=trees (the CART trees of select_trees.cuh) switches between
+    arbitrary pattern combinations per level; depths and per-level features stay exact."""
+    monkeypatch.setenv("GSW_SELECTOR", "trees")
+    for g in (gen.rmat(14, seed=8), gen.grid(83, 61), gen.chung_lu(20000, 200000, seed=5), tiny_graphs()["star5"]):
+        G = gsw.Graph(g.off, g.col)
+        for s in gen.sources(g, 3, seed=6):
+            d, st = _bfs(G, s, records=4096)
+            assert np.array_equal(d, oracle.bfs(g, s)), (g.name, s)
+            Va, Ea, Via, Eia = oracle.bfs_features(g, s)
+            assert [r["Va"] for r in st["records"]] == Va.tolist()

@@ -1,0 +1,91 @@
+#!/usr/bin/env python
+"""Training corpus for the learned selector (Sec. 4.4).
+
+The paper brute-forces every pattern combination per iteration on 644 real graphs and trains one
+CART tree per pattern on the 21 features of each iteration.  Here the corpus is
+synthetic (R-MAT at several skews / edge factors / scales, 2D grids, Chung-Lu power-law graphs --
+the evaluation graphs C1..C5 are NOT in it: other seeds and sizes), and the brute force uses the
+fact that BFS levels are unique: iteration t processes the same active set under every forced
+variant, so the per-iteration device times of the 60 forced runs (gsw_force_config) are directly
+comparable (the methodology of Fig. 14).
+
+Writes one JSON: for every (graph, root, level): the features and the time of every variant.
+
+  python tools/selector_corpus.py --json gpurun_out/selector_corpus.json
+"""
+import argparse
+import itertools
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+DIRS = ["push", "pull"]
+FMTS = ["bitmap", "queue", "sorted_queue"]
+LBS = ["thread", "twc", "wm", "cm", "strict"]
+FUS = ["standalone", "fused"]
+
+
+def corpus(gen):
+    out = []
+    for scale, ef, abc, seed in [(14, 8, (.57, .19, .19), 11), (14, 32, (.57, .19, .19), 12),
+                                 (15, 16, (.45, .25, .15), 13), (15, 16, (.70, .10, .10), 14),
+                                 (16, 8, (.57, .19, .19), 15), (16, 16, (.45, .15, .15), 16),
+                                 (17, 16, (.57, .19, .19), 17), (17, 4, (.57, .19, .19), 18),
+                                 (18, 16, (.57, .19, .19), 19), (18, 8, (.65, .15, .15), 20),
+                                 (19, 16, (.57, .19, .19), 21), (19, 32, (.50, .20, .20), 22),
+                                 (20, 16, (.57, .19, .19), 23), (20, 8, (.60, .15, .15), 24),
+                                 (21, 16, (.57, .19, .19), 25), (21, 24, (.50, .20, .20), 26)]:
+        out.append(gen.rmat(scale, ef, *abc, seed=seed))
+    for w, h in [(192, 192), (400, 100), (700, 700), (1400, 1000)]:
+        out.append(gen.grid(w, h))
+    for n, pairs, gamma, seed in [(200_000, 2_000_000, 2.1, 31), (300_000, 3_000_000, 2.5, 32),
+                                  (500_000, 4_000_000, 2.3, 33), (2_000_000, 24_000_000, 2.3, 34)]:
+        out.append(gen.chung_lu(n, pairs, gamma=gamma, i0=50.0, seed=seed))
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--json", required=True)
+    ap.add_argument("--roots", type=int, default=2)
+    a = ap.parse_args()
+    import torch
+    import gen
+    import paper_conf_ppopp_menglts19_b200 as gsw
+    variants = list(itertools.product(DIRS, FMTS, LBS, FUS))
+    rows = []
+    t0 = time.time()
+    for g in corpus(gen):
+        G = gsw.Graph(g.off, g.col)
+        attrs = G.attributes()
+        for s in gen.sources(g, a.roots, seed=99):
+            per = {}
+            levels = None
+            for v in variants:
+                G.force_config(direction=v[0], format=v[1], load_balance=v[2], fusion=v[3])
+                G.bfs(s)
+                _, st = G.bfs(s, records=1 << 15)
+                recs = st["records"]
+                # cost of iteration t's decision = its Expand + the NEXT iteration's Filter (the
+                # active-set materialisation the decision's output format/fusion forces on t+1)
+                per["-".join(v)] = [recs[i]["expand_us"] + (recs[i + 1]["filter_us"] if i + 1 < len(recs) else 0.0)
+                                    + (recs[i]["filter_us"] if i == 0 else 0.0) for i in range(len(recs))]
+                if levels is None:
+                    levels = [(r["Va"], r["Ea"], r["Via"], r["Eia"]) for r in recs]
+            G.force_config()
+            for t, (Va, Ea, Via, Eia) in enumerate(levels):
+                rows.append({"graph": g.name, "root": int(s), "t": t, "Va": Va, "Ea": Ea, "Via": Via, "Eia": Eia,
+                             "attrs": attrs, "times": {k: v[t] for k, v in per.items() if t < len(v)}})
+        print(f"{g.name}: n={g.n} nnz={g.nnz} levels={len(levels)} rows={len(rows)} {time.time() - t0:.0f}s", flush=True)
+        del G
+        torch.cuda.empty_cache()
+    with open(a.json, "w") as f:
+        json.dump(rows, f)
+
+
+if __name__ == "__main__":
+    main()
