@@ -110,16 +110,23 @@ __global__ void k_invert(const uint32_t *perm, int n, uint32_t *inv) {
     for (long long i = gtid(); i < n; i += gthreads()) inv[perm[i]] = (uint32_t)i;
 }
 // new row i = old row perm[i], columns renamed through inv; one warp per row
-__global__ void k_permute_rows(const uint32_t *noff, const uint32_t *off, const int32_t *col, const uint32_t *w,
-                               const uint32_t *perm, const uint32_t *inv, int n, int32_t *ncol, uint32_t *nw) {
+// rows in the new order, columns renamed, as 64-bit keys (new row << 32 | new column): one
+// device-wide radix sort of the keys then yields every row sorted (stable, ties keep weights)
+__global__ void k_permute_rows_keys(const uint32_t *noff, const uint32_t *off, const int32_t *col, const uint32_t *w,
+                                    const uint32_t *perm, const uint32_t *inv, int n, unsigned long long *keys,
+                                    uint32_t *nw) {
     for (long long i = gwarp(); i < n; i += gwarps()) {
         const uint32_t o = perm[i];
         const uint32_t b = off[o], e = off[o + 1], nb = noff[i];
+        const unsigned long long hi = (unsigned long long)i << 32;
         for (uint32_t k = b + lane_id(); k < e; k += 32) {
-            ncol[nb + (k - b)] = (int32_t)inv[col[k]];
+            keys[nb + (k - b)] = hi | inv[col[k]];
             if (w) nw[nb + (k - b)] = w[k];
         }
     }
+}
+__global__ void k_key_cols(const unsigned long long *keys, long long m, int32_t *col) {
+    for (long long k = gtid(); k < m; k += gthreads()) col[k] = (int32_t)(uint32_t)keys[k];
 }
 __global__ void k_set_u32(uint32_t *p, uint32_t v) { *p = v; }
 __global__ void k_perm_deg(const uint32_t *off, const uint32_t *perm, int n, uint32_t *degp) {
@@ -251,25 +258,33 @@ gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp) {
 // helps the early-exit pull.  Outputs are gathered back to caller ids by each kernel.
 static size_t al256(size_t x) { return (x + 255) & ~size_t(255); }
 
+static int key_end_bit(int64_t n) {
+    int b = 1;
+    while ((int64_t(1) << b) < n) ++b;
+    return 32 + b;
+}
+
 size_t relabel_temp_bytes(int64_t n, int64_t nnz, int has_w) {
     size_t t1 = 0, t2 = 0, t3 = 0;
     cub::DeviceRadixSort::SortPairsDescending(nullptr, t1, (uint32_t *)nullptr, (uint32_t *)nullptr,
                                               (uint32_t *)nullptr, (uint32_t *)nullptr, (int)n);
     cub::DeviceScan::InclusiveSum(nullptr, t2, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)n);
-    if (has_w)
-        cub::DeviceSegmentedSort::SortPairs(nullptr, t3, (int32_t *)nullptr, (int32_t *)nullptr, (uint32_t *)nullptr,
-                                            (uint32_t *)nullptr, (int)nnz, (int)n, (uint32_t *)nullptr,
-                                            (uint32_t *)nullptr);
-    else
-        cub::DeviceSegmentedSort::SortKeys(nullptr, t3, (int32_t *)nullptr, (int32_t *)nullptr, (int)nnz, (int)n,
-                                           (uint32_t *)nullptr, (uint32_t *)nullptr);
+    cub::DoubleBuffer<unsigned long long> kb(nullptr, nullptr);
+    cub::DoubleBuffer<uint32_t> vb(nullptr, nullptr);
+    if (has_w) cub::DeviceRadixSort::SortPairs(nullptr, t3, kb, vb, (int)nnz, 0, key_end_bit(n));
+    else cub::DeviceRadixSort::SortKeys(nullptr, t3, kb, (int)nnz, 0, key_end_bit(n));
     size_t t = std::max(t1, std::max(t2, t3));
-    return al256(t) + 3 * al256((size_t)n * 4) + al256((size_t)(n + 1) * 4) + al256((size_t)std::max<int64_t>(nnz, 1) * 4) * (has_w ? 2 : 1) + 4096;
+    const size_t m = (size_t)std::max<int64_t>(nnz, 1);
+    return al256(t) + 3 * al256((size_t)n * 4) + al256((size_t)(n + 1) * 4) + 2 * al256(m * 8) +
+           (has_w ? 2 * al256(m * 4) : 0) + 4096;
 }
 
+// Rows of the relabeled graph: permuted, columns renamed through inv, sorted ascending (so the
+// highest-degree neighbour comes first).  One 64-bit radix sort of (row, column) keys over all
+// edges -- a segmented sort spent most of its time in one CTA per hub row (C3: ~10 ms).
 static gsw_status relabel_csr(gsw_graph g, uint32_t *off, int32_t *col, uint32_t *w, const uint32_t *perm,
-                              const uint32_t *inv, uint32_t *degp, uint32_t *noff, int32_t *colT, uint32_t *wT,
-                              void *cub_tmp, size_t cub_bytes) {
+                              const uint32_t *inv, uint32_t *degp, uint32_t *noff, unsigned long long *k0,
+                              unsigned long long *k1, uint32_t *w0, uint32_t *w1, void *cub_tmp, size_t cub_bytes) {
     const int n = g->g.n;
     const int64_t nnz = g->g.nnz;
     cudaStream_t s = g->stream;
@@ -277,12 +292,21 @@ static gsw_status relabel_csr(gsw_graph g, uint32_t *off, int32_t *col, uint32_t
     size_t cb = cub_bytes;
     GSW_CUDA(cub::DeviceScan::InclusiveSum(cub_tmp, cb, degp, noff + 1, n, s));
     k_set_u32<<<1, 1, 0, s>>>(noff, 0u);
-    k_permute_rows<<<grid_for((long long)n * 32, g->sms), kBlock, 0, s>>>(noff, off, col, w, perm, inv, n, colT, wT);
+    k_permute_rows_keys<<<grid_for((long long)n * 32, g->sms), kBlock, 0, s>>>(noff, off, col, w, perm, inv, n, k0, w0);
     GSW_CUDA(cudaGetLastError());
     GSW_CUDA(cudaMemcpyAsync(off, noff, (size_t)(n + 1) * 4, cudaMemcpyDeviceToDevice, s));
+    if (nnz == 0) return GSW_OK;
     cb = cub_bytes;
-    if (w) GSW_CUDA(cub::DeviceSegmentedSort::SortPairs(cub_tmp, cb, colT, col, wT, w, (int)nnz, n, noff, noff + 1, s));
-    else GSW_CUDA(cub::DeviceSegmentedSort::SortKeys(cub_tmp, cb, colT, col, (int)nnz, n, noff, noff + 1, s));
+    cub::DoubleBuffer<unsigned long long> kb(k0, k1);
+    if (w) {
+        cub::DoubleBuffer<uint32_t> vb(w0, w1);
+        GSW_CUDA(cub::DeviceRadixSort::SortPairs(cub_tmp, cb, kb, vb, (int)nnz, 0, key_end_bit(n), s));
+        GSW_CUDA(cudaMemcpyAsync(w, vb.Current(), (size_t)nnz * 4, cudaMemcpyDeviceToDevice, s));
+    } else {
+        GSW_CUDA(cub::DeviceRadixSort::SortKeys(cub_tmp, cb, kb, (int)nnz, 0, key_end_bit(n), s));
+    }
+    k_key_cols<<<grid_for(nnz, g->sms), kBlock, 0, s>>>(kb.Current(), nnz, col);
+    GSW_CUDA(cudaGetLastError());
     return GSW_OK;
 }
 
@@ -294,8 +318,9 @@ gsw_status relabel_graph(gsw_graph g, uint32_t *perm, uint32_t *inv, char *tmp, 
     Workspace t{tmp, tmp_bytes, 0};
     uint32_t *deg = (uint32_t *)t.take((size_t)n * 4), *ids = (uint32_t *)t.take((size_t)n * 4);
     uint32_t *degs = (uint32_t *)t.take((size_t)n * 4), *noff = (uint32_t *)t.take((size_t)(n + 1) * 4);
-    int32_t *colT = (int32_t *)t.take((size_t)std::max<int64_t>(nnz, 1) * 4);
-    uint32_t *wT = has_w ? (uint32_t *)t.take((size_t)std::max<int64_t>(nnz, 1) * 4) : nullptr;
+    const size_t m = (size_t)std::max<int64_t>(nnz, 1);
+    unsigned long long *k0 = (unsigned long long *)t.take(m * 8), *k1 = (unsigned long long *)t.take(m * 8);
+    uint32_t *w0 = has_w ? (uint32_t *)t.take(m * 4) : nullptr, *w1 = has_w ? (uint32_t *)t.take(m * 4) : nullptr;
     size_t cub_bytes = tmp_bytes - t.used - 512;
     void *cub_tmp = t.take(cub_bytes);
     cudaStream_t s = g->stream;
@@ -305,11 +330,11 @@ gsw_status relabel_graph(gsw_graph g, uint32_t *perm, uint32_t *inv, char *tmp, 
     k_invert<<<grid_for(n, g->sms), kBlock, 0, s>>>(perm, n, inv);
     GSW_CUDA(cudaGetLastError());
     gsw_status st = relabel_csr(g, (uint32_t *)g->g.off, (int32_t *)g->g.col, (uint32_t *)g->g.w, perm, inv, degs,
-                                noff, colT, wT, cub_tmp, cub_bytes);
+                                noff, k0, k1, w0, w1, cub_tmp, cub_bytes);
     if (st != GSW_OK) return st;
     if (!g->symmetric) {
         st = relabel_csr(g, (uint32_t *)g->g.in_off, (int32_t *)g->g.in_col, (uint32_t *)g->g.in_w, perm, inv, degs,
-                         noff, colT, wT, cub_tmp, cub_bytes);
+                         noff, k0, k1, w0, w1, cub_tmp, cub_bytes);
         if (st != GSW_OK) return st;
     }
     g->g.perm = perm;

@@ -52,6 +52,8 @@ gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCom
     f.N = (float)A.N; f.M = (float)A.M; f.dbar = (float)A.dbar; f.sd = (float)A.sd; f.rd = (float)A.rd;
     f.gini = (float)A.gini; f.her = (float)A.her;
     rc.base = f;
+    // the run's device time starts here: the control-block reset below is part of the call
+    GSW_CUDA(cudaEventRecord(g->ev0, g->stream));
     // solo tier (CTA 0 alone for tiny active sets); GSW_SOLO_E / GSW_SOLO_V override (calibration)
     rc.solo_e = env_ll("GSW_SOLO_E", kSoloE);
     rc.solo_v = env_ll("GSW_SOLO_V", kSoloV);
@@ -60,7 +62,6 @@ gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCom
 }
 
 gsw_status launch_persistent(gsw_graph g, const void *kernel, void **args, const LaunchInfo &li) {
-    GSW_CUDA(cudaEventRecord(g->ev0, g->stream));
     GSW_CUDA(cudaLaunchCooperativeKernel(kernel, dim3(li.grid), dim3(kBlock), args, 0, g->stream));
     GSW_CUDA(cudaEventRecord(g->ev1, g->stream));
     return GSW_OK;

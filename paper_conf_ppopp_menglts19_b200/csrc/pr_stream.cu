@@ -410,6 +410,7 @@ gsw_status run_pr_stream(gsw_graph g, double damping, int32_t iters, double *ran
     f.N = (float)A.N; f.M = (float)A.M; f.dbar = (float)A.dbar; f.sd = (float)A.sd; f.rd = (float)A.rd;
     f.gini = (float)A.gini; f.her = (float)A.her;
     rc.base = f;
+    GSW_CUDA(cudaEventRecord(g->ev0, g->stream));   // device time of the call starts with its resets
     GSW_CUDA(cudaMemsetAsync(rc.ctl, 0, sizeof(Ctl), g->stream));
     GSW_CUDA(cudaMemsetAsync(a.nempty, 0, 4, g->stream));
     GSW_CUDA(cudaFuncSetAttribute((const void *)pr_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -418,7 +419,6 @@ gsw_status run_pr_stream(gsw_graph g, double damping, int32_t iters, double *ran
     GSW_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, (const void *)pr_stream_kernel, kSBlock, smem));
     if (nb < 1) { set_error("pr_stream_kernel does not fit on an SM"); return GSW_ECUDA; }
     void *args[] = {&a};
-    GSW_CUDA(cudaEventRecord(g->ev0, g->stream));
     GSW_CUDA(cudaLaunchCooperativeKernel((const void *)pr_stream_kernel, dim3(g->sms), dim3(kSBlock), args, smem,
                                          g->stream));
     GSW_CUDA(cudaEventRecord(g->ev1, g->stream));
