@@ -63,24 +63,29 @@ struct GridBarrier {
 };
 constexpr uint64_t kBarrierTimeoutNs = 20ull * 1000 * 1000 * 1000;
 
-// (tools/micro_barrier.cu on B200: this acq_rel-arrive + release-publish form costs 1.6-1.9 us at
-// 148-592 CTAs; the fence-heavy form 1.9-2.4 us.)
+// Flip-bit barrier (the cooperative-groups scheme): CTA 0 adds 2^31 - (gridDim - 1), every other
+// CTA adds 1, so the counter's top bit flips exactly when the last CTA arrives; waiters poll the
+// word until they see the flip.  One atomic per CTA and no separate publish store by the last
+// arriver (tools/micro_barrier.cu on B200, 592 CTAs: 1.61 us vs 1.85 us for the acq_rel
+// counter + generation-word form).  The counter must be 0 when the kernel starts (prepare_common).
+__device__ __forceinline__ unsigned ld_volatile_u32(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
 __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch) {
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned target = epoch + 1;
-        unsigned prev;
-        asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(prev) : "l"(b.arrive) : "memory");
-        if (prev == target * gridDim.x - 1) {
-            st_release(b.gen, target);
-        } else {
-            uint64_t t0 = globaltimer();
-            unsigned spins = 0;
-            while (ld_acquire(b.gen) < target) {
-                if (((++spins) & 1023u) == 0 && globaltimer() - t0 > kBarrierTimeoutNs) {
-                    atomicExch(b.err, 0xBA4u);
-                    __trap();
-                }
+        const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;
+        __threadfence();
+        const unsigned old = atomicAdd(b.arrive, add);
+        uint64_t t0 = 0;
+        unsigned spins = 0;
+        while (((old ^ ld_volatile_u32(b.arrive)) & 0x80000000u) == 0u) {
+            if (((++spins) & 1023u) == 0) {
+                const uint64_t now = globaltimer();
+                if (t0 == 0) t0 = now;
+                else if (now - t0 > kBarrierTimeoutNs) { atomicExch(b.err, 0xBA4u); __trap(); }
             }
         }
         __threadfence();
@@ -95,20 +100,16 @@ __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch)
 __device__ __forceinline__ void grid_park(const GridBarrier &b, unsigned &epoch) {
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned target = epoch + 1;
-        unsigned prev;
-        asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(prev) : "l"(b.arrive) : "memory");
-        if (prev == target * gridDim.x - 1) {
-            st_release(b.gen, target);
-        } else {
-            uint64_t t0 = globaltimer();
-            unsigned spins = 0;
-            while (ld_acquire(b.gen) < target) {
-                __nanosleep(200);
-                if (((++spins) & 255u) == 0 && globaltimer() - t0 > kBarrierTimeoutNs) {
-                    atomicExch(b.err, 0xBA5u);
-                    __trap();
-                }
+        const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;
+        __threadfence();
+        const unsigned old = atomicAdd(b.arrive, add);
+        const uint64_t t0 = globaltimer();
+        unsigned spins = 0;
+        while (((old ^ ld_volatile_u32(b.arrive)) & 0x80000000u) == 0u) {
+            __nanosleep(200);
+            if (((++spins) & 255u) == 0 && globaltimer() - t0 > kBarrierTimeoutNs) {
+                atomicExch(b.err, 0xBA5u);
+                __trap();
             }
         }
         __threadfence();
