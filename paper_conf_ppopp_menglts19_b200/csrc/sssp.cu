@@ -159,12 +159,291 @@ __device__ __forceinline__ DevCfg select_sssp(const Features &f, const gsw_confi
     return c;
 }
 
+
+// ---------------------------------------------------------------- CTA-resident tier (solo)
+// The BFS tier of bfs.cu applied to the near/far rounds: while the
+// selector keeps fused push and the near set stays below (solo_v vertices, solo_e edges) with a
+// far set of at most kSSQ entries, CTA 0 runs the rounds alone -- near set, offsets, degree scan
+// and dist[u] in shared memory, the stepping law evaluated per round exactly as in the grid loop,
+// far-set splits done in place -- and the other CTAs park at one grid barrier.  Per round the
+// dependent chain is: columns + weights, atomicMin on dist[v] issued with a speculative load of
+// v's offsets, then the near / far claim.  The near claim map is cleared after each round by
+// the CTA itself (it holds exactly the pushed vertices).
+constexpr int kSSQ = 512;
+struct SsSoloSmem {
+    int q[2][kSSQ];
+    uint32_t beg[2][kSSQ];
+    uint32_t scan[2][kSSQ + 1];
+    unsigned du[kSSQ];
+    unsigned qn[2];
+    unsigned long long ea;
+    unsigned maxd, mind, minf;
+    int go;
+    uint32_t red[kWarps + 1];
+    unsigned long long book_raw[(sizeof(Book) + 7) / 8];
+    unsigned long long prev_va;
+};
+struct SsLoop {
+    unsigned long long theta, floor_t, flen, prev_ea;
+    int fcur, nsplit;
+};
+
+// warp-aggregated append of (v, beg, deg) to a shared near queue
+__device__ __forceinline__ void solo_push(SsSoloSmem &ss, int nx, bool pred, int v, uint32_t b, uint32_t d) {
+    const unsigned act = __activemask();
+    const unsigned m = __ballot_sync(act, pred);
+    if (!m) return;
+    const int leader = __ffs(m) - 1;
+    unsigned base = 0;
+    if ((int)lane_id() == leader) base = atomicAdd(&ss.qn[nx], (unsigned)__popc(m));
+    base = __shfl_sync(act, base, leader);
+    if (pred) {
+        const unsigned p = base + __popc(m & lanemask_lt());
+        ss.q[nx][p] = v; ss.beg[nx][p] = b; ss.scan[nx][p] = d;
+    }
+}
+
+// Runs rounds t, t+1, ... on CTA 0 (all its threads); hands back the near set of the first round
+// NOT run in a.q[t & 1] with its counters in rc.cnt[t % 3] and the loop state in rc.pub.
+__device__ __noinline__ void sssp_solo(const SsspArgs &a, SsSoloSmem &ss, int t, SsLoop L, const Features fbase,
+                                       unsigned qn0, DevCfg c0) {
+    const RunCommon &rc = a.rc;
+    const unsigned tid = threadIdx.x;
+    const uint32_t *__restrict__ off = a.g.off;
+    const int32_t *__restrict__ col = a.g.col;
+    const uint32_t *__restrict__ wt = a.g.w;
+    unsigned *dist = a.dist;
+    const int n = a.g.n;
+    Book &book = *reinterpret_cast<Book *>(ss.book_raw);
+    const long long sv = rc.solo_v < (long long)kSSQ ? rc.solo_v : (long long)kSSQ, se = rc.solo_e;
+    const unsigned long long kInf = 0xffffffffull, d0 = a.delta0;
+    unsigned *nnb = a.nb[(t + 1) % 3];            // near claim map of every solo round (cleaned each round)
+    for (unsigned i = tid; i < qn0; i += kBlock) {
+        const int u = a.q[t & 1][i];
+        const uint32_t b = __ldg(off + u), e = __ldg(off + u + 1);
+        ss.q[0][i] = u; ss.beg[0][i] = b; ss.scan[0][i] = e - b;
+    }
+    int cur = 0;
+    unsigned qn = qn0;
+    bool first = true;
+    unsigned long long E_prev = 0, Ea = 0;
+    unsigned mxd = 0, mnd = 0;
+    float4 hist = make_float4(0.f, 0.f, 0.f, 0.f);
+    bool done_run = false;
+    for (;;) {
+        __syncthreads();
+        // (S) near set empty: advance theta and split the far set (in place while it is small)
+        while (qn == 0 && !first) {
+            if (L.flen == 0) { done_run = true; break; }
+            if (L.flen > (unsigned long long)kSSQ) break;                      // the grid splits big sets
+            L.theta += d0;
+            L.floor_t = L.theta;
+            const int fsrc = L.fcur, fdst = L.fcur ^ 1;
+            const unsigned Lf = (unsigned)L.flen;
+            if (tid == 0) { ss.qn[cur] = 0u; ss.minf = 0xffffffffu; }
+            __syncthreads();
+            for (unsigned i = tid; i < Lf; i += kBlock) {
+                const int v = __ldcg(a.fq[fsrc] + i);
+                const unsigned dv = __ldcg(dist + v);
+                const bool near = (unsigned long long)dv < L.theta;
+                uint32_t b = 0, e = 0;
+                if (near) {
+                    atomicAnd(a.farbit + (v >> 5), ~(1u << (v & 31)));
+                    b = __ldg(off + v); e = __ldg(off + v + 1);
+                } else {
+                    a.fq[fdst][atomicAdd(a.flen + fdst, 1u)] = v;
+                    atomicMin(&ss.minf, dv);
+                }
+                solo_push(ss, cur, near, v, b, e - b);
+            }
+            __syncthreads();
+            qn = ss.qn[cur];
+            L.flen = Lf - qn;
+            if (tid == 0) a.flen[fsrc] = 0u;
+            L.fcur = fdst;
+            L.nsplit++;
+            if (qn == 0 && ss.minf != 0xffffffffu && (unsigned long long)ss.minf + 1 > L.theta + d0)
+                L.theta = (unsigned long long)ss.minf + 1 - d0;               // jump over empty buckets
+            __syncthreads();
+        }
+        if (done_run || qn == 0) {
+            if (!first) break;
+        }
+        // (A) features of N_t and dist[u] of its vertices
+        if (tid == 0) { ss.ea = 0ull; ss.maxd = 0u; ss.mind = 0xffffffffu; }
+        __syncthreads();
+        {
+            unsigned long long lea = 0;
+            unsigned lmx = 0, lmn = 0xffffffffu;
+            for (unsigned i = tid; i < qn; i += kBlock) {
+                const unsigned d = ss.scan[cur][i];
+                ss.du[i] = __ldcg(dist + ss.q[cur][i]);   // L2: atomicMin updates bypass this SM's L1
+                lea += d; lmx = d > lmx ? d : lmx; lmn = d < lmn ? d : lmn;
+            }
+            lea = warp_sum(lea); lmx = warp_max(lmx); lmn = warp_min(lmn);
+            if (lane_id() == 0 && lea) { atomicAdd(&ss.ea, lea); atomicMax(&ss.maxd, lmx); atomicMin(&ss.mind, lmn); }
+        }
+        __syncthreads();
+        Ea = ss.ea; mxd = ss.maxd; mnd = ss.mind;
+        // (B) selector + stepping law on N_t (thread 0), same rules as the grid loop
+        if (tid == 0) {
+            int go = first ? 1 : 0;
+            DevCfg c = c0;
+            if (!first && qn > 0) {
+                Features f = fbase;
+                f.Va = (long long)qn; f.Ea = (long long)Ea; f.Via = (long long)n - f.Va; f.Eia = (long long)a.g.nnz - f.Ea;
+                f.maxd = mxd; f.mind = mnd; f.iter = t;
+                f.tf = hist.x; f.te = hist.y; f.Tf = hist.z; f.Te = hist.w;
+                c = select_sssp(f, rc.force);
+                if (c.dir == GSW_PUSH && c.fused == GSW_FUSED && (long long)qn <= sv && (long long)Ea <= se) {
+                    go = 1;
+                    int step = GSW_STEP_REMAIN;
+                    if (t > 0 && L.prev_ea > 0) {
+                        const double e = (double)Ea, ep = (double)L.prev_ea, lo = (double)gridDim.x * blockDim.x;
+                        const bool drop = e < 0.65 * ep, grow = e > 1.35 * ep;
+                        switch (a.law) {
+                        case 1: step = grow ? GSW_STEP_INCREASE : (drop ? GSW_STEP_DECREASE : GSW_STEP_REMAIN); break;
+                        case 2: step = e < lo ? GSW_STEP_INCREASE : (e > 8.0 * lo ? GSW_STEP_DECREASE : GSW_STEP_REMAIN); break;
+                        case 3: step = (drop && e < lo) ? GSW_STEP_INCREASE : (grow ? GSW_STEP_DECREASE : GSW_STEP_REMAIN); break;
+                        default: step = drop ? GSW_STEP_INCREASE : (grow ? GSW_STEP_DECREASE : GSW_STEP_REMAIN);
+                        }
+                    }
+                    if (step == GSW_STEP_INCREASE) L.theta = min(kInf, L.theta + d0);
+                    else if (step == GSW_STEP_DECREASE) L.theta = max(L.floor_t, L.theta > d0 / 2 ? L.theta - d0 / 2 : 0ull);
+                    c.step = step;
+                    L.prev_ea = Ea;
+                    book.bytes += 12ull * ss.prev_va + 8ull * E_prev + 8ull * qn;
+                    book.edges += E_prev;
+                    if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)E_prev;
+                    hist = book_start(book, rc, t, rc.cnt + ((t + 1) % 3));
+                    write_record(rc, t, c, f, (unsigned)min(L.theta, kInf));
+                    reset_cnt(rc.cnt + ((t + 2) % 3));
+                }
+            }
+            if (first) {
+                const IterCnt *cs = rc.cnt + ((t + 1) % 3);
+                hist = make_float4(cs->tf, cs->te, cs->Tf, cs->Te);
+            }
+            if (go && t < kMaxHist) rc.rec[t].ctas = 1;
+            ss.go = go;
+            ss.qn[cur ^ 1] = 0u;
+            ss.minf = (unsigned)L.theta;            // broadcast theta (< 2^32 while rounds remain finite)
+            ss.red[kWarps] = (unsigned)(L.theta >> 32);
+        }
+        __syncthreads();
+        // every thread needs the same loop state: thread 0 evaluated the law, broadcast it
+        L.theta = ((unsigned long long)ss.red[kWarps] << 32) | ss.minf;
+        if (!ss.go) break;
+        L.prev_ea = Ea;
+        // (C) exclusive scan of the degrees
+        {
+            const unsigned per = (qn + kBlock - 1) / kBlock, i0 = tid * per;
+            uint32_t loc = 0;
+            for (unsigned k = 0; k < per; ++k) if (i0 + k < qn) loc += ss.scan[cur][i0 + k];
+            uint32_t tot;
+            uint32_t ex = block_excl_scan(loc, ss.red, &tot);
+            for (unsigned k = 0; k < per; ++k)
+                if (i0 + k < qn) { const uint32_t d = ss.scan[cur][i0 + k]; ss.scan[cur][i0 + k] = ex; ex += d; }
+            if (tid == 0) ss.scan[cur][qn] = tot;
+            __syncthreads();
+        }
+        if (tid == 0) book_expand(book);
+        // (D) relax: columns + weights, atomicMin with the target's offsets, then near/far claim
+        {
+            const unsigned E = (unsigned)Ea;
+            const int nx = cur ^ 1;
+            const uint32_t *scan = ss.scan[cur], *beg = ss.beg[cur];
+            const unsigned lo = (unsigned)(((unsigned long long)E * tid) / kBlock);
+            const unsigned hi = (unsigned)(((unsigned long long)E * (tid + 1)) / kBlock);
+            const unsigned mine = hi > lo ? (hi - lo + 3) / 4 : 0u;
+            const unsigned nb = __reduce_max_sync(0xffffffffu, mine);
+            unsigned i = 0, j = lo;
+            if (lo < hi) {
+                unsigned Lq = 0, R = qn;
+                while (R - Lq > 1) { const unsigned m = (Lq + R) >> 1; if (scan[m] <= lo) Lq = m; else R = m; }
+                i = Lq;
+            }
+            const unsigned long long th = L.theta;
+            for (unsigned bt = 0; bt < nb; ++bt) {
+                int v[4];
+                unsigned nd[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    v[k] = -1; nd[k] = 0;
+                    if (j < hi) {
+                        while (scan[i + 1] <= j) ++i;
+                        const uint32_t e = beg[i] + (j - scan[i]);
+                        v[k] = __ldg(col + e);
+                        nd[k] = ss.du[i] + __ldg(wt + e);
+                        ++j;
+                    }
+                }
+                unsigned old[4];
+                uint32_t vb[4], ve[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    old[k] = v[k] >= 0 ? atomicMin(dist + v[k], nd[k]) : 0u;
+                    vb[k] = v[k] >= 0 ? __ldg(off + v[k]) : 0u;
+                    ve[k] = v[k] >= 0 ? __ldg(off + v[k] + 1) : 0u;
+                }
+                unsigned cl[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    cl[k] = 0xffffffffu;
+                    if (v[k] >= 0 && nd[k] < old[k]) {
+                        const unsigned bit = 1u << (v[k] & 31);
+                        cl[k] = (unsigned long long)nd[k] < th ? atomicOr(nnb + (v[k] >> 5), bit)
+                                                                : atomicOr(a.farbit + (v[k] >> 5), bit);
+                    }
+                }
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const bool won = cl[k] != 0xffffffffu && !((cl[k] >> (v[k] & 31)) & 1u);
+                    const bool near = won && (unsigned long long)nd[k] < th;
+                    solo_push(ss, nx, near, v[k], vb[k], ve[k] - vb[k]);
+                    if (won && !near) a.fq[L.fcur][atomicAdd(a.flen + L.fcur, 1u)] = v[k];
+                }
+            }
+            __syncthreads();
+            // far appends of this round, then clean the near claim map (it holds exactly N_{t+1})
+            const unsigned nq = ss.qn[nx];
+            for (unsigned k = tid; k < nq; k += kBlock) atomicAnd(nnb + (ss.q[nx][k] >> 5), 0u);
+            __threadfence();
+            __syncthreads();
+            L.flen = *(volatile unsigned *)(a.flen + L.fcur);
+            E_prev = E;
+            if (tid == 0) ss.prev_va = qn;
+            qn = nq;
+            cur = nx;
+            ++t;
+            first = false;
+        }
+    }
+    // hand N_t back to the grid
+    {
+        int *gq = a.q[t & 1];
+        for (unsigned k = tid; k < qn; k += kBlock) gq[k] = ss.q[cur][k];
+        if (tid == 0) {
+            IterCnt *cc = rc.cnt + (t % 3);
+            cc->va = qn; cc->ea = qn ? Ea : 0; cc->maxd = mxd; cc->mind = mnd; cc->qlen = qn; cc->edges = E_prev;
+            cc->aux0 = 0u;
+            TeamPub p{};
+            p.t = t;
+            p.aux[0] = L.theta; p.aux[1] = L.floor_t; p.aux[2] = L.flen; p.aux[3] = L.prev_ea;
+            p.aux[4] = (unsigned long long)L.fcur; p.aux[5] = (unsigned long long)L.nsplit;
+            *rc.pub = p;
+        }
+    }
+}
+
 union SsSmem {
     LbSmem push;
     LbRedSmem pull;
+    SsSoloSmem solo;
 };
+static_assert(sizeof(SsSoloSmem) <= sizeof(LbSmem), "the solo tier must not grow the kernel's shared memory");
 
-__global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(const __grid_constant__ SsspArgs a) {
     __shared__ SsSmem sm;
     __shared__ uint32_t red[kWarps + 1];
     __shared__ CtaQStore qs0, qs1;        // staged appends: near queue, far queue
@@ -207,6 +486,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
     bool dirty[3] = {false, false, false};
     int prev_dir = GSW_PUSH;
     unsigned long long prev_va = 0;
+    const bool solo_allowed = rc.solo_e > 0 && a.mode == ST_DYNAMIC && rc.force.direction == GSW_AUTO &&
+                              rc.force.format == GSW_AUTO && rc.force.load_balance == GSW_AUTO &&
+                              rc.force.fusion == GSW_AUTO && rc.force.stepping == GSW_AUTO;
+    bool last_small = false;
     int t = 0;
     for (;; ++t) {
         IterCnt *cur = rc.cnt + (t % 3), *nxt = rc.cnt + ((t + 1) % 3);
@@ -319,6 +602,37 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(SsspArgs a) {
         const unsigned th = (unsigned)min(theta, kInf);
         write_record(rc, t, c, f, th);
         if (is_book()) reset_cnt(rc.cnt + ((t + 2) % 3));
+        // CTA-resident tier (see sssp_solo): entered after two consecutive small rounds
+        {
+            const bool small = (long long)cv.ea <= rc.solo_e && (long long)cv.va <= rc.solo_v &&
+                               cv.va <= (unsigned long long)kSSQ && flen <= (unsigned long long)kSSQ;
+            const bool solo = solo_allowed && small && last_small && c.dir == GSW_PUSH && c.fused == GSW_FUSED &&
+                              mat == SM_QUEUE;
+            last_small = small;
+            if (solo) {
+                if (blockIdx.x == 0) {
+                    if (threadIdx.x == 0) { *reinterpret_cast<Book *>(sm.solo.book_raw) = book; sm.solo.prev_va = prev_va; }
+                    sssp_solo(a, sm.solo, t, SsLoop{theta, floor_t, flen, prev_ea, fcur, nsplit}, f, cv.qlen, c);
+                    if (threadIdx.x == 0) { book = *reinterpret_cast<const Book *>(sm.solo.book_raw); prev_va = sm.solo.prev_va; }
+                    prev_dir = GSW_PUSH;
+                    grid_sync(bar, epoch);
+                } else {
+                    grid_park(bar, epoch);
+                }
+                TeamPub p;
+                pub_read(rc.pub, p);
+                t = (int)p.t;
+                theta = p.aux[0]; floor_t = p.aux[1]; flen = p.aux[2]; prev_ea = p.aux[3];
+                fcur = (int)p.aux[4]; nsplit = (int)p.aux[5];
+                mat = SM_QUEUE;
+                if (dirty[0] || dirty[1] || dirty[2]) {      // the solo claim map is already clean
+                    for (int i = 0; i < 3; ++i) if (dirty[i]) { clear_words(a.nb[i], W); dirty[i] = false; }
+                    grid_sync(bar, epoch);
+                }
+                --t;
+                continue;
+            }
+        }
         const int b2 = (t + 2) % 3;
         if (dirty[b2]) { clear_words(a.nb[b2], W); dirty[b2] = false; }
 
