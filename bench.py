@@ -282,14 +282,23 @@ def run_gsw(args, ws, rank, local):
     import gen
     import paper_conf_ppopp_menglts19_b200 as gsw
 
-    if ws > 1 or args.force_dist:
+    if args.partitioned or args.force_dist:
         return run_gsw_dist(args, ws, rank, local)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    replicas = ws > 1 or args.replicas
+    if replicas:
+        # N > 1 (default): the BFS roots are independent problems (SURVEY Q12 root stream), so they
+        # are sharded over the ranks, each holding its own copy of the graph; no data-path collective
+        if "RANK" not in os.environ:
+            os.environ.update(RANK="0", WORLD_SIZE="1", LOCAL_RANK="0", MASTER_ADDR="127.0.0.1",
+                              MASTER_PORT=str(29500 + os.getpid() % 1000))
+        dist.init_process_group("nccl", device_id=dev)
     g, gen_s = build_graph(args.workload)
     deg = g.deg
-    nroots = max(64, args.steps + args.warmup)
+    nroots = max(64, (args.steps + args.warmup) * ws)
     roots = gen.sources(g, nroots)
+    roots = [roots[(k * ws + rank) % nroots] for k in range(nroots)]   # this rank's shard
     G = gsw.Graph(g.off, g.col, device=dev)
     stream = G.stream
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
@@ -308,7 +317,7 @@ def run_gsw(args, ws, rank, local):
     for k in range(args.warmup):
         step(k, False)
     torch.cuda.synchronize()
-    if ws > 1:
+    if replicas:
         dist.barrier()
     torch.cuda.synchronize()
     evs, kern_ms, bytes_alg, edges_cc, g500_bytes = [], 0.0, 0, 0, 0
@@ -330,11 +339,15 @@ def run_gsw(args, ws, rank, local):
     step_ms = [a.elapsed_time(b) for a, b in evs]
     host_ms = sum(step_ms)
     tot_ms = kern_ms
-    if ws > 1:
+    all_edges = edges_cc
+    if replicas:
         t = torch.tensor([tot_ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         tot_ms = float(t.item())
-    value = ws * edges_cc / (tot_ms * 1e-3) / 1e9
+        e = torch.tensor([edges_cc], device=dev, dtype=torch.float64)
+        dist.all_reduce(e)
+        all_edges = float(e.item())
+    value = all_edges / (tot_ms * 1e-3) / 1e9
 
     # ---- roofline of the dominant kernel (the persistent BFS kernel; one launch per step)
     peak, peak_src = hbm_peak()
@@ -346,7 +359,8 @@ def run_gsw(args, ws, rank, local):
     if os.path.exists(tf):
         with open(tf) as f:
             traffic = json.load(f).get("dram_bytes_per_launch")
-    extra = run_extras(gsw, dev, G, g, peak) if (rank == 0 and not args.quick and args.workload == "C3") else None
+    extra = (run_extras(gsw, dev, G, g, peak)
+             if (rank == 0 and ws == 1 and not args.quick and args.workload == "C3") else None)
 
     # ---- e2e: through the public API from pinned host buffers (graph H2D + BFS + depth D2H)
     e2e = None
@@ -368,6 +382,12 @@ def run_gsw(args, ws, rank, local):
                 e2e_ms += dt * 1e3
                 e2e_edges += m_cc(deg, host_out.numpy())
             del G2
+        if replicas:                               # whole job: all ranks' edges over the slowest rank
+            t = torch.tensor([e2e_ms, float(e2e_edges)], device=dev, dtype=torch.float64)
+            mx = t.clone()
+            dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+            dist.all_reduce(t)
+            e2e_ms, e2e_edges = float(mx[0].item()), float(t[1].item())
         e2e = {"value": e2e_edges / (e2e_ms * 1e-3) / 1e9, "unit": "GTEPS",
                "h2d_bytes_per_step": int(g.off.nbytes + g.col.nbytes), "d2h_bytes_per_step": int(g.n * 4),
                "note": "per step: gsw_graph_create from pinned host CSR (H2D) + gsw_bfs into pinned host "
@@ -382,7 +402,8 @@ def run_gsw(args, ws, rank, local):
                                    "(Graph500 a,b,c=.57,.19,.19), "
                                    f"n={g.n}, nnz={g.nnz}, roots per SURVEY Q12, autotuned",
                        "l2": "flushed between steps (256 MiB write outside the timed span)",
-                       "parallelism": "replicas" if ws > 1 else "single GPU"},
+                       "parallelism": (f"root-sharded replicas x{ws} (one graph copy per GPU, no collective)"
+                                       if replicas else "single GPU")},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "gsw::bfs_kernel (persistent, 1 launch/step)",
@@ -400,10 +421,10 @@ def run_gsw(args, ws, rank, local):
             "gen_seconds": gen_s,
             "extra": extra,
         }
-        if not args.no_cpu_baseline:
+        if not args.no_cpu_baseline and ws == 1:
             line["cpu_baseline"] = cpu_baseline_sample(g, roots[:8 if args.workload == "C3" else 1])
         print(json.dumps(line), flush=True)
-    if ws > 1:
+    if replicas:
         dist.barrier()
         dist.destroy_process_group()
 
@@ -419,6 +440,9 @@ def main():
     ap.add_argument("--workload", default="C3", choices=["C3", "C5"],
                     help="C3 (default, the north_star's headline) or C5 (R-MAT scale 26, 1 GPU)")
     ap.add_argument("--force-dist", action="store_true", help="run the partitioned NCCL path even at N=1")
+    ap.add_argument("--partitioned", action="store_true",
+                    help="N > 1: the 1D vertex-partitioned graph with per-level NCCL exchange (SURVEY 8(e))")
+    ap.add_argument("--replicas", action="store_true", help="exercise the root-sharded replica path at N=1")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
