@@ -28,7 +28,7 @@
 
 namespace gsw {
 
-constexpr int kSBlock = 768;
+constexpr int kSBlock = 1024;
 constexpr int kSWarps = kSBlock / 32;
 constexpr int kEpt = 8;                       // edges per lane per warp-tile
 constexpr int kWt = 32 * kEpt;                // edges per warp-tile
