@@ -99,7 +99,14 @@ struct CcPullOp {
 };
 
 __device__ __forceinline__ DevCfg select_cc(const Features &f, const gsw_config &force) {
-    DevCfg c = select_traversal(f, force);
+    // Direction (P1) for min-label propagation: unlike BFS there is no "inactive" set that pull
+    // could skip -- a CC pull iteration reduces over every non-isolated row (all 2M entries) while
+    // push touches only the Ea out-edges of the changed vertices.  Measured on C3 (B200): pull
+    // 730 us per iteration, push ~25 us per million active edges, so the split is pull <=> Ea > 2M/4
+    // (the BFS rule's Ea*16 > Eia flipped C3's third iteration between 140 us and 730 us).
+    gsw_config fc = force;
+    if (fc.direction == GSW_AUTO) fc.direction = ((float)f.Ea * 4.f > 2.f * f.M) ? GSW_PULL : GSW_PUSH;
+    DevCfg c = select_traversal(f, fc);
     // the pull workload is every non-isolated vertex: reduce with the owner mappings
     if (c.dir == GSW_PULL && force.load_balance == GSW_AUTO) c.lb = GSW_LB_TWC;
     return c;
