@@ -42,6 +42,7 @@ def _load():
         lib.orc_sssp.argtypes = [i64, P, P, P, i32, P]
         lib.orc_cc.argtypes = [i64, P, P, P]
         lib.orc_pr.argtypes = [i64, P, P, P, dbl, i32, P]
+        lib.orc_dpr.argtypes = [i64, P, P, P, dbl, dbl, i32, P, P]
         lib.orc_bc.argtypes = [i64, P, P, P, i32, P]
         lib.orc_attrs.argtypes = [i64, P, P]
         lib.orc_ratios.argtypes = [i64, i64, i64, i64, i64, i64, P]
@@ -116,6 +117,18 @@ def pr(g, damping: float = 0.85, iters: int = 20, csc=None) -> np.ndarray:
     out = np.empty(g.n, np.float64)
     _check(_load().orc_pr(g.n, _p(off), _p(coff), _p(ccol), damping, iters, _p(out)), "pr")
     return out
+
+
+def dpr(g, damping: float = 0.85, eps: float = 1e-6, max_iters: int = 100000, csc=None):
+    """fp64 Delta-PageRank (oracle.c orc_dpr, DESIGN R15).  eps is the ABSOLUTE residual threshold.
+
+    Returns (rank, iterations)."""
+    off, col = _arrs(g)
+    coff, ccol = (off, col) if csc is None else _arrs(csc)
+    out = np.empty(g.n, np.float64)
+    it = np.zeros(1, np.int32)
+    _check(_load().orc_dpr(g.n, _p(off), _p(coff), _p(ccol), damping, eps, max_iters, _p(out), _p(it)), "dpr")
+    return out, int(it[0])
 
 
 def bc(g, sources) -> np.ndarray:

@@ -14,6 +14,7 @@
  *   orc_sssp         binary-heap Dijkstra (lazy deletion)      P:264-265 ([42]); footnote 2 P:411-413
  *   orc_cc           union-find, labels = min vertex id        P:263-264 ([53]); north_star
  *   orc_pr           fp64 power iteration, dangling mass       P:264 ([11]); SURVEY Q9
+ *   orc_dpr          Delta-PageRank, fp64, threshold eps       P:386-388 ([19]); Fig. 3; DESIGN R15
  *   orc_bc           Brandes, sigma u64, delta fp64            P:265-266 ([47],[10] P:1584-1585)
  *   orc_attrs        dataset attributes N,M,dbar,sd,rd,GI,Her  Table 1; [29]
  *   orc_ratios       Vap,Eap,Viap,Eiap,cd from counts          Table 1; record R P:948-951
@@ -204,6 +205,52 @@ int orc_pr(int64_t n, const int64_t *csr_off, const int64_t *csc_off, const int3
         memcpy(pr, nxt, (size_t)n * sizeof(double));
     }
     free(nxt);
+    return ORC_OK;
+}
+
+/* ---------------------------------------------------------------- Delta-PageRank (fp64) */
+/*
+ * Delta-PageRank ([19]; Fig. 3 "Iteration No. of Delta-PR"), reading R15.
+ * Each vertex holds a rank r and an unpropagated residual delta.  With M(w,v) = 1/deg_out(v) for
+ * every edge v->w (no dangling teleport), the fixed point is x = (1-d)/N 1 + d M x, and
+ *   delta_0(v) = (1-d)/N,  r_0 = 0;   iteration t:
+ *     A_t = { v : delta_t(v) > eps }                                     (Filter: active set)
+ *     r(v) += delta_t(v)                                 for v in A_t
+ *     delta_{t+1}(w) = [w not in A_t] delta_t(w) + sum_{v in A_t, v->w} d delta_t(v)/deg_out(v)
+ *                                                                         (Expand)
+ *   stop when A_t is empty or after max_iters iterations.
+ * Invariant: x = r + (I - dM)^{-1} delta, so 0 <= x - r and ||x - r||_1 <= ||delta||_1/(1-d).
+ * eps < 0 makes every vertex active every iteration: r is then the Neumann partial sum
+ * sum_{k<T} (dM)^k (1-d)/N 1.  Sums in ascending in-edge order (csc_off/csc_col).
+ * iters_out: iterations executed (the last, empty A_t is not counted).
+ */
+int orc_dpr(int64_t n, const int64_t *csr_off, const int64_t *csc_off, const int32_t *csc_col,
+            double d, double eps, int32_t max_iters, double *r, int32_t *iters_out) {
+    if (n <= 0 || max_iters < 0) return ORC_EINVAL;
+    double *delta = (double *)malloc((size_t)n * sizeof(double));
+    double *nxt = (double *)malloc((size_t)n * sizeof(double));
+    char *act = (char *)malloc((size_t)n);
+    if (!delta || !nxt || !act) { free(delta); free(nxt); free(act); return ORC_ENOMEM; }
+    for (int64_t v = 0; v < n; ++v) { r[v] = 0.0; delta[v] = (1.0 - d) / (double)n; }
+    int32_t t = 0;
+    for (; t < max_iters; ++t) {
+        int64_t na = 0;
+        for (int64_t v = 0; v < n; ++v) { act[v] = delta[v] > eps; na += act[v]; }
+        if (na == 0) break;
+        for (int64_t v = 0; v < n; ++v)
+            if (act[v]) r[v] += delta[v];
+        for (int64_t w = 0; w < n; ++w) {
+            double s = 0.0;
+            for (int64_t e = csc_off[w]; e < csc_off[w + 1]; ++e) {
+                int32_t v = csc_col[e];
+                if (act[v]) s += d * delta[v] / (double)(csr_off[v + 1] - csr_off[v]);
+            }
+            nxt[w] = (act[w] ? 0.0 : delta[w]) + s;
+        }
+        memcpy(delta, nxt, (size_t)n * sizeof(double));
+    }
+    if (iters_out) *iters_out = t;
+    free(delta); free(nxt); free(act);
     return ORC_OK;
 }
 

@@ -70,6 +70,21 @@ def pagerank_dense(g, d=0.85, iters=20):
     return x
 
 
+def dpr_fixed_point(g, d=0.85):
+    """Exact fixed point of Delta-PageRank's linear system (DESIGN R15), by a dense solve:
+    (I - d A^T Dinv) x = (1-d)/N 1, dangling columns zero (no teleport of their mass)."""
+    n = g.n
+    A = np.zeros((n, n))
+    for u, v, _ in edge_list(g):
+        A[u, v] += 1.0
+    deg = A.sum(1)
+    M = np.zeros((n, n))
+    for u in range(n):
+        if deg[u] > 0:
+            M[:, u] = A[u] / deg[u]
+    return np.linalg.solve(np.eye(n) - d * M, np.full(n, (1 - d) / n))
+
+
 def path_counts(g):
     """dist[s,t] (hops) and sigma[s,t] (# shortest paths, counting parallel edges) for all pairs
     via dynamic programming over hop length."""

@@ -232,6 +232,75 @@ def test_pr_regular_graphs_uniform_and_mass():
         assert np.abs(xs[t + 1] - xs[t]).sum() <= d ** t * base * (1 + 1e-9)
 
 
+# ------------------------------------------------------------------ Delta-PR
+@pytest.mark.parametrize("name", sorted(tiny_graphs()))
+def test_dpr_tiny_vs_dense_solve(tiny, name):
+    g = tiny[name]
+    x = brute.dpr_fixed_point(g)
+    # eps < 0: every vertex active every iteration -> Neumann partial sums converge to x
+    r, it = oracle.dpr(g, eps=-1.0, max_iters=400)
+    assert it == 400
+    np.testing.assert_allclose(r, x, rtol=1e-12, atol=0)
+    # thresholded: 0 <= x - r and ||x - r||_1 <= ||delta_final||_1/(1-d) <= N eps/(1-d)
+    for eps in (1e-3 / g.n, 1e-6 / g.n):
+        r, _ = oracle.dpr(g, eps=eps)
+        assert np.all(x - r >= -1e-15)
+        assert (x - r).sum() <= g.n * eps / 0.15 * (1 + 1e-9)
+
+
+@pytest.mark.parametrize("seed,n,p", RNG_CASES)
+def test_dpr_random_vs_dense_solve(seed, n, p):
+    g = brute.random_graph(np.random.default_rng(700 + seed), n, p)
+    x = brute.dpr_fixed_point(g)
+    eps = 1e-7 / g.n
+    r, it = oracle.dpr(g, eps=eps)
+    assert it > 0
+    assert np.all(x - r >= -1e-15) and (x - r).sum() <= g.n * eps / 0.15 * (1 + 1e-9)
+    # one iteration from delta_0: active vertices gain (1-d)/N, the rest keep 0
+    r1, it1 = oracle.dpr(g, eps=eps, max_iters=1)
+    assert it1 == 1 and np.allclose(r1, 0.15 / g.n, rtol=1e-15)
+
+
+def test_dpr_directed_vs_dense_solve():
+    rng = np.random.default_rng(11)
+    n = 9
+    edges = [(u, v) for u in range(n) for v in range(n) if u != v and rng.random() < 0.25]
+    g = gen.from_edges(n, edges, symmetric=False)
+    csc = gen.from_edges(n, [(v, u) for u, v in edges], symmetric=False)
+    r, _ = oracle.dpr(g, eps=-1.0, max_iters=400, csc=csc)
+    np.testing.assert_allclose(r, brute.dpr_fixed_point(g), rtol=1e-12)
+
+
+def test_dpr_regular_closed_form():
+    # k-regular graph: every delta_t = (1-d) d^t / N, all active together, so after the T
+    # iterations with delta_t > eps, r = (1-d^T)/N exactly (geometric series), x = 1/N
+    d = 0.85
+    for g in (gen.from_edges(10, [(i, (i + 1) % 10) for i in range(10)]),
+              gen.from_edges(6, [(i, j) for i in range(6) for j in range(i + 1, 6)])):
+        for tol in (1e-2, 1e-5):
+            eps = tol * (1 - d) / g.n
+            T = next(t for t in range(10 ** 4) if not (1 - d) * d ** t / g.n > eps)
+            r, it = oracle.dpr(g, d, eps)
+            assert it == T
+            np.testing.assert_allclose(r, (1 - d ** T) / g.n, rtol=1e-12)
+    # isolated vertex: active once with (1-d)/N, never receives mass
+    r, it = oracle.dpr(gen.from_edges(3, [(0, 1)]), d, 1e-9)
+    assert abs(r[2] - (1 - d) / 3) < 1e-17
+
+
+def test_dpr_rmat_mass_and_bound():
+    g = gen.rmat(12)
+    d, eps = 0.85, 1e-6 / g.n
+    r, it = oracle.dpr(g, d, eps)
+    x, _ = oracle.dpr(g, d, -1.0, max_iters=260)       # d^260 < 1e-18
+    assert np.all(x - r >= -1e-15) and (x - r).sum() <= g.n * eps / (1 - d)
+    # mass: M is column-stochastic on non-isolated vertices (they total (N-iso)/N); an isolated
+    # vertex keeps its (1-d)/N (no dangling teleport, R15)
+    iso = int((np.diff(np.asarray(g.off)) == 0).sum())
+    assert iso > 0
+    assert abs(x.sum() - ((g.n - iso) + iso * (1 - d)) / g.n) < 1e-12
+
+
 # ------------------------------------------------------------------ BC (c5)
 @pytest.mark.parametrize("name", sorted(tiny_graphs()))
 def test_bc_tiny_vs_pair_enumeration(tiny, name):
