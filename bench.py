@@ -160,7 +160,7 @@ def cpu_baseline_sample(g, roots, budget_s=12.0):
 
 def run_extras(gsw, dev, G3, g3, peak):
     """The other BASELINE.json configs (device time of one autotuned call, best of 3, L2 flushed
-    before each): C3 CC and PageRank (20 iterations, d = 0.85), C2 SSSP, C4 BC (16 sources)."""
+    before each): C3 CC, PageRank (20 iterations, d = 0.85) and Delta-PR (tol 1e-6), C2 SSSP, C4 BC (16 sources)."""
     import torch
     import gen
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
@@ -185,6 +185,9 @@ def run_extras(gsw, dev, G3, g3, peak):
     out["C3_cc"] = rec(g3.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
     st = best(lambda: G3.pr(0.85, 20))
     out["C3_pr"] = rec(20 / (st["gpu_ms"] * 1e-3), "PR iters/s", st)
+    # Delta-PR (DESIGN R16): tol = 1e-6 in L1; GTEPS over the edges its Expand read
+    st = best(lambda: G3.dpr(0.85, 1e-6))
+    out["C3_dpr"] = rec(st["edges_touched"] / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS (edges read)", st)
     g2 = gen.config_graph("C2")
     G2 = gsw.Graph(g2.off, g2.col, g2.w, device=dev)
     st = best(lambda: G2.sssp(0))

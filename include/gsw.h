@@ -158,6 +158,23 @@ gsw_status gsw_cc(gsw_graph g, int32_t *label, gsw_run_stats *stats);
  * rank: n doubles, host or device.                                                            */
 gsw_status gsw_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *stats);
 
+/* Delta-PageRank (P:386-388 [19]; Fig. 3; reading R16).  Residual
+ * propagation with an active set: delta_0 = (1-d)/N, r_0 = 0; each iteration the vertices with
+ * delta(v) > eps = tol*(1-d)/N add delta(v) to r(v) and push d*delta(v)/deg_out(v) to their
+ * out-neighbours' residuals; the run ends when no vertex is active (or after max_iters).  The
+ * fixed point x solves x = (1-d)/N + d * sum_{u->v} x(u)/deg_out(u) (no dangling teleport: a
+ * vertex without out-edges keeps its mass), and the result satisfies 0 <= x - rank and
+ * ||x - rank||_1 <= tol.  Per iteration the selector picks push (queue of active vertices, fp64
+ * atomics) or pull (in-edge reduction) from the active-edge count;
+ * gsw_force_config's direction pins it, its other fields are ignored.
+ *   tol: >= 0, finite (0 = run until residuals underflow or max_iters).
+ *   max_iters: 1 .. 2^20.   rank: n doubles, host or device.
+ * stats->iterations counts non-empty iterations; records carry Va/Ea and the direction run.
+ * Errors: GSW_EINVAL (bad arguments), GSW_EUNSUPPORTED (distributed handle, forced direction
+ * other than push/pull).                                                                      */
+gsw_status gsw_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, double *rank,
+                   gsw_run_stats *stats);
+
 /* Betweenness centrality (Brandes): bc[v] = sum_{s in sources, s != v} delta_s(v),
  * unnormalised.  sources: nsrc int32 on the HOST.  bc: n doubles, host or device.              */
 gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc,

@@ -184,6 +184,15 @@ class Graph:
         check(_lib.load().gsw_pr(self._h, float(damping), int(iters), out.data_ptr(), ctypes.byref(st)), "gsw_pr")
         return out, _stats_dict(st, recs)
 
+    def dpr(self, damping: float = 0.85, tol: float = 1e-6, max_iters: int = 10000, out=None, records: int = 0):
+        """Delta-PageRank (gsw_dpr): ||fixed point - rank||_1 <= tol."""
+        import torch
+        out = self._out(out, torch.float64)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_dpr(self._h, float(damping), float(tol), int(max_iters), out.data_ptr(),
+                                  ctypes.byref(st)), "gsw_dpr")
+        return out, _stats_dict(st, recs)
+
     def bc(self, sources: Sequence[int], out=None, records: int = 0):
         import torch
         out = self._out(out, torch.float64)

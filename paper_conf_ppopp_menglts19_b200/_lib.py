@@ -70,6 +70,7 @@ SIGNATURES = {
     "gsw_sssp": (ctypes.c_int, [_P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_cc": (ctypes.c_int, [_P, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_pr": (ctypes.c_int, [_P, ctypes.c_double, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
+    "gsw_dpr": (ctypes.c_int, [_P, ctypes.c_double, ctypes.c_double, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_bc": (ctypes.c_int, [_P, _P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_dist_slice": (ctypes.c_int64, [ctypes.c_int64, ctypes.c_int32]),
     "gsw_dist_unique_id": (ctypes.c_int, [_P]),

@@ -209,6 +209,12 @@ gsw_status gsw_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_
     return run_pr(g, damping, iters, rank, stats);
 }
 
+gsw_status gsw_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, double *rank, gsw_run_stats *stats) {
+    if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (gsw_status s = no_dist(g, "gsw_dpr")) return s;
+    return run_dpr(g, damping, tol, max_iters, rank, stats);
+}
+
 gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
     if (gsw_status s = no_dist(g, "gsw_bc")) return s;

@@ -1,0 +1,394 @@
+// dpr.cu -- Delta-PageRank ([19]; Fig. 3 "Iteration No. of Delta-PR"), the
+// SURVEY F2 row.  Unlike the power iteration of pr.cu, only vertices whose unpropagated residual
+// exceeds eps are active, so the active set shrinks over the run and direction switching matters
+// ("the push mode outperforms the pull mode when the active vertices decrease").
+// Reading R16, identical to oracle.c orc_dpr:
+//   delta_0 = (1-d)/N, r_0 = 0;   A_t = { v : delta_t(v) > eps },  r(v) += delta_t(v) on A_t,
+//   delta_{t+1}(w) = [w not in A_t] delta_t(w) + sum_{v in A_t, v->w} d delta_t(v)/deg_out(v).
+// eps = tol (1-d)/N bounds the result: 0 <= x - r and ||x - r||_1 <= tol (x = fixed point).
+//
+// One iteration = three stream-ordered kernels, no host round trip:
+//   Filter  k_dpr_filter  one pass over N: delta += acc, acc = 0, activation, rank update, the
+//                         contribution c(v) = d delta/deg (0 when inactive), block-aggregated
+//                         enqueue of A_t, Va/Ea of A_t (Table 1 features) -> cnt[t]
+//   Expand  k_dpr_push    fp64 atomicAdd of c(u) into acc of u's targets, for queued u
+//           k_dpr_pull    acc(w) = sum of c over in-neighbours (atomics only for heavy rows)
+//           both in three edge-balanced tiers: 8-lane groups for short rows, a warp for mid
+//           rows, 1024-edge warp chunks of heavy rows (table built at run start)
+// The selector (pull iff Ea > nnz - Ea, "the pull mode is preferable ... when the number of the
+// active edges is greater than that of inactive edges") is evaluated on the device by
+// both expand kernels from cnt[t]; the one not chosen returns at once.  The host only polls the
+// active count every kBatch iterations; kernels after the empty iteration are no-ops.
+#include <algorithm>
+#include <vector>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace gsw {
+
+namespace {
+
+constexpr int kDprBlock = 256;
+constexpr int kBatch = 4;          // iterations enqueued between two host polls
+constexpr int kFilterChunk = 4;    // vertices per thread per block round of the filter
+constexpr uint32_t kChunk = 1024;  // heavy-row chunk (edges per warp task)
+constexpr uint32_t kSmall = 48;    // rows up to this many edges go to an 8-lane group
+struct Chunk;
+
+struct DprCnt {                    // per-iteration record, zeroed at run start
+    unsigned long long va, ea;
+    int dir, pad0;
+    unsigned long long pad1;
+};
+
+struct DprArgs {
+    int n;
+    uint32_t nnz;
+    const uint32_t *off;       // out-edges (push, deg_out)
+    const int32_t *col;
+    const uint32_t *in_off;    // in-edges (pull)
+    const int32_t *in_col;
+    double d, eps;
+    double *r, *delta, *acc, *c;
+    int32_t *q;
+    unsigned *qlen;            // per iteration (max_iters entries)
+    DprCnt *cnt;
+    int force_dir;
+    const Chunk *chunk_out, *chunk_in;   // heavy-row chunk tables (push: out-rows, pull: in-rows)
+    unsigned nchunk_out, nchunk_in;
+};
+
+__global__ void k_dpr_init(DprArgs a) {
+    const double base = (1.0 - a.d) / (double)a.n;
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < a.n; v += (long long)gridDim.x * blockDim.x) {
+        a.r[v] = 0.0;
+        a.delta[v] = base;
+        a.acc[v] = 0.0;
+    }
+}
+
+__device__ __forceinline__ bool dpr_done(const DprArgs &a, int t) { return t > 0 && a.cnt[t - 1].va == 0; }
+
+__global__ void __launch_bounds__(kDprBlock) k_dpr_filter(DprArgs a, int t) {
+    if (dpr_done(a, t)) return;
+    constexpr int W = kDprBlock / 32;
+    __shared__ unsigned s_off[kFilterChunk][W];
+    __shared__ unsigned s_base;
+    __shared__ unsigned long long s_ea[W];
+    __shared__ unsigned s_va[W];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    unsigned long long ea = 0;
+    unsigned va = 0;
+    const long long chunk = (long long)kDprBlock * kFilterChunk;
+    for (long long c0 = blockIdx.x * chunk; c0 < a.n; c0 += gridDim.x * chunk) {
+        unsigned m[kFilterChunk];
+#pragma unroll
+        for (int k = 0; k < kFilterChunk; ++k) {
+            const long long v = c0 + k * kDprBlock + threadIdx.x;
+            bool act = false;
+            if (v < a.n) {
+                const double dl = a.delta[v] + a.acc[v];
+                a.acc[v] = 0.0;
+                double cv = 0.0;
+                if (dl > a.eps) {
+                    act = true;
+                    a.r[v] += dl;
+                    a.delta[v] = 0.0;
+                    const uint32_t deg = __ldg(a.off + v + 1) - __ldg(a.off + v);
+                    if (deg) cv = a.d * dl / (double)deg;
+                    ea += deg;
+                    ++va;
+                } else {
+                    a.delta[v] = dl;
+                }
+                a.c[v] = cv;
+            }
+            m[k] = __ballot_sync(0xffffffffu, act);
+            if (lane == 0) s_off[k][w] = __popc(m[k]);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {   // exclusive scan over (k, w) and one queue reservation per round
+            unsigned s = 0;
+            for (int k = 0; k < kFilterChunk; ++k)
+                for (int j = 0; j < W; ++j) { unsigned x = s_off[k][j]; s_off[k][j] = s; s += x; }
+            s_base = s ? atomicAdd(a.qlen + t, s) : 0u;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int k = 0; k < kFilterChunk; ++k)
+            if (m[k] >> lane & 1u)
+                a.q[s_base + s_off[k][w] + __popc(m[k] & lanemask_lt())] = (int32_t)(c0 + k * kDprBlock + threadIdx.x);
+        __syncthreads();
+    }
+    for (int o = 16; o; o >>= 1) {
+        ea += __shfl_xor_sync(0xffffffffu, ea, o);
+        va += __shfl_xor_sync(0xffffffffu, va, o);
+    }
+    if (lane == 0) { s_ea[w] = ea; s_va[w] = va; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long E = 0, V = 0;
+        for (int j = 0; j < W; ++j) { E += s_ea[j]; V += s_va[j]; }
+        if (V) { atomicAdd(&a.cnt[t].va, V); atomicAdd(&a.cnt[t].ea, E); }
+    }
+}
+
+// 1 = push, 2 = pull (GSW_PUSH / GSW_PULL)
+__device__ __forceinline__ int dpr_dir(const DprArgs &a, const DprCnt &c) {
+    if (a.force_dir) return a.force_dir;
+    return c.ea > (unsigned long long)a.nnz - c.ea ? GSW_PULL : GSW_PUSH;
+}
+
+// Edge-balanced tiers shared by push and pull (Delta-PR):
+//   heavy rows (deg > kChunk): cut into kChunk-edge chunks at run start (host-built table), one
+//     warp per chunk, partial results by fp64 atomics -- a 163K-edge R-MAT hub no longer runs on
+//     one warp for milliseconds;
+//   mid rows (kSmall < deg <= kChunk): one warp, 4 loads in flight per lane;
+//   short rows (deg <= kSmall): an 8-lane group per row, 4 rows per warp.
+struct Chunk {
+    int row;
+    uint32_t beg, end;
+};
+
+// push a mid row u (whole warp): acc[v] += cu for every out-edge
+__device__ __forceinline__ void push_range(const DprArgs &a, uint32_t j, uint32_t e, double cu, int stride) {
+    for (; j + 3 * stride < e; j += 4 * stride) {
+        const int v0 = __ldg(a.col + j), v1 = __ldg(a.col + j + stride), v2 = __ldg(a.col + j + 2 * stride),
+                  v3 = __ldg(a.col + j + 3 * stride);
+        atomicAdd(a.acc + v0, cu); atomicAdd(a.acc + v1, cu); atomicAdd(a.acc + v2, cu); atomicAdd(a.acc + v3, cu);
+    }
+    for (; j < e; j += stride) atomicAdd(a.acc + __ldg(a.col + j), cu);
+}
+
+__device__ __forceinline__ double pull_range(const DprArgs &a, uint32_t j, uint32_t e, int stride) {
+    double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+    for (; j + 3 * stride < e; j += 4 * stride) {
+        const int u0 = __ldg(a.in_col + j), u1 = __ldg(a.in_col + j + stride), u2 = __ldg(a.in_col + j + 2 * stride),
+                  u3 = __ldg(a.in_col + j + 3 * stride);
+        s0 += a.c[u0]; s1 += a.c[u1]; s2 += a.c[u2]; s3 += a.c[u3];
+    }
+    for (; j < e; j += stride) s0 += a.c[__ldg(a.in_col + j)];
+    return (s0 + s1) + (s2 + s3);
+}
+
+__global__ void __launch_bounds__(kDprBlock) k_dpr_push(DprArgs a, int t) {
+    const DprCnt cn = a.cnt[t];
+    if (cn.va == 0 || dpr_dir(a, cn) != GSW_PUSH) return;
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.cnt[t].dir = GSW_PUSH;
+    const unsigned qn = a.qlen[t];
+    const int lane = threadIdx.x & 31, sub = lane >> 3, sl = lane & 7;
+    const unsigned gw = blockIdx.x * (kDprBlock / 32) + (threadIdx.x >> 5);
+    const unsigned nw = gridDim.x * (kDprBlock / 32);
+    // heavy chunks (inactive rows have c = 0 and return at once)
+    for (unsigned k = gw; k < a.nchunk_out; k += nw) {
+        const Chunk ch = a.chunk_out[k];
+        const double cu = a.c[ch.row];
+        if (cu != 0.0) push_range(a, ch.beg + lane, ch.end, cu, 32);
+    }
+    // queued vertices, 4 per warp
+    for (unsigned i0 = gw * 4; i0 < qn; i0 += nw * 4) {
+        const unsigned i = i0 + sub;
+        int u = -1;
+        uint32_t b = 0, e = 0;
+        double cu = 0.0;
+        if (i < qn) {
+            u = a.q[i];
+            cu = a.c[u];
+            b = __ldg(a.off + u); e = __ldg(a.off + u + 1);
+        }
+        const uint32_t deg = e - b;
+        if (cu != 0.0 && deg <= kSmall) push_range(a, b + sl, e, cu, 8);
+        unsigned mid = __ballot_sync(0xffffffffu, sl == 0 && cu != 0.0 && deg > kSmall && deg <= kChunk);
+        while (mid) {
+            const int k = __ffs(mid) - 1;
+            mid &= mid - 1;
+            const uint32_t bb = __shfl_sync(0xffffffffu, b, k), ee = __shfl_sync(0xffffffffu, e, k);
+            const double cc = __shfl_sync(0xffffffffu, cu, k);
+            push_range(a, bb + lane, ee, cc, 32);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kDprBlock) k_dpr_pull(DprArgs a, int t) {
+    const DprCnt cn = a.cnt[t];
+    if (cn.va == 0 || dpr_dir(a, cn) != GSW_PULL) return;
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.cnt[t].dir = GSW_PULL;
+    const int lane = threadIdx.x & 31, sub = lane >> 3, sl = lane & 7;
+    const unsigned gw = blockIdx.x * (kDprBlock / 32) + (threadIdx.x >> 5);
+    const unsigned nw = gridDim.x * (kDprBlock / 32);
+    // heavy chunks: partial sums into acc (zeroed by the filter)
+    for (unsigned k = gw; k < a.nchunk_in; k += nw) {
+        const Chunk ch = a.chunk_in[k];
+        double s = pull_range(a, ch.beg + lane, ch.end, 32);
+        for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+        if (lane == 0 && s != 0.0) atomicAdd(a.acc + ch.row, s);
+    }
+    for (unsigned v0 = gw * 4; v0 < (unsigned)a.n; v0 += nw * 4) {
+        const unsigned v = v0 + sub;
+        uint32_t b = 0, e = 0;
+        if (v < (unsigned)a.n) { b = __ldg(a.in_off + v); e = __ldg(a.in_off + v + 1); }
+        const uint32_t deg = e - b;
+        double s = deg <= kSmall ? pull_range(a, b + sl, e, 8) : 0.0;
+        s += __shfl_xor_sync(0xffffffffu, s, 4);
+        s += __shfl_xor_sync(0xffffffffu, s, 2);
+        s += __shfl_xor_sync(0xffffffffu, s, 1);
+        if (sl == 0 && v < (unsigned)a.n && deg <= kSmall) a.acc[v] = s;
+        unsigned mid = __ballot_sync(0xffffffffu, sl == 0 && deg > kSmall && deg <= kChunk);
+        while (mid) {
+            const int k = __ffs(mid) - 1;
+            mid &= mid - 1;
+            const uint32_t bb = __shfl_sync(0xffffffffu, b, k), ee = __shfl_sync(0xffffffffu, e, k);
+            double m = pull_range(a, bb + lane, ee, 32);
+            for (int o = 16; o; o >>= 1) m += __shfl_xor_sync(0xffffffffu, m, o);
+            if (lane == 0) a.acc[v0 + (k >> 3)] = m;
+        }
+    }
+}
+
+// heavy-row list (run start): rows with more than kChunk edges, (row, begin, end) appended
+__global__ void k_dpr_heavy(const uint32_t *off, int n, Chunk *list, unsigned *cnt, unsigned cap) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
+        const uint32_t b = off[v], e = off[v + 1];
+        if (e - b > kChunk) {
+            const unsigned i = atomicAdd(cnt, 1u);
+            if (i < cap) list[i] = Chunk{(int)v, b, e};
+        }
+    }
+}
+
+__global__ void k_dpr_out(const double *r, const uint32_t *perm, int n, double *out) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
+        out[perm ? perm[v] : v] = r[v];
+}
+
+}  // namespace
+
+gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, double *rank, gsw_run_stats *st) {
+    const int n = g->g.n;
+    if (!rank) { set_error("gsw_dpr: rank is NULL"); return GSW_EINVAL; }
+    if (max_iters < 1 || max_iters > (1 << 20)) { set_error("gsw_dpr: max_iters must be in [1, 2^20]"); return GSW_EINVAL; }
+    if (!(damping >= 0.0 && damping < 1.0)) { set_error("gsw_dpr: damping must be in [0,1)"); return GSW_EINVAL; }
+    if (!(tol >= 0.0 && tol < 1e300)) { set_error("gsw_dpr: tol must be finite and >= 0"); return GSW_EINVAL; }
+    const int fdir = g->forced.direction;
+    if (fdir != GSW_AUTO && fdir != GSW_PUSH && fdir != GSW_PULL) { set_error("gsw_dpr: bad forced direction"); return GSW_EUNSUPPORTED; }
+    Workspace ws{g->scratch, g->scratch_bytes, 0};
+    const bool dev_out = is_device_ptr(rank) == 1;
+    DprArgs a{};
+    a.n = n;
+    a.nnz = g->g.nnz;
+    a.off = g->g.off; a.col = g->g.col;
+    a.in_off = g->g.in_off; a.in_col = g->g.in_col;
+    a.d = damping;
+    a.eps = tol * (1.0 - damping) / (double)n;
+    a.force_dir = fdir;
+    a.r = (double *)ws.take((size_t)n * 8);
+    a.delta = (double *)ws.take((size_t)n * 8);
+    a.acc = (double *)ws.take((size_t)n * 8);
+    a.c = (double *)ws.take((size_t)n * 8);
+    a.q = (int32_t *)ws.take((size_t)n * 4);
+    a.qlen = (unsigned *)ws.take((size_t)max_iters * 4);
+    a.cnt = (DprCnt *)ws.take((size_t)max_iters * sizeof(DprCnt));
+    double *out = dev_out ? rank : (double *)ws.take((size_t)n * 8);
+    if (!a.r || !a.delta || !a.acc || !a.c || !a.q || !a.qlen || !a.cnt || !out) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
+    cudaStream_t s = g->stream;
+    const int grid = g->sms * 8;
+    GSW_CUDA(cudaEventRecord(g->ev0, s));
+    // heavy-row chunk tables (once per run; one host round trip each)
+    const size_t hcap = (size_t)a.nnz / kChunk + 1, ccap = 2 * hcap + 1;
+    unsigned *hcnt = (unsigned *)ws.take(256);
+    Chunk *hlist = (Chunk *)ws.take(hcap * sizeof(Chunk));
+    if (!hcnt || !hlist) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
+    auto build = [&](const uint32_t *off, const Chunk **tab, unsigned *nt) -> gsw_status {
+        GSW_CUDA(cudaMemsetAsync(hcnt, 0, 4, s));
+        k_dpr_heavy<<<grid, kDprBlock, 0, s>>>(off, n, hlist, hcnt, (unsigned)hcap);
+        GSW_CUDA(cudaGetLastError());
+        unsigned nh = 0;
+        GSW_CUDA(cudaMemcpyAsync(&nh, hcnt, 4, cudaMemcpyDeviceToHost, s));
+        GSW_CUDA(cudaStreamSynchronize(s));
+        nh = std::min<unsigned>(nh, (unsigned)hcap);
+        std::vector<Chunk> rows(nh), ch;
+        if (nh) GSW_CUDA(cudaMemcpy(rows.data(), hlist, nh * sizeof(Chunk), cudaMemcpyDeviceToHost));
+        for (const Chunk &r : rows)
+            for (uint32_t b = r.beg; b < r.end; b += kChunk) ch.push_back(Chunk{r.row, b, std::min(r.end, b + kChunk)});
+        Chunk *t = (Chunk *)ws.take(std::max<size_t>(1, std::min(ch.size(), ccap)) * sizeof(Chunk));
+        if (!t) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
+        if (!ch.empty()) GSW_CUDA(cudaMemcpyAsync(t, ch.data(), ch.size() * sizeof(Chunk), cudaMemcpyHostToDevice, s));
+        GSW_CUDA(cudaStreamSynchronize(s));   // ch is a local vector
+        *tab = t;
+        *nt = (unsigned)ch.size();
+        return GSW_OK;
+    };
+    if (gsw_status e = build(a.off, &a.chunk_out, &a.nchunk_out)) return e;
+    if (a.in_off == a.off && a.in_col == a.col) {
+        a.chunk_in = a.chunk_out;
+        a.nchunk_in = a.nchunk_out;
+    } else if (gsw_status e = build(a.in_off, &a.chunk_in, &a.nchunk_in)) {
+        return e;
+    }
+    GSW_CUDA(cudaMemsetAsync(a.qlen, 0, (size_t)max_iters * 4, s));
+    GSW_CUDA(cudaMemsetAsync(a.cnt, 0, (size_t)max_iters * sizeof(DprCnt), s));
+    k_dpr_init<<<grid, kDprBlock, 0, s>>>(a);
+    GSW_CUDA(cudaGetLastError());
+    int t = 0;
+    bool done = false;
+    while (!done && t < max_iters) {
+        const int t1 = std::min(max_iters, t + kBatch);
+        for (; t < t1; ++t) {
+            k_dpr_filter<<<grid, kDprBlock, 0, s>>>(a, t);
+            k_dpr_push<<<grid, kDprBlock, 0, s>>>(a, t);
+            k_dpr_pull<<<grid, kDprBlock, 0, s>>>(a, t);
+        }
+        GSW_CUDA(cudaGetLastError());
+        unsigned long long va = 0;
+        GSW_CUDA(cudaMemcpyAsync(&va, &a.cnt[t - 1].va, 8, cudaMemcpyDeviceToHost, s));
+        GSW_CUDA(cudaStreamSynchronize(s));
+        done = va == 0;
+    }
+    const int launched = t;
+    k_dpr_out<<<grid, kDprBlock, 0, s>>>(a.r, g->g.perm, n, out);
+    GSW_CUDA(cudaGetLastError());
+    GSW_CUDA(cudaEventRecord(g->ev1, s));
+    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(rank, out, (size_t)n * 8, cudaMemcpyDeviceToHost, s));
+    std::vector<DprCnt> h((size_t)launched);
+    GSW_CUDA(cudaMemcpyAsync(h.data(), a.cnt, sizeof(DprCnt) * (size_t)launched, cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    if (st) {
+        int it = 0;
+        while (it < launched && h[it].va) ++it;
+        float ms = 0.f;
+        GSW_CUDA(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+        long long edges = 0, bytes = 0;
+        const long long N = n, E = a.nnz;
+        for (int i = 0; i < it; ++i) {
+            const long long Va = (long long)h[i].va, Ea = (long long)h[i].ea;
+            const bool pull = h[i].dir == GSW_PULL;
+            const long long ed = pull ? E : Ea;
+            edges += ed;
+            // DESIGN.md section 6, Delta-PR: filter 40 B/vertex (delta, acc r/w; c write) + 20 B
+            // per active vertex (rank r/w, queue); push 8 B/active vertex (offsets) + 4 B column
+            // + 16 B atomic RMW per edge; pull 8 B/row + 8 B acc write + 12 B per in-edge
+            bytes += 40 * N + 20 * Va + (pull ? 16 * N + 12 * E : 8 * Va + 20 * Ea);
+            if (st->records && i < st->max_records) {
+                gsw_iter_record &rec = st->records[i];
+                rec = gsw_iter_record{};
+                rec.iteration = i;
+                rec.direction = h[i].dir;
+                rec.format = GSW_QUEUE;
+                rec.load_balance = GSW_LB_WM;
+                rec.fusion = GSW_STANDALONE;
+                rec.Va = Va; rec.Ea = Ea;
+                rec.Via = N - Va; rec.Eia = E - Ea;
+                rec.edges = ed;
+                rec.ctas = grid;
+            }
+        }
+        st->iterations = it;
+        st->gpu_ms = ms;
+        st->edges_touched = edges;
+        st->bytes_alg = bytes;
+    }
+    return GSW_OK;
+}
+
+}  // namespace gsw

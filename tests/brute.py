@@ -71,7 +71,7 @@ def pagerank_dense(g, d=0.85, iters=20):
 
 
 def dpr_fixed_point(g, d=0.85):
-    """Exact fixed point of Delta-PageRank's linear system (DESIGN R15), by a dense solve:
+    """Exact fixed point of Delta-PageRank's linear system (DESIGN R16), by a dense solve:
     (I - d A^T Dinv) x = (1-d)/N 1, dangling columns zero (no teleport of their mass)."""
     n = g.n
     A = np.zeros((n, n))

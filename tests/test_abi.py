@@ -27,7 +27,7 @@ def lib():
 
 def test_header_declares_north_star_api():
     names = _declared()
-    for must in ["gsw_graph_create", "gsw_bfs", "gsw_sssp", "gsw_cc", "gsw_pr", "gsw_bc", "gsw_force_config"]:
+    for must in ["gsw_graph_create", "gsw_bfs", "gsw_sssp", "gsw_cc", "gsw_pr", "gsw_dpr", "gsw_bc", "gsw_force_config"]:
         assert must in names
 
 

@@ -232,7 +232,7 @@ def test_pr_regular_graphs_uniform_and_mass():
         assert np.abs(xs[t + 1] - xs[t]).sum() <= d ** t * base * (1 + 1e-9)
 
 
-# ------------------------------------------------------------------ Delta-PR (SURVEY F2, R15)
+# ------------------------------------------------------------------ Delta-PR (SURVEY F2, R16)
 @pytest.mark.parametrize("name", sorted(tiny_graphs()))
 def test_dpr_tiny_vs_dense_solve(tiny, name):
     g = tiny[name]
@@ -295,7 +295,7 @@ def test_dpr_rmat_mass_and_bound():
     x, _ = oracle.dpr(g, d, -1.0, max_iters=260)       # d^260 < 1e-18
     assert np.all(x - r >= -1e-15) and (x - r).sum() <= g.n * eps / (1 - d)
     # mass: M is column-stochastic on non-isolated vertices (they total (N-iso)/N); an isolated
-    # vertex keeps its (1-d)/N (no dangling teleport, R15)
+    # vertex keeps its (1-d)/N (no dangling teleport, R16)
     iso = int((np.diff(np.asarray(g.off)) == 0).sum())
     assert iso > 0
     assert abs(x.sum() - ((g.n - iso) + iso * (1 - d)) / g.n) < 1e-12
