@@ -16,4 +16,5 @@ for _ in range(2):
     elif algo == "cc": G.cc()
     elif algo == "sssp": G.sssp(0)
     elif algo == "bc": G.bc(gen.sources(g, 2))
+    elif algo == "dpr": G.dpr(0.85, 1e-6)
 print("done")

@@ -80,7 +80,8 @@ def main():
                         f"step's device work; under ncu its mean duration is {ns / n / 1e3:.1f} us per launch "
                         f"({n} launches: warm-up + timed steps + e2e leg).\n")
     for rep, kernel in [("bfs_c3_full", "bfs_kernel"), ("pr_c3_full", "pr_kernel"), ("sssp_c2_full", "sssp_kernel"),
-                        ("bfs_c2_full", "bfs_kernel_c2")]:
+                        ("bfs_c2_full", "bfs_kernel_c2"), ("dpr_pull_c3_full", "dpr_pull"),
+                        ("dpr_push_c3_full", "dpr_push"), ("dpr_filter_c3_full", "dpr_filter")]:
         path = os.path.join(OUT, rep + ".ncu-rep")
         if not os.path.exists(path):
             continue
