@@ -13,8 +13,9 @@
 //                         enqueue of A_t, Va/Ea of A_t (Table 1 features) -> cnt[t]
 //   Expand  k_dpr_push    fp64 atomicAdd of c(u) into acc of u's targets, for queued u
 //           k_dpr_pull    acc(w) = sum of c over in-neighbours (atomics only for heavy rows)
-//           both in three edge-balanced tiers: 8-lane groups for short rows, a warp for mid
-//           rows, 1024-edge warp chunks of heavy rows (table built at run start)
+//           both in four edge-balanced tiers: a lane per tiny row, 8-lane groups for short
+//           rows, a warp per mid row, 1024-edge warp chunks of heavy rows (table built at
+//           run start)
 // The selector (pull iff Ea > nnz - Ea, "the pull mode is preferable ... when the number of the
 // active edges is greater than that of inactive edges") is evaluated on the device by
 // both expand kernels from cnt[t]; the one not chosen returns at once.  The host only polls the
@@ -33,7 +34,8 @@ constexpr int kDprBlock = 256;
 constexpr int kBatch = 4;          // iterations enqueued between two host polls
 constexpr int kFilterChunk = 4;    // vertices per thread per block round of the filter
 constexpr uint32_t kChunk = 1024;  // heavy-row chunk (edges per warp task)
-constexpr uint32_t kSmall = 48;    // rows up to this many edges go to an 8-lane group
+constexpr uint32_t kSmall = 64;    // rows up to this many edges go to an 8-lane group
+constexpr uint32_t kTiny = 8;      // rows up to this many edges are finished by one lane
 struct Chunk;
 
 struct DprCnt {                    // per-iteration record, zeroed at run start
@@ -83,24 +85,35 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_filter(DprArgs a, int t) {
     const long long chunk = (long long)kDprBlock * kFilterChunk;
     for (long long c0 = blockIdx.x * chunk; c0 < a.n; c0 += gridDim.x * chunk) {
         unsigned m[kFilterChunk];
+        double dl[kFilterChunk];
+        uint32_t deg[kFilterChunk];
+        // all loads of the round first (4 independent vertices in flight per thread)
+#pragma unroll
+        for (int k = 0; k < kFilterChunk; ++k) {
+            const long long v = c0 + k * kDprBlock + threadIdx.x;
+            dl[k] = 0.0;
+            deg[k] = 0;
+            if (v < a.n) {
+                dl[k] = a.delta[v] + a.acc[v];
+                deg[k] = __ldg(a.off + v + 1) - __ldg(a.off + v);
+            }
+        }
 #pragma unroll
         for (int k = 0; k < kFilterChunk; ++k) {
             const long long v = c0 + k * kDprBlock + threadIdx.x;
             bool act = false;
             if (v < a.n) {
-                const double dl = a.delta[v] + a.acc[v];
                 a.acc[v] = 0.0;
                 double cv = 0.0;
-                if (dl > a.eps) {
+                if (dl[k] > a.eps) {
                     act = true;
-                    a.r[v] += dl;
+                    a.r[v] += dl[k];
                     a.delta[v] = 0.0;
-                    const uint32_t deg = __ldg(a.off + v + 1) - __ldg(a.off + v);
-                    if (deg) cv = a.d * dl / (double)deg;
-                    ea += deg;
+                    if (deg[k]) cv = a.d * dl[k] / (double)deg[k];
+                    ea += deg[k];
                     ++va;
                 } else {
-                    a.delta[v] = dl;
+                    a.delta[v] = dl[k];
                 }
                 a.c[v] = cv;
             }
@@ -172,12 +185,76 @@ __device__ __forceinline__ double pull_range(const DprArgs &a, uint32_t j, uint3
     return (s0 + s1) + (s2 + s3);
 }
 
+// Rows of one 32-row warp batch, one row per lane: tiny rows (deg <= kTiny) are finished by
+// their own lane, short rows by 8-lane groups (4 at a time, __fns picks each group's row), mid
+// rows by the whole warp; heavy rows are skipped (chunk tasks).  Op: push or pull body.
+template <class Op>
+__device__ __forceinline__ void row_tiers(const Op &op, bool valid, uint32_t b, uint32_t e) {
+    const int lane = threadIdx.x & 31, sub = lane >> 3, sl = lane & 7;
+    const uint32_t deg = e - b;
+    const bool live = valid && op.live();
+    if (live && deg <= kTiny) op.tiny(b, e);
+    unsigned sm = __ballot_sync(0xffffffffu, live && deg > kTiny && deg <= kSmall);
+    while (sm) {
+        const unsigned k = __fns(sm, 0, sub + 1);
+        const int src = k < 32 ? (int)k : lane;
+        const uint32_t bb = __shfl_sync(0xffffffffu, b, src), ee = __shfl_sync(0xffffffffu, e, src);
+        op.group(src, k < 32, bb, ee, sl);
+        for (int i = 0; i < 4 && sm; ++i) sm &= sm - 1;
+    }
+    unsigned mid = __ballot_sync(0xffffffffu, live && deg > kSmall && deg <= kChunk);
+    while (mid) {
+        const int k = __ffs(mid) - 1;
+        mid &= mid - 1;
+        const uint32_t bb = __shfl_sync(0xffffffffu, b, k), ee = __shfl_sync(0xffffffffu, e, k);
+        op.warp(k, bb, ee, lane);
+    }
+}
+
+struct PushOp {
+    const DprArgs &a;
+    double cu;
+    __device__ bool live() const { return cu != 0.0; }
+    __device__ void tiny(uint32_t b, uint32_t e) const { for (uint32_t j = b; j < e; ++j) atomicAdd(a.acc + __ldg(a.col + j), cu); }
+    __device__ void group(int src, bool on, uint32_t b, uint32_t e, int sl) const {
+        const double c = __shfl_sync(0xffffffffu, cu, src);
+        if (on) push_range(a, b + sl, e, c, 8);
+    }
+    __device__ void warp(int src, uint32_t b, uint32_t e, int lane) const {
+        const double c = __shfl_sync(0xffffffffu, cu, src);
+        push_range(a, b + lane, e, c, 32);
+    }
+};
+
+struct PullOp {
+    const DprArgs &a;
+    unsigned v0;
+    __device__ bool live() const { return true; }
+    __device__ void tiny(uint32_t b, uint32_t e) const {
+        double s = 0.0;
+        for (uint32_t j = b; j < e; ++j) s += a.c[__ldg(a.in_col + j)];
+        a.acc[v0 + (threadIdx.x & 31)] = s;
+    }
+    __device__ void group(int src, bool on, uint32_t b, uint32_t e, int sl) const {
+        double s = on ? pull_range(a, b + sl, e, 8) : 0.0;
+        s += __shfl_xor_sync(0xffffffffu, s, 4);
+        s += __shfl_xor_sync(0xffffffffu, s, 2);
+        s += __shfl_xor_sync(0xffffffffu, s, 1);
+        if (on && sl == 0) a.acc[v0 + src] = s;
+    }
+    __device__ void warp(int src, uint32_t b, uint32_t e, int lane) const {
+        double m = pull_range(a, b + lane, e, 32);
+        for (int o = 16; o; o >>= 1) m += __shfl_xor_sync(0xffffffffu, m, o);
+        if (lane == 0) a.acc[v0 + src] = m;
+    }
+};
+
 __global__ void __launch_bounds__(kDprBlock) k_dpr_push(DprArgs a, int t) {
     const DprCnt cn = a.cnt[t];
     if (cn.va == 0 || dpr_dir(a, cn) != GSW_PUSH) return;
     if (blockIdx.x == 0 && threadIdx.x == 0) a.cnt[t].dir = GSW_PUSH;
     const unsigned qn = a.qlen[t];
-    const int lane = threadIdx.x & 31, sub = lane >> 3, sl = lane & 7;
+    const int lane = threadIdx.x & 31;
     const unsigned gw = blockIdx.x * (kDprBlock / 32) + (threadIdx.x >> 5);
     const unsigned nw = gridDim.x * (kDprBlock / 32);
     // heavy chunks (inactive rows have c = 0 and return at once)
@@ -186,27 +263,17 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_push(DprArgs a, int t) {
         const double cu = a.c[ch.row];
         if (cu != 0.0) push_range(a, ch.beg + lane, ch.end, cu, 32);
     }
-    // queued vertices, 4 per warp
-    for (unsigned i0 = gw * 4; i0 < qn; i0 += nw * 4) {
-        const unsigned i = i0 + sub;
-        int u = -1;
+    // queued vertices, 32 per warp batch
+    for (unsigned i0 = gw * 32; i0 < qn; i0 += nw * 32) {
+        const unsigned i = i0 + lane;
         uint32_t b = 0, e = 0;
         double cu = 0.0;
         if (i < qn) {
-            u = a.q[i];
+            const int u = a.q[i];
             cu = a.c[u];
             b = __ldg(a.off + u); e = __ldg(a.off + u + 1);
         }
-        const uint32_t deg = e - b;
-        if (cu != 0.0 && deg <= kSmall) push_range(a, b + sl, e, cu, 8);
-        unsigned mid = __ballot_sync(0xffffffffu, sl == 0 && cu != 0.0 && deg > kSmall && deg <= kChunk);
-        while (mid) {
-            const int k = __ffs(mid) - 1;
-            mid &= mid - 1;
-            const uint32_t bb = __shfl_sync(0xffffffffu, b, k), ee = __shfl_sync(0xffffffffu, e, k);
-            const double cc = __shfl_sync(0xffffffffu, cu, k);
-            push_range(a, bb + lane, ee, cc, 32);
-        }
+        row_tiers(PushOp{a, cu}, i < qn, b, e);
     }
 }
 
@@ -214,7 +281,7 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_pull(DprArgs a, int t) {
     const DprCnt cn = a.cnt[t];
     if (cn.va == 0 || dpr_dir(a, cn) != GSW_PULL) return;
     if (blockIdx.x == 0 && threadIdx.x == 0) a.cnt[t].dir = GSW_PULL;
-    const int lane = threadIdx.x & 31, sub = lane >> 3, sl = lane & 7;
+    const int lane = threadIdx.x & 31;
     const unsigned gw = blockIdx.x * (kDprBlock / 32) + (threadIdx.x >> 5);
     const unsigned nw = gridDim.x * (kDprBlock / 32);
     // heavy chunks: partial sums into acc (zeroed by the filter)
@@ -224,25 +291,11 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_pull(DprArgs a, int t) {
         for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
         if (lane == 0 && s != 0.0) atomicAdd(a.acc + ch.row, s);
     }
-    for (unsigned v0 = gw * 4; v0 < (unsigned)a.n; v0 += nw * 4) {
-        const unsigned v = v0 + sub;
+    for (unsigned v0 = gw * 32; v0 < (unsigned)a.n; v0 += nw * 32) {
+        const unsigned v = v0 + lane;
         uint32_t b = 0, e = 0;
         if (v < (unsigned)a.n) { b = __ldg(a.in_off + v); e = __ldg(a.in_off + v + 1); }
-        const uint32_t deg = e - b;
-        double s = deg <= kSmall ? pull_range(a, b + sl, e, 8) : 0.0;
-        s += __shfl_xor_sync(0xffffffffu, s, 4);
-        s += __shfl_xor_sync(0xffffffffu, s, 2);
-        s += __shfl_xor_sync(0xffffffffu, s, 1);
-        if (sl == 0 && v < (unsigned)a.n && deg <= kSmall) a.acc[v] = s;
-        unsigned mid = __ballot_sync(0xffffffffu, sl == 0 && deg > kSmall && deg <= kChunk);
-        while (mid) {
-            const int k = __ffs(mid) - 1;
-            mid &= mid - 1;
-            const uint32_t bb = __shfl_sync(0xffffffffu, b, k), ee = __shfl_sync(0xffffffffu, e, k);
-            double m = pull_range(a, bb + lane, ee, 32);
-            for (int o = 16; o; o >>= 1) m += __shfl_xor_sync(0xffffffffu, m, o);
-            if (lane == 0) a.acc[v0 + (k >> 3)] = m;
-        }
+        row_tiers(PullOp{a, v0}, v < (unsigned)a.n, b, e);
     }
 }
 
@@ -260,6 +313,17 @@ __global__ void k_dpr_heavy(const uint32_t *off, int n, Chunk *list, unsigned *c
 __global__ void k_dpr_out(const double *r, const uint32_t *perm, int n, double *out) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x)
         out[perm ? perm[v] : v] = r[v];
+}
+
+// one full wave: SMs x resident blocks of this kernel (a second partial wave of a grid-stride
+// kernel would leave most SMs idle during its tail)
+int wave_grid(const void *k, int sms) {
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, kDprBlock, 0) != cudaSuccess || nb < 1) {
+        cudaGetLastError();
+        nb = 1;
+    }
+    return sms * nb;
 }
 
 }  // namespace
@@ -293,6 +357,9 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
     if (!a.r || !a.delta || !a.acc || !a.c || !a.q || !a.qlen || !a.cnt || !out) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
     cudaStream_t s = g->stream;
     const int grid = g->sms * 8;
+    static const int g_filter = wave_grid((const void *)k_dpr_filter, g->sms);
+    static const int g_push = wave_grid((const void *)k_dpr_push, g->sms);
+    static const int g_pull = wave_grid((const void *)k_dpr_pull, g->sms);
     GSW_CUDA(cudaEventRecord(g->ev0, s));
     // heavy-row chunk tables (once per run; one host round trip each)
     const size_t hcap = (size_t)a.nnz / kChunk + 1, ccap = 2 * hcap + 1;
@@ -335,9 +402,9 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
     while (!done && t < max_iters) {
         const int t1 = std::min(max_iters, t + kBatch);
         for (; t < t1; ++t) {
-            k_dpr_filter<<<grid, kDprBlock, 0, s>>>(a, t);
-            k_dpr_push<<<grid, kDprBlock, 0, s>>>(a, t);
-            k_dpr_pull<<<grid, kDprBlock, 0, s>>>(a, t);
+            k_dpr_filter<<<g_filter, kDprBlock, 0, s>>>(a, t);
+            k_dpr_push<<<g_push, kDprBlock, 0, s>>>(a, t);
+            k_dpr_pull<<<g_pull, kDprBlock, 0, s>>>(a, t);
         }
         GSW_CUDA(cudaGetLastError());
         unsigned long long va = 0;
