@@ -18,8 +18,9 @@
 //           run start)
 // The selector (pull iff Ea > nnz - Ea, "the pull mode is preferable ... when the number of the
 // active edges is greater than that of inactive edges") is evaluated on the device by
-// both expand kernels from cnt[t]; the one not chosen returns at once.  The host only polls the
-// active count every kBatch iterations; kernels after the empty iteration are no-ops.
+// both expand kernels from cnt[t]; the one not chosen returns at once.  The host polls the active
+// count once per batch of iterations, one batch behind the stream; kernels after the empty
+// iteration are no-ops.
 #include <algorithm>
 #include <vector>
 
@@ -31,9 +32,13 @@ namespace gsw {
 namespace {
 
 constexpr int kDprBlock = 256;
-constexpr int kBatch = 4;          // iterations enqueued between two host polls
+constexpr int kBatch = 4;          // iterations enqueued between two host polls (at least)
+constexpr int kBatchMax = 32;      // ... and at most
 constexpr int kFilterChunk = 4;    // vertices per thread per block round of the filter
 constexpr uint32_t kChunk = 1024;  // heavy-row chunk (edges per warp task)
+constexpr uint32_t kHeavy = 128;   // rows above this many edges become chunk tasks: after the
+                                   // degree-ordered relabeling the mid rows sit together, and 32
+                                   // of them serialised on one warp were the tail of small graphs
 constexpr uint32_t kSmall = 64;    // rows up to this many edges go to an 8-lane group
 constexpr uint32_t kTiny = 8;      // rows up to this many edges are finished by one lane
 struct Chunk;
@@ -154,10 +159,10 @@ __device__ __forceinline__ int dpr_dir(const DprArgs &a, const DprCnt &c) {
 }
 
 // Edge-balanced tiers shared by push and pull (Delta-PR):
-//   heavy rows (deg > kChunk): cut into kChunk-edge chunks at run start (host-built table), one
+//   heavy rows (deg > kHeavy): cut into kChunk-edge chunks at run start (host-built table), one
 //     warp per chunk, partial results by fp64 atomics -- a 163K-edge R-MAT hub no longer runs on
 //     one warp for milliseconds;
-//   mid rows (kSmall < deg <= kChunk): one warp, 4 loads in flight per lane;
+//   mid rows (kSmall < deg <= kHeavy): one warp, 4 loads in flight per lane;
 //   short rows (deg <= kSmall): an 8-lane group per row, 4 rows per warp.
 struct Chunk {
     int row;
@@ -202,7 +207,7 @@ __device__ __forceinline__ void row_tiers(const Op &op, bool valid, uint32_t b, 
         op.group(src, k < 32, bb, ee, sl);
         for (int i = 0; i < 4 && sm; ++i) sm &= sm - 1;
     }
-    unsigned mid = __ballot_sync(0xffffffffu, live && deg > kSmall && deg <= kChunk);
+    unsigned mid = __ballot_sync(0xffffffffu, live && deg > kSmall && deg <= kHeavy);
     while (mid) {
         const int k = __ffs(mid) - 1;
         mid &= mid - 1;
@@ -299,11 +304,11 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_pull(DprArgs a, int t) {
     }
 }
 
-// heavy-row list (run start): rows with more than kChunk edges, (row, begin, end) appended
+// heavy-row list (run start): rows with more than kHeavy edges, (row, begin, end) appended
 __global__ void k_dpr_heavy(const uint32_t *off, int n, Chunk *list, unsigned *cnt, unsigned cap) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
         const uint32_t b = off[v], e = off[v + 1];
-        if (e - b > kChunk) {
+        if (e - b > kHeavy) {
             const unsigned i = atomicAdd(cnt, 1u);
             if (i < cap) list[i] = Chunk{(int)v, b, e};
         }
@@ -362,7 +367,7 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
     static const int g_pull = wave_grid((const void *)k_dpr_pull, g->sms);
     GSW_CUDA(cudaEventRecord(g->ev0, s));
     // heavy-row chunk tables (once per run; one host round trip each)
-    const size_t hcap = (size_t)a.nnz / kChunk + 1, ccap = 2 * hcap + 1;
+    const size_t hcap = (size_t)a.nnz / kHeavy + 1, ccap = 2 * hcap + 1;
     unsigned *hcnt = (unsigned *)ws.take(256);
     Chunk *hlist = (Chunk *)ws.take(hcap * sizeof(Chunk));
     if (!hcnt || !hlist) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
@@ -397,21 +402,46 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
     GSW_CUDA(cudaMemsetAsync(a.cnt, 0, (size_t)max_iters * sizeof(DprCnt), s));
     k_dpr_init<<<grid, kDprBlock, 0, s>>>(a);
     GSW_CUDA(cudaGetLastError());
-    int t = 0;
+    // Pipelined termination poll: batch b is enqueued (with an async copy of its last active
+    // count into pinned memory and an event) BEFORE the host waits on batch b-1's event, so the
+    // stream never drains while the host decides.  Batches grow with t (clamp(t/4, 4, 32)), so at
+    // most one batch of no-op kernels runs past the empty iteration.
+    static thread_local unsigned long long *hva = nullptr;   // 2 pinned slots, one per in-flight batch
+    if (!hva) GSW_CUDA(cudaHostAlloc((void **)&hva, 2 * sizeof(unsigned long long), cudaHostAllocDefault));
+    cudaEvent_t evb[2] = {nullptr, nullptr};
+    GSW_CUDA(cudaEventCreateWithFlags(&evb[0], cudaEventDisableTiming));
+    GSW_CUDA(cudaEventCreateWithFlags(&evb[1], cudaEventDisableTiming));
+    auto poll_fail = [&](cudaError_t e, const char *what) {
+        cudaEventDestroy(evb[0]);
+        cudaEventDestroy(evb[1]);
+        return cuda_fail(e, what);
+    };
+    int t = 0, b = 0;
     bool done = false;
-    while (!done && t < max_iters) {
-        const int t1 = std::min(max_iters, t + kBatch);
-        for (; t < t1; ++t) {
-            k_dpr_filter<<<g_filter, kDprBlock, 0, s>>>(a, t);
-            k_dpr_push<<<g_push, kDprBlock, 0, s>>>(a, t);
-            k_dpr_pull<<<g_pull, kDprBlock, 0, s>>>(a, t);
+    while (!done) {
+        {
+            const int t1 = std::min(max_iters, t + std::min(kBatchMax, std::max(kBatch, t / 4)));
+            for (; t < t1; ++t) {
+                k_dpr_filter<<<g_filter, kDprBlock, 0, s>>>(a, t);
+                k_dpr_push<<<g_push, kDprBlock, 0, s>>>(a, t);
+                k_dpr_pull<<<g_pull, kDprBlock, 0, s>>>(a, t);
+            }
+            cudaError_t e = cudaGetLastError();
+            if (e == cudaSuccess) e = cudaMemcpyAsync(&hva[b & 1], &a.cnt[t - 1].va, 8, cudaMemcpyDeviceToHost, s);
+            if (e == cudaSuccess) e = cudaEventRecord(evb[b & 1], s);
+            if (e != cudaSuccess) return poll_fail(e, "gsw_dpr: batch enqueue");
+            ++b;
         }
-        GSW_CUDA(cudaGetLastError());
-        unsigned long long va = 0;
-        GSW_CUDA(cudaMemcpyAsync(&va, &a.cnt[t - 1].va, 8, cudaMemcpyDeviceToHost, s));
-        GSW_CUDA(cudaStreamSynchronize(s));
-        done = va == 0;
+        if (b >= 2 || t >= max_iters) {
+            // check the previous batch (or, when no more can be enqueued, the last one)
+            const int chk = (t >= max_iters) ? (b - 1) : (b - 2);
+            const int slot = chk & 1;
+            if (cudaError_t e = cudaEventSynchronize(evb[slot])) return poll_fail(e, "gsw_dpr: batch poll");
+            done = hva[slot] == 0 || t >= max_iters;
+        }
     }
+    cudaEventDestroy(evb[0]);
+    cudaEventDestroy(evb[1]);
     const int launched = t;
     k_dpr_out<<<grid, kDprBlock, 0, s>>>(a.r, g->g.perm, n, out);
     GSW_CUDA(cudaGetLastError());
