@@ -120,7 +120,7 @@ def pr(g, damping: float = 0.85, iters: int = 20, csc=None) -> np.ndarray:
 
 
 def dpr(g, damping: float = 0.85, eps: float = 1e-6, max_iters: int = 100000, csc=None):
-    """fp64 Delta-PageRank (oracle.c orc_dpr, DESIGN R15).  eps is the ABSOLUTE residual threshold.
+    """fp64 Delta-PageRank (oracle.c orc_dpr, DESIGN R16).  eps is the ABSOLUTE residual threshold.
 
     Returns (rank, iterations)."""
     off, col = _arrs(g)

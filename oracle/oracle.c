@@ -14,7 +14,7 @@
  *   orc_sssp         binary-heap Dijkstra (lazy deletion)      P:264-265 ([42]); footnote 2 P:411-413
  *   orc_cc           union-find, labels = min vertex id        P:263-264 ([53]); north_star
  *   orc_pr           fp64 power iteration, dangling mass       P:264 ([11]); SURVEY Q9
- *   orc_dpr          Delta-PageRank, fp64, threshold eps       P:386-388 ([19]); Fig. 3; DESIGN R15
+ *   orc_dpr          Delta-PageRank, fp64, threshold eps       P:386-388 ([19]); Fig. 3; DESIGN R16
  *   orc_bc           Brandes, sigma u64, delta fp64            P:265-266 ([47],[10] P:1584-1585)
  *   orc_attrs        dataset attributes N,M,dbar,sd,rd,GI,Her  Table 1; [29]
  *   orc_ratios       Vap,Eap,Viap,Eiap,cd from counts          Table 1; record R P:948-951
@@ -210,7 +210,7 @@ int orc_pr(int64_t n, const int64_t *csr_off, const int64_t *csc_off, const int3
 
 /* ---------------------------------------------------------------- Delta-PageRank (fp64) */
 /*
- * Delta-PageRank ([19]; Fig. 3 "Iteration No. of Delta-PR"), reading R15.
+ * Delta-PageRank ([19]; Fig. 3 "Iteration No. of Delta-PR"), reading R16.
  * Each vertex holds a rank r and an unpropagated residual delta.  With M(w,v) = 1/deg_out(v) for
  * every edge v->w (no dangling teleport), the fixed point is x = (1-d)/N 1 + d M x, and
  *   delta_0(v) = (1-d)/N,  r_0 = 0;   iteration t:
