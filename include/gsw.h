@@ -133,7 +133,8 @@ gsw_status gsw_graph_attributes(gsw_graph g, double out[7]);
  * Each non-AUTO field overrides the selector.  Unsupported combinations return
  * GSW_EUNSUPPORTED at run time:
  *   - PR: fusion is ignored (every vertex is active every iteration);
- *   - BC backward sweep always pulls; forcing applies to the forward (sigma) phase.
+ *   - BC backward sweep always pulls; forcing applies to the forward (sigma) phase;
+ *   - Delta-PR (gsw_dpr): only the direction is honoured (push or pull every iteration).
  * Pinning any field also disables the CTA-resident ("solo") tier of BFS/SSSP, so a forced run
  * executes exactly the pinned patterns.  Environment knobs read at each run (calibration only):
  * GSW_SELECTOR=trees (BFS: learned CART trees instead of the hand-set rules), GSW_SOLO_E /
