@@ -138,7 +138,8 @@ gsw_status gsw_graph_attributes(gsw_graph g, double out[7]);
  * Pinning any field also disables the CTA-resident ("solo") tier of BFS/SSSP, so a forced run
  * executes exactly the pinned patterns.  Environment knobs read at each run (calibration only):
  * GSW_SELECTOR=trees (BFS: learned CART trees instead of the hand-set rules), GSW_SOLO_E /
- * GSW_SOLO_V (solo-tier thresholds; GSW_SOLO_E=0 disables it), GSW_SSSP_LAW (stepping law).
+ * GSW_SOLO_V (solo-tier thresholds; GSW_SOLO_E=0 disables it), GSW_SSSP_LAW (stepping law),
+ * GSW_DPR_PULL_K (Delta-PR: pull iff K*Ea > nnz, default 2).
  */
 gsw_status gsw_force_config(gsw_graph g, const gsw_config *cfg);
 

@@ -22,6 +22,7 @@
 // count once per batch of iterations, one batch behind the stream; kernels after the empty
 // iteration are no-ops.
 #include <algorithm>
+#include <cstdlib>
 #include <vector>
 
 #include "common.cuh"
@@ -62,6 +63,7 @@ struct DprArgs {
     unsigned *qlen;            // per iteration (max_iters entries)
     DprCnt *cnt;
     int force_dir;
+    unsigned pull_k;                     // pull iff Ea * pull_k > nnz (2: the paper's Ea > Eia)
     const Chunk *chunk_out, *chunk_in;   // heavy-row chunk tables (push: out-rows, pull: in-rows)
     unsigned nchunk_out, nchunk_in;
 };
@@ -155,7 +157,7 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_filter(DprArgs a, int t) {
 // 1 = push, 2 = pull (GSW_PUSH / GSW_PULL)
 __device__ __forceinline__ int dpr_dir(const DprArgs &a, const DprCnt &c) {
     if (a.force_dir) return a.force_dir;
-    return c.ea > (unsigned long long)a.nnz - c.ea ? GSW_PULL : GSW_PUSH;
+    return c.ea * a.pull_k > (unsigned long long)a.nnz ? GSW_PULL : GSW_PUSH;
 }
 
 // Edge-balanced tiers shared by push and pull (Delta-PR):
@@ -351,6 +353,10 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
     a.d = damping;
     a.eps = tol * (1.0 - damping) / (double)n;
     a.force_dir = fdir;
+    {   // GSW_DPR_PULL_K: calibration knob for the direction split (default 2)
+        const char *e = std::getenv("GSW_DPR_PULL_K");
+        a.pull_k = (e && *e && std::atoi(e) > 0) ? (unsigned)std::atoi(e) : 2u;
+    }
     a.r = (double *)ws.take((size_t)n * 8);
     a.delta = (double *)ws.take((size_t)n * 8);
     a.acc = (double *)ws.take((size_t)n * 8);
