@@ -133,11 +133,12 @@ def test_c1_full(gsw):
 
 
 @pytest.mark.slow
-def test_c3_mass_band(gsw):
-    """Full C3: x's total mass is known in closed form ((N - iso) + iso (1-d)) / N for an
+@pytest.mark.parametrize("cfg", ["C3", "C4"])
+def test_full_mass_band(gsw, cfg):
+    """Full C3 / C4: x's total mass is known in closed form ((N - iso) + iso (1-d)) / N for an
     undirected graph (M column-stochastic off the isolated vertices), so 0 <= sum(x - r) <= tol
     is checked at full size without the fixed point."""
-    g = gen.config_graph("C3")
+    g = gen.config_graph(cfg)
     tol = 1e-6
     r, st = gsw.Graph(g.off, g.col).dpr(D, tol)
     r = r.cpu().numpy()
