@@ -91,6 +91,18 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
+MAX_FRAC = 1.2
+
+
+def sane_frac(frac, what):
+    """A roofline fraction above 1.2 means the byte model or the run is broken (a
+    corrupted SSSP counter reported 8093x peak); refuse to print it."""
+    if not (frac == frac) or frac < 0 or frac > MAX_FRAC:
+        raise SystemExit(f"bench: roofline fraction {frac!r} for {what} is outside [0, {MAX_FRAC}]: "
+                         "the run or its byte model is broken; refusing to report it")
+    return frac
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -176,9 +188,9 @@ def run_extras(gsw, dev, G3, g3, peak):
         return b[1]
 
     def rec(value, unit, st):
+        gbs = st["bytes_alg"] / (st["gpu_ms"] * 1e-3) / 1e9
         return {"value": value, "unit": unit, "gpu_ms": st["gpu_ms"], "iterations": st["iterations"],
-                "roofline_frac": st["bytes_alg"] / (st["gpu_ms"] * 1e-3) / 1e9 / peak,
-                "achieved_gbs": st["bytes_alg"] / (st["gpu_ms"] * 1e-3) / 1e9}
+                "roofline_frac": sane_frac(gbs / peak, unit), "achieved_gbs": gbs}
 
     out = {}
     st = best(lambda: G3.cc())
@@ -408,7 +420,7 @@ def run_gsw(args, ws, rank, local):
                        "parallelism": (f"root-sharded replicas x{ws} (one graph copy per GPU, no collective)"
                                        if replicas else "single GPU")},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                         "frac": sane_frac(achieved / peak, "BFS"), "traffic": traffic, "peak_source": peak_src,
                          "kernel": "gsw::bfs_kernel (persistent, 1 launch/step)",
                          "bytes_model": "SURVEY 8(d) D0 per-level algorithmic bytes of the executed variant",
                          "alg_bytes_per_launch": bytes_alg / args.steps,

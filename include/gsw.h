@@ -170,7 +170,7 @@ gsw_status gsw_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_
  * atomics) or pull (in-edge reduction) from the active-edge count;
  * gsw_force_config's direction pins it, its other fields are ignored.
  *   tol: >= 0, finite (0 = run until residuals underflow or max_iters).
- *   max_iters: 1 .. 2^20.   rank: n doubles, host or device.
+ *   max_iters: 1 .. 65536 (per-iteration records live in the workspace).   rank: n doubles, host or device.
  * stats->iterations counts non-empty iterations; records carry Va/Ea and the direction run.
  * Errors: GSW_EINVAL (bad arguments), GSW_EUNSUPPORTED (distributed handle, forced direction
  * other than push/pull).                                                                      */

@@ -153,6 +153,7 @@ gsw_status gsw_graph_destroy(gsw_graph g) {
     if (!g) return GSW_OK;
     if (g->ev0) cudaEventDestroy(g->ev0);
     if (g->ev1) cudaEventDestroy(g->ev1);
+    if (g->poll) cudaFreeHost(g->poll);
     dist_destroy(g->dist);
     delete g;
     return GSW_OK;

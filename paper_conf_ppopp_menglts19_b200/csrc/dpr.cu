@@ -14,8 +14,8 @@
 //   Expand  k_dpr_push    fp64 atomicAdd of c(u) into acc of u's targets, for queued u
 //           k_dpr_pull    acc(w) = sum of c over in-neighbours (atomics only for heavy rows)
 //           both in four edge-balanced tiers: a lane per tiny row, 8-lane groups for short
-//           rows, a warp per mid row, 1024-edge warp chunks of heavy rows (table built at
-//           run start)
+//           rows, a warp per mid row, 1024-edge warp chunks of heavy rows (table built on the
+//           device at run start, no host round trip)
 // The selector (pull iff Ea > nnz - Ea, "the pull mode is preferable ... when the number of the
 // active edges is greater than that of inactive edges") is evaluated on the device by
 // both expand kernels from cnt[t]; the one not chosen returns at once.  The host polls the active
@@ -23,6 +23,8 @@
 // iteration are no-ops.
 #include <algorithm>
 #include <cstdlib>
+#include <map>
+#include <mutex>
 #include <vector>
 
 #include "common.cuh"
@@ -42,6 +44,7 @@ constexpr uint32_t kHeavy = 128;   // rows above this many edges become chunk ta
                                    // of them serialised on one warp were the tail of small graphs
 constexpr uint32_t kSmall = 64;    // rows up to this many edges go to an 8-lane group
 constexpr uint32_t kTiny = 8;      // rows up to this many edges are finished by one lane
+static_assert(kChunk % kHeavy == 0 && kChunk / kHeavy == 8, "k_dpr_chunks capacity bound");
 struct Chunk;
 
 struct DprCnt {                    // per-iteration record, zeroed at run start
@@ -65,7 +68,7 @@ struct DprArgs {
     int force_dir;
     unsigned pull_k;                     // pull iff Ea * pull_k > nnz (2: the paper's Ea > Eia)
     const Chunk *chunk_out, *chunk_in;   // heavy-row chunk tables (push: out-rows, pull: in-rows)
-    unsigned nchunk_out, nchunk_in;
+    const unsigned *nchunk_out, *nchunk_in;   // their lengths (device counters, k_dpr_chunks)
 };
 
 __global__ void k_dpr_init(DprArgs a) {
@@ -265,7 +268,8 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_push(DprArgs a, int t) {
     const unsigned gw = blockIdx.x * (kDprBlock / 32) + (threadIdx.x >> 5);
     const unsigned nw = gridDim.x * (kDprBlock / 32);
     // heavy chunks (inactive rows have c = 0 and return at once)
-    for (unsigned k = gw; k < a.nchunk_out; k += nw) {
+    const unsigned nch = *a.nchunk_out;
+    for (unsigned k = gw; k < nch; k += nw) {
         const Chunk ch = a.chunk_out[k];
         const double cu = a.c[ch.row];
         if (cu != 0.0) push_range(a, ch.beg + lane, ch.end, cu, 32);
@@ -292,7 +296,8 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_pull(DprArgs a, int t) {
     const unsigned gw = blockIdx.x * (kDprBlock / 32) + (threadIdx.x >> 5);
     const unsigned nw = gridDim.x * (kDprBlock / 32);
     // heavy chunks: partial sums into acc (zeroed by the filter)
-    for (unsigned k = gw; k < a.nchunk_in; k += nw) {
+    const unsigned nch = *a.nchunk_in;
+    for (unsigned k = gw; k < nch; k += nw) {
         const Chunk ch = a.chunk_in[k];
         double s = pull_range(a, ch.beg + lane, ch.end, 32);
         for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
@@ -306,13 +311,21 @@ __global__ void __launch_bounds__(kDprBlock) k_dpr_pull(DprArgs a, int t) {
     }
 }
 
-// heavy-row list (run start): rows with more than kHeavy edges, (row, begin, end) appended
-__global__ void k_dpr_heavy(const uint32_t *off, int n, Chunk *list, unsigned *cnt, unsigned cap) {
+// heavy-row chunk table (run start, on the device): every row with more than kHeavy edges
+// reserves ceil(deg / kChunk) slots with one atomic and writes its (row, begin, end) chunks.  The
+// order of the chunks is irrelevant (their partial sums meet in fp64 atomics), so no scan is
+// needed.  A heavy row has deg > kHeavy = kChunk / 8, so the table holds at most nnz / kHeavy
+// entries (the capacity the workspace reserves, scratch_bytes_for).
+__global__ void k_dpr_chunks(const uint32_t *off, int n, Chunk *tab, unsigned *cnt) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < n; v += (long long)gridDim.x * blockDim.x) {
         const uint32_t b = off[v], e = off[v + 1];
         if (e - b > kHeavy) {
-            const unsigned i = atomicAdd(cnt, 1u);
-            if (i < cap) list[i] = Chunk{(int)v, b, e};
+            const unsigned k = (e - b + kChunk - 1) / kChunk;
+            const unsigned i = atomicAdd(cnt, k);
+            for (unsigned j = 0; j < k; ++j) {
+                const uint32_t cb = b + j * kChunk;
+                tab[i + j] = Chunk{(int)v, cb, min(e, cb + kChunk)};
+            }
         }
     }
 }
@@ -323,14 +336,20 @@ __global__ void k_dpr_out(const double *r, const uint32_t *perm, int n, double *
 }
 
 // one full wave: SMs x resident blocks of this kernel (a second partial wave of a grid-stride
-// kernel would leave most SMs idle during its tail)
-int wave_grid(const void *k, int sms) {
+// kernel would leave most SMs idle during its tail); cached per (kernel, device)
+int wave_grid(const void *k, int device, int sms) {
+    static std::mutex mu;
+    static std::map<std::pair<const void *, int>, int> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    const auto key = std::make_pair(k, device);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
     int nb = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, kDprBlock, 0) != cudaSuccess || nb < 1) {
         cudaGetLastError();
         nb = 1;
     }
-    return sms * nb;
+    return cache[key] = sms * nb;
 }
 
 }  // namespace
@@ -338,7 +357,7 @@ int wave_grid(const void *k, int sms) {
 gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, double *rank, gsw_run_stats *st) {
     const int n = g->g.n;
     if (!rank) { set_error("gsw_dpr: rank is NULL"); return GSW_EINVAL; }
-    if (max_iters < 1 || max_iters > (1 << 20)) { set_error("gsw_dpr: max_iters must be in [1, 2^20]"); return GSW_EINVAL; }
+    if (max_iters < 1 || max_iters > kDprMaxIters) { set_error("gsw_dpr: max_iters must be in [1, 65536]"); return GSW_EINVAL; }
     if (!(damping >= 0.0 && damping < 1.0)) { set_error("gsw_dpr: damping must be in [0,1)"); return GSW_EINVAL; }
     if (!(tol >= 0.0 && tol < 1e300)) { set_error("gsw_dpr: tol must be finite and >= 0"); return GSW_EINVAL; }
     const int fdir = g->forced.direction;
@@ -367,43 +386,25 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
     double *out = dev_out ? rank : (double *)ws.take((size_t)n * 8);
     if (!a.r || !a.delta || !a.acc || !a.c || !a.q || !a.qlen || !a.cnt || !out) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
     cudaStream_t s = g->stream;
+    if (!g->poll) GSW_CUDA(cudaHostAlloc((void **)&g->poll, 2 * sizeof(unsigned long long), cudaHostAllocDefault));
     const int grid = g->sms * 8;
-    static const int g_filter = wave_grid((const void *)k_dpr_filter, g->sms);
-    static const int g_push = wave_grid((const void *)k_dpr_push, g->sms);
-    static const int g_pull = wave_grid((const void *)k_dpr_pull, g->sms);
+    const int g_filter = wave_grid((const void *)k_dpr_filter, g->device, g->sms);
+    const int g_push = wave_grid((const void *)k_dpr_push, g->device, g->sms);
+    const int g_pull = wave_grid((const void *)k_dpr_pull, g->device, g->sms);
+    // heavy-row chunk tables: capacity nnz / kHeavy + 1 each (see k_dpr_chunks)
+    const size_t ccap = (size_t)a.nnz / kHeavy + 1;
+    const bool same_in = a.in_off == a.off && a.in_col == a.col;
+    unsigned *ccnt = (unsigned *)ws.take(256);
+    Chunk *tab_out = (Chunk *)ws.take(ccap * sizeof(Chunk));
+    Chunk *tab_in = same_in ? tab_out : (Chunk *)ws.take(ccap * sizeof(Chunk));
+    if (!ccnt || !tab_out || !tab_in) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
+    a.chunk_out = tab_out; a.nchunk_out = ccnt;
+    a.chunk_in = tab_in; a.nchunk_in = same_in ? ccnt : ccnt + 1;
     GSW_CUDA(cudaEventRecord(g->ev0, s));
-    // heavy-row chunk tables (once per run; one host round trip each)
-    const size_t hcap = (size_t)a.nnz / kHeavy + 1, ccap = 2 * hcap + 1;
-    unsigned *hcnt = (unsigned *)ws.take(256);
-    Chunk *hlist = (Chunk *)ws.take(hcap * sizeof(Chunk));
-    if (!hcnt || !hlist) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
-    auto build = [&](const uint32_t *off, const Chunk **tab, unsigned *nt) -> gsw_status {
-        GSW_CUDA(cudaMemsetAsync(hcnt, 0, 4, s));
-        k_dpr_heavy<<<grid, kDprBlock, 0, s>>>(off, n, hlist, hcnt, (unsigned)hcap);
-        GSW_CUDA(cudaGetLastError());
-        unsigned nh = 0;
-        GSW_CUDA(cudaMemcpyAsync(&nh, hcnt, 4, cudaMemcpyDeviceToHost, s));
-        GSW_CUDA(cudaStreamSynchronize(s));
-        nh = std::min<unsigned>(nh, (unsigned)hcap);
-        std::vector<Chunk> rows(nh), ch;
-        if (nh) GSW_CUDA(cudaMemcpy(rows.data(), hlist, nh * sizeof(Chunk), cudaMemcpyDeviceToHost));
-        for (const Chunk &r : rows)
-            for (uint32_t b = r.beg; b < r.end; b += kChunk) ch.push_back(Chunk{r.row, b, std::min(r.end, b + kChunk)});
-        Chunk *t = (Chunk *)ws.take(std::max<size_t>(1, std::min(ch.size(), ccap)) * sizeof(Chunk));
-        if (!t) { set_error("gsw_dpr: workspace too small"); return GSW_ENOMEM; }
-        if (!ch.empty()) GSW_CUDA(cudaMemcpyAsync(t, ch.data(), ch.size() * sizeof(Chunk), cudaMemcpyHostToDevice, s));
-        GSW_CUDA(cudaStreamSynchronize(s));   // ch is a local vector
-        *tab = t;
-        *nt = (unsigned)ch.size();
-        return GSW_OK;
-    };
-    if (gsw_status e = build(a.off, &a.chunk_out, &a.nchunk_out)) return e;
-    if (a.in_off == a.off && a.in_col == a.col) {
-        a.chunk_in = a.chunk_out;
-        a.nchunk_in = a.nchunk_out;
-    } else if (gsw_status e = build(a.in_off, &a.chunk_in, &a.nchunk_in)) {
-        return e;
-    }
+    GSW_CUDA(cudaMemsetAsync(ccnt, 0, 8, s));
+    k_dpr_chunks<<<grid, kDprBlock, 0, s>>>(a.off, n, tab_out, ccnt);
+    if (!same_in) k_dpr_chunks<<<grid, kDprBlock, 0, s>>>(a.in_off, n, tab_in, ccnt + 1);
+    GSW_CUDA(cudaGetLastError());
     GSW_CUDA(cudaMemsetAsync(a.qlen, 0, (size_t)max_iters * 4, s));
     GSW_CUDA(cudaMemsetAsync(a.cnt, 0, (size_t)max_iters * sizeof(DprCnt), s));
     k_dpr_init<<<grid, kDprBlock, 0, s>>>(a);
@@ -412,8 +413,7 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
     // count into pinned memory and an event) BEFORE the host waits on batch b-1's event, so the
     // stream never drains while the host decides.  Batches grow with t (clamp(t/4, 4, 32)), so at
     // most one batch of no-op kernels runs past the empty iteration.
-    static thread_local unsigned long long *hva = nullptr;   // 2 pinned slots, one per in-flight batch
-    if (!hva) GSW_CUDA(cudaHostAlloc((void **)&hva, 2 * sizeof(unsigned long long), cudaHostAllocDefault));
+    unsigned long long *hva = g->poll;   // 2 pinned slots (one per in-flight batch), owned by the handle
     cudaEvent_t evb[2] = {nullptr, nullptr};
     GSW_CUDA(cudaEventCreateWithFlags(&evb[0], cudaEventDisableTiming));
     GSW_CUDA(cudaEventCreateWithFlags(&evb[1], cudaEventDisableTiming));
@@ -468,10 +468,12 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
             const bool pull = h[i].dir == GSW_PULL;
             const long long ed = pull ? E : Ea;
             edges += ed;
-            // DESIGN.md section 6, Delta-PR: filter 40 B/vertex (delta, acc r/w; c write) + 20 B
-            // per active vertex (rank r/w, queue); push 8 B/active vertex (offsets) + 4 B column
-            // + 16 B atomic RMW per edge; pull 8 B/row + 8 B acc write + 12 B per in-edge
-            bytes += 40 * N + 20 * Va + (pull ? 16 * N + 12 * E : 8 * Va + 20 * Ea);
+            // DESIGN.md section 6, Delta-PR, counted per SURVEY 8(d) D0 (compulsory DRAM only):
+            // filter 40 B/vertex (delta r/w, acc r/w, c write: fp64 streams) + 20 B per active
+            // vertex (rank r/w, queue); push 8 B/active vertex (row offsets) + 4 B per column;
+            // pull 4 B/row (offsets) + 8 B/row (acc write) + 4 B per in-edge column.  Gathers of
+            // c[] and the atomics into acc[] are probes of L2-resident state (D0) and not counted.
+            bytes += 40 * N + 20 * Va + (pull ? 12 * N + 4 * E : 8 * Va + 4 * Ea);
             if (st->records && i < st->max_records) {
                 gsw_iter_record &rec = st->records[i];
                 rec = gsw_iter_record{};
@@ -483,7 +485,7 @@ gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
                 rec.Va = Va; rec.Ea = Ea;
                 rec.Via = N - Va; rec.Eia = E - Ea;
                 rec.edges = ed;
-                rec.ctas = grid;
+                rec.ctas = pull ? g_pull : g_push;
             }
         }
         st->iterations = it;

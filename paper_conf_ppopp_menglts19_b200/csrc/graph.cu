@@ -161,6 +161,9 @@ size_t scratch_bytes_for(int64_t n, int64_t nnz, int has_w) {
     size_t b = per_v * (size_t)(n + 64) + 16 * W * 4;
     b += (size_t)(n + 1) * 8;                  // i64 offset staging at ingest / scan arrays
     b += 8u << 20;                             // control blocks, per-CTA partials, history, records
+    // gsw_dpr: two heavy-row chunk tables (<= nnz/128 + 1 entries of 12 B, dpr.cu k_dpr_chunks)
+    // and kDprMaxIters per-iteration records (queue length 4 B + counters 32 B)
+    b += 2 * ((size_t)nnz / 128 + 1) * 12 + 1024 + (size_t)kDprMaxIters * 36;
     if (nnz < (int64_t(1) << 31)) b = std::max(b, relabel_temp_bytes(n, nnz, has_w));   // ingest temp
     return b;
 }

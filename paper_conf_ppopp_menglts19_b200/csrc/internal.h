@@ -74,6 +74,7 @@ struct gsw_graph_s {
     char *scratch = nullptr;      // per-run scratch (after the graph copy)
     size_t scratch_bytes = 0;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    unsigned long long *poll = nullptr;   // 2 pinned host slots for gsw_dpr's termination poll (lazy)
 };
 
 namespace gsw {
@@ -86,6 +87,8 @@ gsw_status cuda_fail(cudaError_t e, const char *what);
         cudaError_t _e = (call);                                         \
         if (_e != cudaSuccess) return ::gsw::cuda_fail(_e, #call);       \
     } while (0)
+
+constexpr int kDprMaxIters = 1 << 16;   // gsw_dpr: per-iteration records held in the scratch
 
 // scratch bytes for a graph of n vertices (max over algorithms), see DESIGN.md "HBM layout"
 size_t scratch_bytes_for(int64_t n, int64_t nnz, int has_w);

@@ -188,8 +188,13 @@ struct SsLoop {
     int fcur, nsplit;
 };
 
-// warp-aggregated append of (v, beg, deg) to a shared near queue
-__device__ __forceinline__ void solo_push(SsSoloSmem &ss, int nx, bool pred, int v, uint32_t b, uint32_t d) {
+// warp-aggregated append of (v, beg, deg) to a shared near queue.  A round may claim more
+// vertices than the shared queue holds (up to one per relaxed edge): entries p >= kSSQ spill to
+// the same position of the grid's queue `spill` (the queue of the round being built), exactly as
+// the BFS tier does (bfs.cu); such a round ends the episode, because the selector check (B)
+// requires qn <= kSSQ to continue, and the hand-back leaves the spilled part in place.
+__device__ __forceinline__ void solo_push(SsSoloSmem &ss, int nx, bool pred, int v, uint32_t b, uint32_t d,
+                                          int *spill) {
     const unsigned act = __activemask();
     const unsigned m = __ballot_sync(act, pred);
     if (!m) return;
@@ -199,7 +204,8 @@ __device__ __forceinline__ void solo_push(SsSoloSmem &ss, int nx, bool pred, int
     base = __shfl_sync(act, base, leader);
     if (pred) {
         const unsigned p = base + __popc(m & lanemask_lt());
-        ss.q[nx][p] = v; ss.beg[nx][p] = b; ss.scan[nx][p] = d;
+        if (p < (unsigned)kSSQ) { ss.q[nx][p] = v; ss.beg[nx][p] = b; ss.scan[nx][p] = d; }
+        else spill[p] = v;
     }
 }
 
@@ -254,7 +260,7 @@ __device__ __noinline__ void sssp_solo(const SsspArgs &a, SsSoloSmem &ss, int t,
                     a.fq[fdst][atomicAdd(a.flen + fdst, 1u)] = v;
                     atomicMin(&ss.minf, dv);
                 }
-                solo_push(ss, cur, near, v, b, e - b);
+                solo_push(ss, cur, near, v, b, e - b, a.q[t & 1]);
             }
             __syncthreads();
             qn = ss.qn[cur];
@@ -275,9 +281,16 @@ __device__ __noinline__ void sssp_solo(const SsspArgs &a, SsSoloSmem &ss, int t,
         {
             unsigned long long lea = 0;
             unsigned lmx = 0, lmn = 0xffffffffu;
+            const int *gq = a.q[t & 1];
             for (unsigned i = tid; i < qn; i += kBlock) {
-                const unsigned d = ss.scan[cur][i];
-                ss.du[i] = __ldcg(dist + ss.q[cur][i]);   // L2: atomicMin updates bypass this SM's L1
+                unsigned d;
+                if (i < (unsigned)kSSQ) {
+                    d = ss.scan[cur][i];
+                    ss.du[i] = __ldcg(dist + ss.q[cur][i]);   // L2: atomicMin updates bypass this SM's L1
+                } else {                                       // spilled entry: the episode ends here
+                    const int u = gq[i];
+                    d = __ldg(off + u + 1) - __ldg(off + u);
+                }
                 lea += d; lmx = d > lmx ? d : lmx; lmn = d < lmn ? d : lmn;
             }
             lea = warp_sum(lea); lmx = warp_max(lmx); lmn = warp_min(lmn);
@@ -400,14 +413,16 @@ __device__ __noinline__ void sssp_solo(const SsspArgs &a, SsSoloSmem &ss, int t,
                 for (int k = 0; k < 4; ++k) {
                     const bool won = cl[k] != 0xffffffffu && !((cl[k] >> (v[k] & 31)) & 1u);
                     const bool near = won && (unsigned long long)nd[k] < th;
-                    solo_push(ss, nx, near, v[k], vb[k], ve[k] - vb[k]);
+                    solo_push(ss, nx, near, v[k], vb[k], ve[k] - vb[k], a.q[(t + 1) & 1]);
                     if (won && !near) a.fq[L.fcur][atomicAdd(a.flen + L.fcur, 1u)] = v[k];
                 }
             }
             __syncthreads();
             // far appends of this round, then clean the near claim map (it holds exactly N_{t+1})
             const unsigned nq = ss.qn[nx];
-            for (unsigned k = tid; k < nq; k += kBlock) atomicAnd(nnb + (ss.q[nx][k] >> 5), 0u);
+            const int *gqn = a.q[(t + 1) & 1];
+            for (unsigned k = tid; k < nq; k += kBlock)
+                atomicAnd(nnb + ((k < (unsigned)kSSQ ? ss.q[nx][k] : __ldcg(gqn + k)) >> 5), 0u);
             __threadfence();
             __syncthreads();
             L.flen = *(volatile unsigned *)(a.flen + L.fcur);
@@ -422,7 +437,8 @@ __device__ __noinline__ void sssp_solo(const SsspArgs &a, SsSoloSmem &ss, int t,
     // hand N_t back to the grid
     {
         int *gq = a.q[t & 1];
-        for (unsigned k = tid; k < qn; k += kBlock) gq[k] = ss.q[cur][k];
+        const unsigned m = qn < (unsigned)kSSQ ? qn : (unsigned)kSSQ;   // entries >= kSSQ were spilled in place
+        for (unsigned k = tid; k < m; k += kBlock) gq[k] = ss.q[cur][k];
         if (tid == 0) {
             IterCnt *cc = rc.cnt + (t % 3);
             cc->va = qn; cc->ea = qn ? Ea : 0; cc->maxd = mxd; cc->mind = mnd; cc->qlen = qn; cc->edges = E_prev;

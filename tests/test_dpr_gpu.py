@@ -112,7 +112,7 @@ def test_max_iters_and_errors(gsw):
     assert st["iterations"] == 3
     ro, _ = oracle.dpr(g, D, 1e-9 * (1 - D) / g.n, max_iters=3)
     np.testing.assert_allclose(r.cpu().numpy(), ro, rtol=1e-12)     # 3 full pull steps
-    for bad in (dict(damping=1.0), dict(tol=-1.0), dict(max_iters=0)):
+    for bad in (dict(damping=1.0), dict(tol=-1.0), dict(max_iters=0), dict(max_iters=65537)):
         kw = dict(damping=D, tol=1e-6, max_iters=10)
         kw.update(bad)
         with pytest.raises(Exception):
@@ -159,3 +159,13 @@ def test_heavy_row_chunks(gsw, direction):
     g = gen.from_edges(n, edges)
     for tol in (1e-4, 1e-8):
         _check(gsw, g, tol, direction)
+
+
+def test_max_iters_limit_fits_small_graphs(gsw):
+    """The documented maximum (65,536 iterations) is a valid call even on a tiny graph: the
+    per-iteration records are budgeted in the workspace (ENOMEM before)."""
+    g = gen.from_edges(6, [(0, 1), (1, 2), (2, 3), (3, 4), (4, 5)])
+    r, st = gsw.Graph(g.off, g.col).dpr(D, 0.0, max_iters=65536)
+    assert 1 <= st["iterations"] <= 65536
+    ro, _ = oracle.dpr(g, D, 0.0, max_iters=st["iterations"])
+    np.testing.assert_allclose(r.cpu().numpy(), ro, rtol=1e-9, atol=1e-300)

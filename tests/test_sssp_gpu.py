@@ -95,3 +95,50 @@ def test_c2_full_size(gsw):
     d, st = _sssp(gsw.Graph(g.off, g.col, g.w), 0)
     assert np.array_equal(d, oracle.sssp(g, 0))
     assert int(d.max()) == 62467 and int(d[-1]) == 62436
+
+
+def _hub_graph(n_leaves=3000, path=24):
+    """A path 0..path-1 ending at a hub with n_leaves leaves, each leaf with its own pendant vertex:
+    a solo round relaxing the hub's row claims n_leaves > 512 near vertices at once (VERDICT r1
+    weak #1: the CTA-resident queue holds 512)."""
+    edges = [(i, i + 1) for i in range(path - 1)]
+    hub = path - 1
+    leaves = range(path, path + n_leaves)
+    edges += [(hub, v) for v in leaves]
+    edges += [(v, v + n_leaves) for v in leaves]
+    return gen.from_edges(path + 2 * n_leaves, edges)
+
+
+@pytest.mark.parametrize("n_leaves", [511, 512, 513, 3000])
+def test_solo_tier_overflow_claims(gsw, monkeypatch, n_leaves):
+    """The SSSP solo tier with thresholds raised so a round claims more vertices than its shared
+    queue holds: distances stay bit-exact and the byte model stays physical, on 5 reruns."""
+    monkeypatch.setenv("GSW_SOLO_E", str(10 ** 7))
+    monkeypatch.setenv("GSW_SOLO_V", "512")
+    g = gen.with_hash_weights(_hub_graph(n_leaves), 77, 64)
+    ref = oracle.sssp(g, 0)
+    G = gsw.Graph(g.off, g.col, g.w)
+    for delta0 in (0, 10 ** 6):
+        G.force_config(delta0=delta0)
+        for _ in range(5):
+            d, st = _sssp(G, 0, records=4096)
+            assert np.array_equal(d, ref), (n_leaves, delta0)
+            # every counted byte is a touched CSR/state element: far below nnz*64 + n*64
+            assert 0 < st["bytes_alg"] < 64 * (g.nnz + g.n) * max(1, st["iterations"]), st["bytes_alg"]
+            assert st["edges_touched"] <= 64 * g.nnz
+
+
+def test_solo_tier_overflow_rmat(gsw, monkeypatch):
+    """Same on weighted R-MAT with a huge delta0 (every improved vertex near) and an unbounded
+    solo edge budget: hub rows inside the tier claim thousands of vertices."""
+    monkeypatch.setenv("GSW_SOLO_E", str(10 ** 7))
+    monkeypatch.setenv("GSW_SOLO_V", "512")
+    g = gen.with_hash_weights(gen.rmat(14, seed=11), 3, 64)
+    G = gsw.Graph(g.off, g.col, g.w)
+    for s in gen.sources(g, 3, seed=2):
+        ref = oracle.sssp(g, s)
+        for delta0 in (0, 10 ** 6):
+            G.force_config(delta0=delta0)
+            d, st = _sssp(G, s)
+            assert np.array_equal(d, ref), (s, delta0)
+            assert st["bytes_alg"] < 64 * (g.nnz + g.n) * max(1, st["iterations"])
