@@ -24,7 +24,7 @@ gen/libgswgen.so: gen/gen.c
 	gcc -O3 -fopenmp -fPIC -shared -o $@ $< -lm
 
 oracle/liboracle.so: oracle/oracle.c
-	gcc -O2 -fPIC -shared -o $@ $< -lm
+	gcc -O2 -fopenmp -fPIC -shared -o $@ $< -lm
 
 clean:
 	rm -rf build $(LIB) gen/libgswgen.so oracle/liboracle.so

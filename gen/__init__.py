@@ -43,6 +43,9 @@ def _load():
         lib = ctypes.CDLL(_SO)
         lib.gen_rmat.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_double, ctypes.c_double,
                                  ctypes.c_double, ctypes.c_uint64, ctypes.c_int, ctypes.POINTER(_Csr)]
+        lib.gen_rmat_slice.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_double, ctypes.c_double,
+                                       ctypes.c_double, ctypes.c_uint64, ctypes.c_int, ctypes.c_int64,
+                                       ctypes.c_int64, ctypes.POINTER(_Csr)]
         lib.gen_grid.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(_Csr)]
         lib.gen_chung_lu.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_double, ctypes.c_double,
                                      ctypes.c_uint64, ctypes.POINTER(_Csr)]
@@ -92,6 +95,19 @@ def rmat(scale: int, edgefactor: int = 16, a: float = 0.57, b: float = 0.19, c: 
     if rc != 0:
         raise MemoryError(f"gen_rmat failed rc={rc}")
     return _take(out, f"rmat{scale}_ef{edgefactor}_s{seed}")
+
+
+def rmat_slice(scale: int, vb: int, ve: int, edgefactor: int = 16, a: float = 0.57, b: float = 0.19,
+               c: float = 0.19, seed: int = 1, permute: bool = True):
+    """Rows [vb, ve) of ``rmat(scale, ...)`` as (offsets rebased to 0, global column ids), built
+    without materialising the other rows (gen.c gen_rmat_slice): one rank's share of a 1D
+    vertex-partitioned graph, or with [0, 2^scale) the whole graph."""
+    lib, out = _load(), _Csr()
+    rc = lib.gen_rmat_slice(scale, edgefactor, a, b, c, seed, int(permute), vb, ve, ctypes.byref(out))
+    if rc != 0:
+        raise MemoryError(f"gen_rmat_slice failed rc={rc}")
+    g = _take(out, "")
+    return g.off, g.col
 
 
 def grid(width: int, height: Optional[int] = None) -> Graph:
@@ -192,5 +208,6 @@ def config_graph(name: str) -> Graph:
     if name == "C4":
         return chung_lu(4_847_571, 68_993_773, gamma=2.3, i0=150.0, seed=3)
     if name == "C5":
-        return rmat(26, 16, seed=1)
+        off, col = rmat_slice(26, 0, 1 << 26, 16, seed=1)    # the same graph as rmat(26), built in parallel
+        return Graph(1 << 26, off, col, None, "rmat26_ef16_s1")
     raise KeyError(name)

@@ -154,6 +154,89 @@ int gen_rmat(int scale, int edgefactor, double a, double b, double c, uint64_t s
     return rc;
 }
 
+/* The l-th R-MAT tuple of gen_rmat (before the permutation). */
+static inline void rmat_tuple(int scale, double a, double ab, double abc, uint64_t seed, int64_t k,
+                              uint32_t *pu, uint32_t *pv) {
+    uint32_t u = 0, v = 0;
+    for (int l = 0; l < scale; ++l) {
+        double r = u01(crng(seed, 1, (uint64_t)k * (uint64_t)scale + (uint64_t)l));
+        uint32_t bu, bv;
+        if (r < a) { bu = 0; bv = 0; }
+        else if (r < ab) { bu = 0; bv = 1; }
+        else if (r < abc) { bu = 1; bv = 0; }
+        else { bu = 1; bv = 1; }
+        u = (u << 1) | bu; v = (v << 1) | bv;
+    }
+    *pu = u; *pv = v;
+}
+
+/* Rows [vb, ve) of exactly the graph gen_rmat builds (same tuples, permutation, symmetrisation,
+ * loop removal and per-row dedupe), with offsets rebased to 0 (out->n = ve - vb rows, columns are
+ * global ids).  No tuple array is held: the tuples are regenerated twice (count, then fill), so
+ * memory is the slice's CSR plus the permutation.  This is how each rank of the partitioned C5
+ * runs builds only its own rows, and with [0, n) a memory-light parallel builder of
+ * the whole graph. */
+int gen_rmat_slice(int scale, int edgefactor, double a, double b, double c, uint64_t seed,
+                   int permute, int64_t vb, int64_t ve, gen_csr *out) {
+    if (scale < 1 || scale > 30 || edgefactor < 1) return -2;
+    const int64_t n = (int64_t)1 << scale, m = (int64_t)edgefactor * n;
+    if (vb < 0 || ve > n || vb > ve) return -2;
+    const int64_t rows = ve - vb;
+    const double ab = a + b, abc = a + b + c;
+    uint32_t *p = permute ? make_perm(n, seed) : NULL;
+    if (permute && !p) return -1;
+    int64_t *cnt = (int64_t *)calloc((size_t)rows + 1, sizeof(int64_t));
+    if (!cnt) { free(p); return -1; }
+#pragma omp parallel for schedule(static)
+    for (int64_t k = 0; k < m; ++k) {
+        uint32_t u, v;
+        rmat_tuple(scale, a, ab, abc, seed, k, &u, &v);
+        if (p) { u = p[u]; v = p[v]; }
+        if (u == v) continue;
+        if ((int64_t)u >= vb && (int64_t)u < ve) __atomic_fetch_add(&cnt[u - vb + 1], 1, __ATOMIC_RELAXED);
+        if ((int64_t)v >= vb && (int64_t)v < ve) __atomic_fetch_add(&cnt[v - vb + 1], 1, __ATOMIC_RELAXED);
+    }
+    for (int64_t i = 0; i < rows; ++i) cnt[i + 1] += cnt[i];
+    const int64_t tot = cnt[rows];
+    int32_t *col = (int32_t *)malloc((size_t)(tot ? tot : 1) * sizeof(int32_t));
+    int64_t *pos = (int64_t *)malloc((size_t)(rows ? rows : 1) * sizeof(int64_t));
+    if (!col || !pos) { free(p); free(cnt); free(col); free(pos); return -1; }
+    memcpy(pos, cnt, (size_t)rows * sizeof(int64_t));
+#pragma omp parallel for schedule(static)
+    for (int64_t k = 0; k < m; ++k) {
+        uint32_t u, v;
+        rmat_tuple(scale, a, ab, abc, seed, k, &u, &v);
+        if (p) { u = p[u]; v = p[v]; }
+        if (u == v) continue;
+        if ((int64_t)u >= vb && (int64_t)u < ve) col[__atomic_fetch_add(&pos[u - vb], 1, __ATOMIC_RELAXED)] = (int32_t)v;
+        if ((int64_t)v >= vb && (int64_t)v < ve) col[__atomic_fetch_add(&pos[v - vb], 1, __ATOMIC_RELAXED)] = (int32_t)u;
+    }
+    free(p);
+    free(pos);
+    int64_t *deg = (int64_t *)malloc((size_t)(rows ? rows : 1) * sizeof(int64_t));
+    if (!deg) { free(cnt); free(col); return -1; }
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t i = 0; i < rows; ++i) {
+        int32_t *r = col + cnt[i];
+        int64_t len = cnt[i + 1] - cnt[i];
+        if (len > 1) qsort(r, (size_t)len, sizeof(int32_t), cmp_i32);
+        int64_t k = 0;
+        for (int64_t j = 0; j < len; ++j)
+            if (k == 0 || r[j] != r[k - 1]) r[k++] = r[j];
+        deg[i] = k;
+    }
+    int64_t *off = (int64_t *)malloc(((size_t)rows + 1) * sizeof(int64_t));
+    if (!off) { free(cnt); free(col); free(deg); return -1; }
+    off[0] = 0;
+    for (int64_t i = 0; i < rows; ++i) off[i + 1] = off[i] + deg[i];
+    /* compact in place: rows move only towards lower addresses (off[i] <= cnt[i]) */
+    for (int64_t i = 0; i < rows; ++i)
+        if (off[i] != cnt[i]) memmove(col + off[i], col + cnt[i], (size_t)deg[i] * sizeof(int32_t));
+    free(cnt); free(deg);
+    out->n = rows; out->nnz = off[rows]; out->off = off; out->col = col; out->w = NULL;
+    return 0;
+}
+
 int gen_grid(int64_t width, int64_t height, gen_csr *out) {
     if (width < 1 || height < 1) return -2;
     int64_t n = width * height;

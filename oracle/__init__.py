@@ -4,8 +4,9 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
 reference`` legs may import this package.  The product path never imports it; it shares no code
 with ``paper_conf_ppopp_menglts19_b200``.
 
-Thin ctypes wrapper over ``oracle/oracle.c`` (plain single-threaded C, see its header for the
-paper citations of every function).
+Thin ctypes wrapper over ``oracle/oracle.c`` (plain C, see its header for the paper citations of
+every function and for the one place OpenMP is used: the per-vertex loops of PR / Delta-PR,
+bit-identical to one thread).
 """
 from __future__ import annotations
 
@@ -25,8 +26,9 @@ P = ctypes.c_void_p
 def build() -> str:
     src = os.path.join(_HERE, "oracle.c")
     if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
-        # -O2 plain C, single thread; no -ffast-math (keeps fp64 order as written)
-        subprocess.check_call(["gcc", "-O2", "-fPIC", "-shared", "-o", _SO, src, "-lm"])
+        # -O2 plain C; no -ffast-math (keeps fp64 order as written); OpenMP only across the
+        # vertices of orc_pr / orc_dpr (bit-identical to one thread, see oracle.c's header)
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", _SO, src, "-lm"])
     return _SO
 
 
@@ -47,6 +49,9 @@ def _load():
         lib.orc_attrs.argtypes = [i64, P, P]
         lib.orc_ratios.argtypes = [i64, i64, i64, i64, i64, i64, P]
         lib.orc_ratios.restype = None
+        lib.orc_set_threads.argtypes = [ctypes.c_int]
+        lib.orc_set_threads.restype = None
+        lib.orc_threads.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -152,3 +157,12 @@ def ratios(N, M, Va, Ea, Via, Eia) -> dict:
     out = np.empty(5, np.float64)
     _load().orc_ratios(N, M, Va, Ea, Via, Eia, _p(out))
     return dict(zip(["Vap", "Eap", "Viap", "Eiap", "cd"], out.tolist()))
+
+
+def set_threads(k: int) -> None:
+    """Threads for the per-vertex loops of pr / dpr (0 = all cores); results do not depend on it."""
+    _load().orc_set_threads(int(k))
+
+
+def threads() -> int:
+    return int(_load().orc_threads())

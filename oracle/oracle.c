@@ -7,7 +7,12 @@
  * and neither side includes or links the other.
  *
  * Every function computes the plain definition of what the method computes,
- * single-threaded, in the textbook order.  Citations are PAPER.md line numbers ("P:nnn").
+ * in the textbook order.  Citations are PAPER.md line numbers ("P:nnn").  Everything is single-
+ * threaded except the per-vertex loops of orc_pr and orc_dpr, which OpenMP spreads over vertices:
+ * each vertex's sum is still computed by one thread in ascending in-edge order and the dangling
+ * mass / activation counts stay serial, so the result is bit-identical to the serial loop
+ * (tests/test_oracle.py checks 1 thread vs all); this only makes full-size checks (C3 Delta-PR,
+ * C5 PageRank) finish in minutes.  orc_set_threads(k) pins the thread count (0 = OpenMP default).
  *
  *   orc_bfs          FIFO-queue BFS depths                    P:262-263 ([7]); Fig. 11
  *   orc_bfs_features per-level Va/Ea/Via/Eia of the BFS        Table 1; record R P:948-951
@@ -30,11 +35,30 @@
 #include <stdlib.h>
 #include <string.h>
 #include <math.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 #define ORC_OK 0
 #define ORC_ENOMEM (-1)
 #define ORC_EINVAL (-2)
 #define ORC_EOVERFLOW (-3)
+
+void orc_set_threads(int k) {
+#ifdef _OPENMP
+    omp_set_num_threads(k > 0 ? k : omp_get_num_procs());
+#else
+    (void)k;
+#endif
+}
+
+int orc_threads(void) {
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
 
 /* ---------------------------------------------------------------- BFS (FIFO) */
 int orc_bfs(int64_t n, const int64_t *off, const int32_t *col, int32_t src, int32_t *depth) {
@@ -194,6 +218,7 @@ int orc_pr(int64_t n, const int64_t *csr_off, const int64_t *csc_off, const int3
         double D = 0.0;
         for (int64_t u = 0; u < n; ++u)
             if (csr_off[u + 1] == csr_off[u]) D += pr[u];
+#pragma omp parallel for schedule(dynamic, 4096)
         for (int64_t v = 0; v < n; ++v) {
             double s = 0.0;
             for (int64_t e = csc_off[v]; e < csc_off[v + 1]; ++e) {
@@ -239,6 +264,7 @@ int orc_dpr(int64_t n, const int64_t *csr_off, const int64_t *csc_off, const int
         if (na == 0) break;
         for (int64_t v = 0; v < n; ++v)
             if (act[v]) r[v] += delta[v];
+#pragma omp parallel for schedule(dynamic, 4096)
         for (int64_t w = 0; w < n; ++w) {
             double s = 0.0;
             for (int64_t e = csc_off[w]; e < csc_off[w + 1]; ++e) {

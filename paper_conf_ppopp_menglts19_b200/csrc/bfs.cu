@@ -215,6 +215,7 @@ __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, 
             word = ~orig;                                   // padding bits are set in V
             found_bits[lane] = 0u;
         }
+        __syncwarp();                                       // found_bits reset before lane 0's stores
         // pass 1: probe the first in-neighbour (the highest-degree one) of every unvisited vertex,
         // coalesced through in_first, 8 words in flight (one load + one probe per vertex: the row
         // bounds are not needed yet).  Hits go to the top of the list (their degrees are loaded

@@ -118,9 +118,38 @@ __device__ __noinline__ LocalCnt lb_thread(const Src src, const Adj g, Op op) {
 }
 
 // ------------------------------------------------------------------ TWC
+// CTA-tier election of TWC (a row with degree >= blockDim is expanded by the whole CTA).  Every
+// warp publishes its ballot of big rows and its first candidate (row, begin, end) into the half
+// of a double buffer selected by the round's parity; after one barrier every thread picks the
+// lowest warp with a candidate.  A half is rewritten two rounds later, after the intervening
+// round's barrier, so no reset store (and no write-write race between candidates) is needed --
+// the single "owner" word with a reset store raced under compute-sanitizer racecheck (round 2).
+struct TwcElect {
+    unsigned ball[2][kWarps];
+    int cx[2][kWarps];
+    uint32_t cb[2][kWarps], ce[2][kWarps];
+};
+// returns true with (xx, bb, ee) of the elected row, consuming it in its owner thread
+__device__ __forceinline__ bool twc_elect(TwcElect &el, unsigned &round, int x, uint32_t &b, uint32_t e, int &xx,
+                                          uint32_t &bb, uint32_t &ee) {
+    const int h = round & 1;
+    ++round;
+    const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
+    const bool big = e - b >= (uint32_t)kBlock;
+    const unsigned m = __ballot_sync(0xffffffffu, big);
+    if (m && (int)lane == __ffs(m) - 1) { el.cx[h][wid] = x; el.cb[h][wid] = b; el.ce[h][wid] = e; }
+    if (lane == 0) el.ball[h][wid] = m;
+    __syncthreads();
+    int w = -1;
+#pragma unroll
+    for (int k = kWarps - 1; k >= 0; --k) if (el.ball[h][k]) w = k;
+    if (w < 0) return false;
+    xx = el.cx[h][w]; bb = el.cb[h][w]; ee = el.ce[h][w];
+    if ((int)wid == w && (int)lane == __ffs(el.ball[h][w]) - 1) b = e;    // consumed by its owner
+    return true;
+}
 struct TwcSmem {
-    int owner, x;
-    uint32_t b, e;
+    TwcElect el;
 };
 template <class Src, class Op>
 __device__ __noinline__ LocalCnt lb_twc(const Src src, const Adj g, Op op, TwcSmem *sm) {
@@ -128,6 +157,7 @@ __device__ __noinline__ LocalCnt lb_twc(const Src src, const Adj g, Op op, TwcSm
     const unsigned sz = src.size();
     const unsigned lane = lane_id();
     constexpr int kTile = kBlock * kIlp;
+    unsigned round = 0;
     for (long long base = (long long)blockIdx.x * kTile; base < sz; base += (long long)gridDim.x * kTile) {
         int x[kIlp];
         uint32_t b[kIlp], e[kIlp];
@@ -147,16 +177,9 @@ __device__ __noinline__ LocalCnt lb_twc(const Src src, const Adj g, Op op, TwcSm
 #pragma unroll
         for (int j = 0; j < kIlp; ++j) {
             for (;;) {
-                if (threadIdx.x == 0) sm->owner = -1;
-                __syncthreads();
-                if (e[j] - b[j] >= (uint32_t)kBlock) sm->owner = threadIdx.x;
-                __syncthreads();
-                int owner = sm->owner;
-                if (owner < 0) break;
-                if ((int)threadIdx.x == owner) { sm->x = x[j]; sm->b = b[j]; sm->e = e[j]; e[j] = b[j]; }
-                __syncthreads();
-                const int xx = sm->x;
-                const uint32_t bb = sm->b, ee = sm->e;
+                int xx;
+                uint32_t bb, ee;
+                if (!twc_elect(sm->el, round, x[j], b[j], e[j], xx, bb, ee)) break;
                 for (uint32_t k0 = bb; k0 < ee; k0 += 2 * kBlock) {
                     int xs[2] = {xx, xx};
                     uint32_t ks[2] = {k0 + threadIdx.x, k0 + kBlock + threadIdx.x};

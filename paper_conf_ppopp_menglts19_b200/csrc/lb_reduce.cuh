@@ -142,8 +142,7 @@ __device__ __noinline__ LocalCnt lbr_thread(const Src src, const Adj g, Op op) {
 
 // ------------------------------------------------------------------ TWC (owner tiers)
 struct TwcRedSmem {
-    int owner, x;
-    uint32_t b, e;
+    TwcElect el;                     // lb.cuh: race-free CTA-tier election
     unsigned long long part[kWarps];
 };
 template <class Src, class Op>
@@ -154,6 +153,7 @@ __device__ __noinline__ LocalCnt lbr_twc(const Src src, const Adj g, Op op, TwcR
     const unsigned sz = src.size();
     const unsigned lane = lane_id(), wid = threadIdx.x >> 5;
     constexpr int kTile = kBlock * kIlp;
+    unsigned round = 0;
     for (long long base = (long long)blockIdx.x * kTile; base < sz; base += (long long)gridDim.x * kTile) {
         int x[kIlp];
         uint32_t b[kIlp], e[kIlp];
@@ -175,16 +175,9 @@ __device__ __noinline__ LocalCnt lbr_twc(const Src src, const Adj g, Op op, TwcR
 #pragma unroll
         for (int j = 0; j < kIlp; ++j) {
             for (;;) {
-                if (threadIdx.x == 0) sm->owner = -1;
-                __syncthreads();
-                if (e[j] - b[j] >= (uint32_t)kBlock) sm->owner = threadIdx.x;
-                __syncthreads();
-                const int owner = sm->owner;
-                if (owner < 0) break;
-                if ((int)threadIdx.x == owner) { sm->x = x[j]; sm->b = b[j]; sm->e = e[j]; e[j] = b[j]; }
-                __syncthreads();
-                const int xx = sm->x;
-                const uint32_t bb = sm->b, ee = sm->e;
+                int xx;
+                uint32_t bb, ee;
+                if (!twc_elect(sm->el, round, x[j], b[j], e[j], xx, bb, ee)) break;
                 Acc a = Op::identity();
                 for (uint32_t k0 = bb; k0 < ee; k0 += 2 * kBlock) {
                     uint32_t k[2] = {k0 + threadIdx.x, k0 + kBlock + threadIdx.x};

@@ -11,6 +11,7 @@ if ROOT not in sys.path:
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a B200 (sm_100a) and the built CUDA library")
     config.addinivalue_line("markers", "slow: large-size parity cases")
+    config.addinivalue_line("markers", "c5: the Kronecker scale-26 config (2.1e9 entries; minutes of host work)")
 
 
 def tiny_graphs():

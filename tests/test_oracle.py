@@ -385,3 +385,16 @@ def test_attrs_gini_mean_abs_difference():
     d = g.deg.astype(np.float64)
     mad = np.abs(d[:, None] - d[None, :]).sum() / (2 * len(d) ** 2 * d.mean())
     assert abs(oracle.attrs(g)["gini"] - mad) < 1e-12
+
+
+def test_pr_dpr_thread_count_invariant():
+    """oracle.c runs the per-vertex loops of PR / Delta-PR with OpenMP; each vertex's sum keeps
+    its ascending order, so 1 thread and all threads give bit-identical results."""
+    g = gen.rmat(13, seed=9)
+    res = []
+    for k in (1, 0):
+        oracle.set_threads(k)
+        res.append((oracle.pr(g, 0.85, 20), oracle.dpr(g, 0.85, 1e-7 * 0.15 / g.n)))
+    oracle.set_threads(0)
+    assert np.array_equal(res[0][0], res[1][0])
+    assert np.array_equal(res[0][1][0], res[1][1][0]) and res[0][1][1] == res[1][1][1]
