@@ -123,32 +123,39 @@ def build_graph(name):
 
 # --------------------------------------------------------------------------------------------
 def run_reference(args, ws, rank):
-    """--impl reference: the CPU oracle (plain single-threaded C) on the host cores."""
+    """--impl reference: the CPU oracle (plain single-threaded C) on the host cores, on the same
+    workload as this arm: C3 BFS at N = 1, the partitioned C5 BFS for N > 1 (rank 0 only; the
+    oracle holds the whole graph).  C5 steps are a bounded sample (2 roots, ~40 s each)."""
     if rank != 0:
         return
     import gen
     import oracle
-    g, _ = build_graph("C3")
+    c5 = (ws > 1 or args.partitioned) and not (args.dist_workload_forced and args.workload == "C3")
+    workload = "C5" if c5 else args.workload
+    g, _ = build_graph(workload)
     deg = g.deg
     roots = gen.sources(g, max(64, args.steps + args.warmup))
-    for k in range(args.warmup):
-        oracle.bfs(g, roots[k % len(roots)])
+    nsteps = min(args.steps, 2) if workload == "C5" else args.steps
+    if workload != "C5":
+        for k in range(args.warmup):
+            oracle.bfs(g, roots[k % len(roots)])
     edges, secs = 0, 0.0
-    for k in range(args.steps):
+    for k in range(nsteps):
         s = roots[(args.warmup + k) % len(roots)]
         t0 = time.perf_counter()
         d = oracle.bfs(g, s)
         secs += time.perf_counter() - t0
         edges += m_cc(deg, d)
     v = edges / secs / 1e9
+    scale = {"C3": 22, "C5": 26}.get(workload, 22)
     line = {"impl": "reference", "metric": "BFS GTEPS", "value": v, "unit": "GTEPS", "n_gpus": ws,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs * 1e3 / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs * 1e3 / nsteps,
+            "higher_is_better": True, "scaling": "strong" if c5 else "weak", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic",
-            "config": {"workload": "C3: BFS on R-MAT scale 22 ef 16 (Graph500 a,b,c=.57,.19,.19), roots per "
-                                   "SURVEY Q12", "parallelism": "single host thread"},
+            "config": {"workload": f"{workload}: BFS on R-MAT scale {scale} ef 16 (Graph500 a,b,c=.57,.19,.19), "
+                                   "roots per SURVEY Q12", "parallelism": "single host thread"},
             "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                             "sample": f"{args.steps} BFS roots, full graph, oracle.bfs (FIFO queue, 1 thread)"},
+                             "sample": f"{nsteps} BFS roots, full {workload} graph, oracle.bfs (FIFO queue, 1 thread)"},
             "e2e": {"value": v, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -223,68 +230,161 @@ def run_extras(gsw, dev, G3, g3, peak):
     return out
 
 
-def run_gsw_dist(args, ws, rank, local):
-    """N > 1: the C3 graph 1D vertex-partitioned over N ranks (one per GPU), BFS with per-level
-    NCCL bitmap all-gather + feature all-reduce inside the library (strong scaling: fixed graph)."""
+def dist_sources(gsw, off_local, vb, n, count, dev, seed=7):
+    """The SURVEY Q12 root stream (gen.sources) on a partitioned graph: candidate k is
+    splitmix64((seed << 32) | k) mod n; its owner says whether it has edges; repeats and
+    degree-0 vertices are skipped, as gen.sources does on the whole graph."""
     import torch
     import torch.distributed as dist
     import gen
+    ncand = 64 * count + 256
+    cand = [gen.splitmix64((seed << 32) | k) % n for k in range(ncand)]
+    deg = np.diff(off_local)
+    ok = torch.zeros(ncand, dtype=torch.int32, device=dev)
+    loc = [1 if vb <= v < vb + deg.size and deg[v - vb] > 0 else 0 for v in cand]
+    ok += torch.tensor(loc, dtype=torch.int32, device=dev)
+    if dist.is_initialized():
+        dist.all_reduce(ok, op=dist.ReduceOp.MAX)
+    ok = ok.cpu().numpy()
+    out, seen = [], set()
+    for v, good in zip(cand, ok):
+        if good and v not in seen:
+            seen.add(v)
+            out.append(int(v))
+            if len(out) == count:
+                break
+    return out
+
+
+def partition_input(workload, rank, ws):
+    """This rank's owned rows of the workload graph, generated directly (gen.rmat_slice)."""
+    import gen
+    import paper_conf_ppopp_menglts19_b200 as gsw
+    scale = {"C5": 26, "C3": 22}[workload]
+    n = 1 << scale
+    S = gsw.dist_slice(n, ws)
+    vb, ve = min(n, rank * S), min(n, (rank + 1) * S)
+    t0 = time.time()
+    off, col = gen.rmat_slice(scale, vb, ve, 16, seed=1)
+    return n, vb, off, col, time.time() - t0
+
+
+def run_gsw_dist(args, ws, rank, local):
+    """N > 1 (default): C5 (Kronecker scale 26) 1D vertex-partitioned over N ranks, one per GPU
+    (BASELINE config 5): BFS with the per-level NCCL bitmap all-gather + feature
+    all-reduce and device-side decisions, and PageRank with the fp32 contribution all-gather.
+    Strong scaling: the graph is fixed, each rank holds 1/N of it.  --partitioned runs the same at
+    N = 1 (NCCL with one rank)."""
+    import torch
+    import torch.distributed as dist
     import paper_conf_ppopp_menglts19_b200 as gsw
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if "RANK" not in os.environ:                       # --force-dist without torchrun
+    if "RANK" not in os.environ:
         os.environ.update(RANK="0", WORLD_SIZE="1", LOCAL_RANK="0", MASTER_ADDR="127.0.0.1",
                           MASTER_PORT=str(29500 + os.getpid() % 1000))
     dist.init_process_group("nccl", device_id=dev)
-    g, gen_s = build_graph("C3")
-    deg = g.deg
-    nroots = max(64, args.steps + args.warmup)
-    roots = gen.sources(g, nroots)
+    workload = args.workload if args.workload != "C3" or args.dist_workload_forced else "C5"
+    n, vb, off, col, gen_s = partition_input(workload, rank, ws)
+    nroots = args.steps + args.warmup
+    roots = dist_sources(gsw, off, vb, n, nroots, dev)
     obj = [gsw.dist_unique_id() if rank == 0 else None]
     dist.broadcast_object_list(obj, src=0)
-    off, col = gsw.owned_rows(g.off, g.col, rank, ws)
-    D = gsw.DistGraph(off, col, g.n, obj[0], ws, rank, device=dev)
-    S = gsw.dist_slice(g.n, ws)
-    out = torch.empty(D.out_len, dtype=torch.int32, device=dev)
+    t0 = time.time()
+    D = gsw.DistGraph(off, col, n, obj[0], ws, rank, device=dev)
+    create_s = time.time() - t0
+    deg = np.diff(off)
+    out = torch.empty(max(D.out_len, 1), dtype=torch.int32, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def mx(x):
+        t = torch.tensor([float(x)], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sm(x):
+        t = torch.tensor([float(x)], device=dev, dtype=torch.float64)
+        dist.all_reduce(t)
+        return float(t.item())
+
     for k in range(args.warmup):
-        D.bfs(roots[k % nroots], out=out)
+        D.bfs(roots[k], out=out)
     torch.cuda.synchronize()
     dist.barrier()
-    tot_ms, edges_cc, bytes_alg, launches = 0.0, 0, 0, 0
+    tot_ms, edges_cc, bytes_alg, levels = 0.0, 0, 0, 0
     with ClockSampler(local) as cs:
         for k in range(args.steps):
             flush.fill_(k & 0xff)
             torch.cuda.synchronize()
             dist.barrier()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(D.stream)
-            _, st = D.bfs(roots[(args.warmup + k) % nroots], out=out)
-            e1.record(D.stream)
-            torch.cuda.synchronize()
-            ms = torch.tensor([e0.elapsed_time(e1)], device=dev)
-            dist.all_reduce(ms, op=dist.ReduceOp.MAX)
-            tot_ms += float(ms.item())
-            bytes_alg += st["bytes_alg"]
-            launches += 3 * st["iterations"] + 4          # init + per level: expand, count-sum (+NCCL)
-            # m_cc from the owned slices (sum over ranks)
-            loc = torch.tensor([int(deg[rank * S:rank * S + D.out_len][out.cpu().numpy() >= 0].sum())], device=dev)
-            dist.all_reduce(loc)
-            edges_cc += int(loc.item()) // 2
+            _, st = D.bfs(roots[args.warmup + k], out=out)
+            tot_ms += mx(st["gpu_ms"])                   # device span of the call, slowest rank
+            bytes_alg += st["bytes_alg"]                 # global (same on every rank)
+            levels += st["iterations"]
+            d = out[:D.out_len].cpu().numpy()
+            edges_cc += int(sm(int(deg[d >= 0].sum()))) // 2
+    value = edges_cc / (tot_ms * 1e-3) / 1e9
+    # PageRank, 20 iterations (d = 0.85), best of 2
+    pr_ms = None
+    for _ in range(2):
+        flush.fill_(1)
+        torch.cuda.synchronize()
+        dist.barrier()
+        _, st = D.pr(0.85, 20)
+        t = mx(st["gpu_ms"])
+        pr_ms = t if pr_ms is None else min(pr_ms, t)
+    pr_bytes = st["bytes_alg"]
     peak, peak_src = hbm_peak()
+    per_gpu_gbs = bytes_alg / ws / (tot_ms * 1e-3) / 1e9
+    # e2e: owned CSR from pinned host memory -> DistGraph (H2D + slice build) -> BFS into pinned host
+    pin_off = torch.from_numpy(off).pin_memory()
+    pin_col = torch.from_numpy(col).pin_memory()
+    host_out = torch.empty(max(D.out_len, 1), dtype=torch.int32).pin_memory()
+    del D
+    torch.cuda.empty_cache()
+    e2e_ms, e2e_edges = 0.0, 0
+    ke = 2
+    for k in range(ke):
+        dist.barrier()
+        t0 = time.perf_counter()
+        D2 = gsw.DistGraph(pin_off, pin_col, n, obj[0], ws, rank, device=dev)
+        D2.bfs(roots[args.warmup + k], out=host_out)
+        e2e_ms += mx((time.perf_counter() - t0) * 1e3)
+        e2e_edges += int(sm(int(deg[host_out.numpy()[:D2.out_len] >= 0].sum()))) // 2
+        del D2
+        torch.cuda.empty_cache()
+    h2d_all = sm(off.nbytes + col.nbytes)           # collectives on every rank, before the rank-0 print
+    d2h_all = sm(4 * max(1, len(host_out)))
     if rank == 0:
+        launches_per_level = 4                      # push, push_heavy, pull, decide (+ NCCL kernels)
         line = {
-            "metric": "BFS GTEPS", "value": edges_cc / (tot_ms * 1e-3) / 1e9, "unit": "GTEPS", "n_gpus": ws,
+            "metric": "BFS GTEPS", "value": value, "unit": "GTEPS", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": f"C3: BFS on R-MAT scale 22 ef 16, n={g.n}, nnz={g.nnz}, 1D vertex partition "
-                                   f"over {ws} ranks (slice {S}), per-level NCCL bitmap all-gather",
-                       "l2": "flushed between steps", "parallelism": f"1D vertex partition x{ws} (NCCL)"},
-            "roofline": {"bound": "hbm", "achieved": bytes_alg / (tot_ms * 1e-3) / 1e9 / ws, "peak": peak,
-                         "unit": "GB/s", "frac": bytes_alg / (tot_ms * 1e-3) / 1e9 / ws / peak, "traffic": None,
-                         "peak_source": peak_src, "kernel": "gsw k_bfs_push/k_bfs_pull (per level) + NCCL"},
-            "gpu_launches": launches, "clocks": cs.summary(), "gen_seconds": gen_s,
+            "config": {"workload": f"{workload}: BFS on R-MAT/Kronecker scale {26 if workload == 'C5' else 22} ef 16 "
+                                   f"(Graph500 a,b,c=.57,.19,.19), n={n}, 1D vertex partition over {ws} ranks "
+                                   f"(slice {gsw.dist_slice(n, ws)}), per-level NCCL bitmap all-gather, roots per "
+                                   "SURVEY Q12",
+                       "l2": "flushed between steps (256 MiB write outside the timed span)",
+                       "parallelism": f"1D vertex partition x{ws} (NCCL over NVLink)"},
+            "roofline": {"bound": "hbm", "achieved": per_gpu_gbs, "peak": peak, "unit": "GB/s",
+                         "frac": sane_frac(per_gpu_gbs / peak, "dist BFS"), "traffic": None,
+                         "peak_source": peak_src,
+                         "kernel": "gsw k_bfs_push/k_bfs_pull per level (+ NCCL all-gather), per GPU",
+                         "bytes_model": "SURVEY 8(d) D0 per-level algorithmic bytes, summed over ranks / N"},
+            "gpu_launches": launches_per_level * (levels + 3 * args.steps) + 3 * args.steps,
+            "timing": "device span of each gsw_bfs call on the library stream (CUDA events), max over ranks",
+            "e2e": {"value": e2e_edges / (e2e_ms * 1e-3) / 1e9, "unit": "GTEPS",
+                    "h2d_bytes_per_step": int(h2d_all), "d2h_bytes_per_step": int(d2h_all),
+                    "note": "per step, every rank: gsw_graph_create_dist from its pinned host slice (H2D + column-"
+                            "slice build) + gsw_bfs into pinned host depth (D2H); bytes summed over ranks; host wall "
+                            "clock of the slowest rank"},
+            "clocks": cs.summary(), "gen_seconds": gen_s, "create_seconds": create_s,
+            "extra": {f"{workload}_pr": {"value": 20 / (pr_ms * 1e-3), "unit": "PR iters/s", "gpu_ms": pr_ms,
+                                         "achieved_gbs_per_gpu": pr_bytes / (pr_ms * 1e-3) / 1e9,
+                                         "bytes_model": "4*nnz_owned + 8*n_owned + 4*N (fp32 all-gather) per "
+                                                        "iteration and rank"}},
         }
         print(json.dumps(line), flush=True)
     dist.barrier()
@@ -297,7 +397,7 @@ def run_gsw(args, ws, rank, local):
     import gen
     import paper_conf_ppopp_menglts19_b200 as gsw
 
-    if args.partitioned or args.force_dist:
+    if args.partitioned or args.force_dist or (ws > 1 and not args.replicas):
         return run_gsw_dist(args, ws, rank, local)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -456,9 +556,11 @@ def main():
                     help="C3 (default, the north_star's headline) or C5 (R-MAT scale 26, 1 GPU)")
     ap.add_argument("--force-dist", action="store_true", help="run the partitioned NCCL path even at N=1")
     ap.add_argument("--partitioned", action="store_true",
-                    help="N > 1: the 1D vertex-partitioned graph with per-level NCCL exchange (SURVEY 8(e))")
-    ap.add_argument("--replicas", action="store_true", help="exercise the root-sharded replica path at N=1")
+                    help="the 1D vertex-partitioned graph with NCCL exchange (SURVEY 8(e)); default for N > 1")
+    ap.add_argument("--replicas", action="store_true",
+                    help="N > 1: root-sharded replicas of C3 instead of the partitioned C5 (or exercise them at N=1)")
     args = ap.parse_args()
+    args.dist_workload_forced = "--workload" in sys.argv
     if args.warmup < 3:
         args.warmup = 3
     ws, rank, local = dist_env()

@@ -185,15 +185,26 @@ gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc,
 /* ---------------------------------------------------------------------------------------------
  * Multi-GPU: 1D vertex partition (the paper itself is single-GPU).  Rank r of p owns
  * the vertex slice [r*S, min(n,(r+1)*S)) with S = gsw_dist_slice(n, p) (a multiple of 64, equal
- * for every rank as NCCL collectives need equal counts).  Every write lands on an owned vertex, so
- * no cross-GPU atomics are needed.  Per BFS level a rank expands into its owned slice of the next
- * frontier bitmap (pull: owned rows = in-edges of owned vertices; push: the column slice "global
- * source -> owned targets" built at create time), then an in-place ncclAllGather of the bitmap
- * slices (n/8 bytes total) and an ncclAllReduce of the 16-byte feature counts give every rank the
- * same frontier and the same selector decision.  PageRank all-gathers the fp64 contributions and
- * all-reduces the dangling mass each iteration.  NCCL is loaded at run time (dlopen); without it
- * the NCCL calls return GSW_ENCCL.  Supported on distributed handles: gsw_bfs, gsw_pr (others
- * return GSW_EUNSUPPORTED).  Outputs of distributed handles cover the OWNED slice only.
+ * for every rank as collectives need equal counts).  Every write lands on an owned vertex, so no
+ * cross-GPU atomics are needed.
+ *   BFS level: the rank expands into its owned slice of the next frontier bitmap (push: the
+ *     column slice "global source -> owned targets" built at create; pull: the owned rows, i.e.
+ *     in-edges of owned vertices, with early exit), then an in-place all-gather of the bitmap
+ *     slices (n/8 bytes) and an all-reduce of (Va, Ea, edges) give every rank the same frontier;
+ *     a device kernel on every rank evaluates the same direction rule on those global counts.
+ *   PageRank iteration: owned rows pull the replicated fp32 contributions pr/deg; all-gather of
+ *     the contribution slices (n*4 bytes) + all-reduce of the dangling mass.
+ *   CC iteration: min-label propagation with the pointer-jumping shortcut label[label[v]] on the
+ *     replicated labels; all-gather of the label slices + all-reduce of the change count.
+ * The host never waits per iteration (NCCL / loopback): it polls the device's done flag two
+ * iterations behind the stream.  Supported on distributed handles: gsw_bfs, gsw_pr, gsw_cc
+ * (others return GSW_EUNSUPPORTED); gsw_force_config's direction pins the BFS direction.
+ * Outputs of NCCL / host-staged handles cover the OWNED slice only; loopback outputs all n.
+ * Three exchange backends run the same kernels:
+ *   NCCL (one process per GPU; NCCL is dlopen'ed, a missing library gives GSW_ENCCL),
+ *   loopback (p virtual ranks on one GPU, exchange = the shared replicated buffers),
+ *   host-staged (caller callbacks, e.g. torch.distributed over gloo; several processes may share
+ *     a GPU; one host round trip per exchange).
  * ------------------------------------------------------------------------------------------- */
 /* Slice size S for n vertices over p ranks. */
 int64_t gsw_dist_slice(int64_t n, int32_t nranks);
@@ -203,11 +214,28 @@ gsw_status gsw_dist_unique_id(void *id128);
 gsw_status gsw_dist_workspace_size(int64_t n_global, int64_t nnz_owned, int32_t nranks, size_t *bytes);
 /* NCCL mode (one process per GPU).  owned: the rows of the owned slice -- owned->n = number of
  * owned vertices, row_offsets start at 0, col_indices are GLOBAL ids (symmetric graph).
- * Collective over all ranks (same call order on every rank).  Errors: GSW_EINVAL (slice size
- * mismatch), GSW_ENCCL (communicator creation failed). */
+ * nccl_id128 may be NULL only when nranks == 1 (a private communicator is created; the
+ * collectives still run).  Collective over all ranks (same call order on every rank).
+ * Errors: GSW_EINVAL (slice size mismatch), GSW_ENCCL (communicator creation failed). */
 gsw_status gsw_graph_create_dist(const gsw_csr *owned, int64_t n_global, const void *nccl_id128,
                                  int32_t nranks, int32_t rank, void *workspace, size_t ws_bytes,
                                  void *cuda_stream, gsw_graph *out);
+/* Host-staged exchange: the library copies its slice / counters to pinned host memory, calls
+ * these callbacks (every rank in the same order, like a collective), and copies the result back.
+ * Each returns 0 on success.
+ *   allgather(user, send, recv, bytes): recv (nranks*bytes) = every rank's send, in rank order;
+ *   allreduce_u64 / allreduce_f64(user, buf, count): in-place element-wise sum over the ranks. */
+typedef struct {
+    void *user;
+    int (*allgather)(void *user, const void *send, void *recv, size_t bytes);
+    int (*allreduce_u64)(void *user, uint64_t *buf, size_t count);
+    int (*allreduce_f64)(void *user, double *buf, size_t count);
+} gsw_exchange;
+/* Same arguments as gsw_graph_create_dist (workspace: gsw_dist_workspace_size), exchange through
+ * `exchange` (copied; its function pointers must stay valid until gsw_graph_destroy). */
+gsw_status gsw_graph_create_dist_host(const gsw_csr *owned, int64_t n_global, const gsw_exchange *exchange,
+                                      int32_t nranks, int32_t rank, void *workspace, size_t ws_bytes,
+                                      void *cuda_stream, gsw_graph *out);
 /* Loopback mode: `nparts` virtual ranks of the full symmetric graph on THIS GPU, exchanging
  * through device memory in stream order (the same partitioned kernels as NCCL mode; used to test
  * the partitioned path on one GPU).  Outputs cover all n vertices. */

@@ -20,7 +20,8 @@ from ._lib import (AUTO, BITMAP, DIRECTIONS, FORMATS, FUSED, FUSIONS, LB_CM, LB_
                    LB_THREAD, LB_TWC, LB_WM, LOAD_BALANCES, PULL, PUSH, QUEUE, SORTED_QUEUE, STANDALONE,
                    STEPPINGS, GswError, check)
 
-__all__ = ["Graph", "GswError", "version", "force_config_struct"]
+__all__ = ["Graph", "GswError", "version", "force_config_struct", "DistGraph", "HostDistGraph",
+           "TorchHostExchange", "PartitionedGraph", "dist_slice", "dist_unique_id", "owned_rows"]
 
 
 def version() -> str:
@@ -204,8 +205,8 @@ class Graph:
 
 
 # ------------------------------------------------------------------------------------------------
-# Multi-GPU: 1D vertex partition (include/gsw.h "Multi-GPU").  BFS and PageRank run on these
-# handles; outputs cover the owned slice (NCCL mode) or all vertices (loopback mode).
+# Multi-GPU: 1D vertex partition (include/gsw.h "Multi-GPU").  BFS, PageRank and CC run on these
+# handles; outputs cover the owned slice (NCCL / host-staged mode) or all vertices (loopback).
 
 def dist_slice(n: int, nranks: int) -> int:
     """Slice size S: rank r owns vertices [r*S, min(n, (r+1)*S))."""
@@ -255,6 +256,82 @@ class DistGraph(_Handle):
             check(lib.gsw_graph_create_dist(ctypes.byref(csr), self.n, idbuf, self.nranks, self.rank,
                                             self.workspace.data_ptr(), nbytes.value, self.stream.cuda_stream,
                                             ctypes.byref(h)), "gsw_graph_create_dist")
+            self._h = h
+            del ko, kc
+
+
+class TorchHostExchange:
+    """Host-staged exchange (gsw_exchange) over a torch.distributed process group -- typically
+    gloo, so several processes can share one GPU in tests.  Marshalling only: the callbacks move
+    the library's pinned host buffers through the group's all_gather / all_reduce."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist, self.group = dist, group
+        self.nranks = dist.get_world_size(group)
+
+        def allgather(_user, send, recv, nbytes):
+            try:
+                import torch
+                src = torch.from_numpy(np.ctypeslib.as_array(ctypes.cast(send, ctypes.POINTER(ctypes.c_uint8)),
+                                                             shape=(nbytes,)).copy())
+                outs = [torch.empty_like(src) for _ in range(self.nranks)]
+                self.dist.all_gather(outs, src, group=self.group)
+                dst = np.ctypeslib.as_array(ctypes.cast(recv, ctypes.POINTER(ctypes.c_uint8)),
+                                            shape=(nbytes * self.nranks,))
+                dst[:] = torch.cat(outs).numpy()
+                return 0
+            except Exception:                     # noqa: BLE001 -- reported to the library as failure
+                return 1
+
+        def allreduce(ctype, np_dtype):
+            def fn(_user, buf, count):
+                try:
+                    import torch
+                    arr = np.ctypeslib.as_array(buf, shape=(count,))
+                    t = torch.from_numpy(arr.astype(np_dtype))
+                    self.dist.all_reduce(t, group=self.group)
+                    arr[:] = t.numpy()
+                    return 0
+                except Exception:                 # noqa: BLE001
+                    return 1
+            return fn
+
+        self._fns = (_lib.ALLGATHER_FN(allgather), _lib.ALLREDUCE_U64_FN(allreduce(ctypes.c_uint64, np.int64)),
+                     _lib.ALLREDUCE_F64_FN(allreduce(ctypes.c_double, np.float64)))
+        self.struct = _lib.gsw_exchange(None, *self._fns)
+
+
+class HostDistGraph(_Handle):
+    """Host-staged mode: like DistGraph, but the per-iteration exchange goes through `exchange`
+    (a TorchHostExchange) instead of NCCL.  The kernels are the same partitioned kernels."""
+
+    def __init__(self, owned_offsets, owned_cols, n_global: int, exchange: "TorchHostExchange", rank: int,
+                 device: str | int = "cuda", stream=None):
+        import torch
+        lib = _lib.load()
+        self.device = torch.device(device)
+        off = _as(owned_offsets, np.int64, torch.int64)
+        col = _as(owned_cols, np.int32, torch.int32)
+        self.n = int(n_global)
+        self.out_len = int(off.shape[0]) - 1
+        self.nnz = int(col.shape[0])
+        self.rank, self.nranks = int(rank), exchange.nranks
+        self._exchange = exchange                 # keeps the callbacks alive
+        with torch.cuda.device(self.device):
+            self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+            po, ko, _ = _ptr_of(off)
+            pc, kc, _ = _ptr_of(col) if self.nnz else (None, None, False)
+            csr = _lib.gsw_csr(self.out_len, self.nnz, po, pc, None)
+            nbytes = ctypes.c_size_t()
+            check(lib.gsw_dist_workspace_size(self.n, self.nnz, self.nranks, ctypes.byref(nbytes)),
+                  "gsw_dist_workspace_size")
+            self.workspace = torch.empty(nbytes.value, dtype=torch.uint8, device=self.device)
+            h = ctypes.c_void_p()
+            check(lib.gsw_graph_create_dist_host(ctypes.byref(csr), self.n, ctypes.byref(exchange.struct),
+                                                 self.nranks, self.rank, self.workspace.data_ptr(), nbytes.value,
+                                                 self.stream.cuda_stream, ctypes.byref(h)),
+                  "gsw_graph_create_dist_host")
             self._h = h
             del ko, kc
 

@@ -57,6 +57,17 @@ class gsw_run_stats(ctypes.Structure):
 
 # every symbol include/gsw.h declares: name -> (restype, argtypes)
 _P = ctypes.c_void_p
+# host-staged exchange callbacks (include/gsw.h gsw_exchange)
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, _P, _P, _P, ctypes.c_size_t)
+ALLREDUCE_U64_FN = ctypes.CFUNCTYPE(ctypes.c_int, _P, ctypes.POINTER(ctypes.c_uint64), ctypes.c_size_t)
+ALLREDUCE_F64_FN = ctypes.CFUNCTYPE(ctypes.c_int, _P, ctypes.POINTER(ctypes.c_double), ctypes.c_size_t)
+
+
+class gsw_exchange(ctypes.Structure):
+    _fields_ = [("user", _P), ("allgather", ALLGATHER_FN), ("allreduce_u64", ALLREDUCE_U64_FN),
+                ("allreduce_f64", ALLREDUCE_F64_FN)]
+
+
 SIGNATURES = {
     "gsw_workspace_size": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                           ctypes.POINTER(ctypes.c_size_t)]),
@@ -78,6 +89,9 @@ SIGNATURES = {
                                                ctypes.POINTER(ctypes.c_size_t)]),
     "gsw_graph_create_dist": (ctypes.c_int, [ctypes.POINTER(gsw_csr), ctypes.c_int64, _P, ctypes.c_int32,
                                              ctypes.c_int32, _P, ctypes.c_size_t, _P, ctypes.POINTER(_P)]),
+    "gsw_graph_create_dist_host": (ctypes.c_int, [ctypes.POINTER(gsw_csr), ctypes.c_int64,
+                                                  ctypes.POINTER(gsw_exchange), ctypes.c_int32, ctypes.c_int32, _P,
+                                                  ctypes.c_size_t, _P, ctypes.POINTER(_P)]),
     "gsw_dist_loopback_workspace_size": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32,
                                                         ctypes.POINTER(ctypes.c_size_t)]),
     "gsw_graph_create_partitioned": (ctypes.c_int, [ctypes.POINTER(gsw_csr), ctypes.c_int32, _P, ctypes.c_size_t,

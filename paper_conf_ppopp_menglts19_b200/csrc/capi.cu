@@ -28,12 +28,14 @@ gsw_status relabel_graph(gsw_graph g, uint32_t *perm, uint32_t *inv, char *tmp, 
 gsw_status build_first_nbr(gsw_graph g, int32_t *first);
 // dist.cu
 int64_t dist_slice(int64_t n, int32_t p);
-gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int32_t nranks, int32_t rank,
-                       bool loopback, void *workspace, size_t ws_bytes, void *stream, gsw_graph *out);
+gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, const gsw_exchange *hx, int32_t nranks,
+                       int32_t rank, int mode, void *workspace, size_t ws_bytes, void *stream, gsw_graph *out);
 void dist_destroy(DistState *d);
 gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stats *st);
 gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out, gsw_run_stats *st);
-size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, bool own_copy);
+gsw_status dist_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st);
+size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, int mode);
+enum { kModeNccl = 0, kModeLoopback = 1, kModeHost = 2 };   // dist.cu DistMode
 gsw_status dist_unique_id(void *id128);
 
 static gsw_status no_dist(gsw_graph g, const char *what) {
@@ -200,7 +202,7 @@ gsw_status gsw_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *
 
 gsw_status gsw_cc(gsw_graph g, int32_t *label, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
-    if (gsw_status s = no_dist(g, "gsw_cc")) return s;
+    if (g->dist) return dist_cc(g, label, stats);
     return run_cc(g, label, stats);
 }
 
@@ -228,13 +230,13 @@ gsw_status gsw_dist_unique_id(void *id128) { return dist_unique_id(id128); }
 
 gsw_status gsw_dist_workspace_size(int64_t n_global, int64_t nnz_owned, int32_t nranks, size_t *bytes) {
     if (!bytes || n_global <= 0 || nnz_owned < 0 || nranks < 1) { set_error("gsw_dist_workspace_size: bad arguments"); return GSW_EINVAL; }
-    *bytes = dist_workspace(n_global, nnz_owned, nranks, 1, true);
+    *bytes = dist_workspace(n_global, nnz_owned, nranks, 1, kModeNccl);
     return GSW_OK;
 }
 
 gsw_status gsw_dist_loopback_workspace_size(int64_t n, int64_t nnz, int32_t nparts, size_t *bytes) {
     if (!bytes || n <= 0 || nnz < 0 || nparts < 1) { set_error("gsw_dist_loopback_workspace_size: bad arguments"); return GSW_EINVAL; }
-    *bytes = dist_workspace(n, nnz, nparts, nparts, false);
+    *bytes = dist_workspace(n, nnz, nparts, nparts, kModeLoopback);
     return GSW_OK;
 }
 
@@ -242,13 +244,27 @@ gsw_status gsw_graph_create_dist(const gsw_csr *owned, int64_t n_global, const v
                                  int32_t rank, void *workspace, size_t ws_bytes, void *cuda_stream, gsw_graph *out) {
     if (!out) { set_error("out is NULL"); return GSW_EINVAL; }
     if (nranks > 1 && !nccl_id128) { set_error("nccl_id128 is NULL"); return GSW_EINVAL; }
-    return dist_create(owned, n_global, nccl_id128, nranks, rank, false, workspace, ws_bytes, cuda_stream, out);
+    unsigned char own_id[128];
+    if (!nccl_id128) {                      // one rank: a private communicator, the collectives still run
+        if (gsw_status s = dist_unique_id(own_id)) return s;
+        nccl_id128 = own_id;
+    }
+    return dist_create(owned, n_global, nccl_id128, nullptr, nranks, rank, kModeNccl, workspace, ws_bytes, cuda_stream,
+                       out);
+}
+
+gsw_status gsw_graph_create_dist_host(const gsw_csr *owned, int64_t n_global, const gsw_exchange *exchange,
+                                      int32_t nranks, int32_t rank, void *workspace, size_t ws_bytes,
+                                      void *cuda_stream, gsw_graph *out) {
+    if (!out || !exchange) { set_error("null argument"); return GSW_EINVAL; }
+    return dist_create(owned, n_global, nullptr, exchange, nranks, rank, kModeHost, workspace, ws_bytes, cuda_stream,
+                       out);
 }
 
 gsw_status gsw_graph_create_partitioned(const gsw_csr *csr, int32_t nparts, void *workspace, size_t ws_bytes,
                                         void *cuda_stream, gsw_graph *out) {
     if (!out || !csr) { set_error("null argument"); return GSW_EINVAL; }
-    return dist_create(csr, csr->n, nullptr, nparts, 0, true, workspace, ws_bytes, cuda_stream, out);
+    return dist_create(csr, csr->n, nullptr, nullptr, nparts, 0, kModeLoopback, workspace, ws_bytes, cuda_stream, out);
 }
 
 }  // extern "C"

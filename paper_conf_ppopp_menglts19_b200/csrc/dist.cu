@@ -1,15 +1,36 @@
-// dist.cu -- multi-GPU frontier step: 1D vertex partition with destination
-// ownership, frontier-bitmap all-gather and feature all-reduce over NCCL (NVLink 5 / NVSwitch),
-// plus a loopback mode that runs p virtual ranks on one GPU through the same partitioned kernels.
+// dist.cu -- multi-GPU frontier step (the paper itself is single-GPU): 1D vertex
+// partition with destination ownership, the per-iteration exchange over NCCL (NVLink 5 /
+// NVSwitch), and two more exchange backends that run the SAME partitioned kernels: loopback (p
+// virtual ranks on one GPU, exchange = the shared replicated buffers) and host-staged (the caller
+// supplies all-gather / all-reduce callbacks, e.g. torch.distributed over gloo, so several
+// processes can share one GPU in tests).
 //
-// BFS level t (every rank):  [host] same direction rule as the single-GPU selector on the GLOBAL
-//   features -> [kernel] push: for every frontier vertex u (replicated bitmap FB_t), walk the
-//   column slice u -> owned targets and claim them; pull: for every owned unvisited v, scan its row
-//   (global in-neighbours) until a frontier bit is found -> each rank writes only its slice of
-//   FB_{t+1} -> [NCCL] in-place AllGather of the slices (n/8 bytes) + AllReduce of (Va, Ea, edges)
-//   -> [host] read the 24-byte totals (termination, next decision).
-// PR iteration: owned rows pull the replicated fp64 contributions, each rank writes its slice of
-//   the next contributions, AllGather + AllReduce(dangling mass) on the stream (no host sync).
+// Device-resident decisions.  The per-iteration control state (global counts, unvisited counts,
+// the next direction, the done flag, per-level records) lives in device memory: every rank's
+// `decide` kernel evaluates the same selector rule on the same all-reduced counts, and both
+// expand kernels of a level are launched, the one not chosen returning at once.  The host only
+// enqueues: it polls the done flag LOOKAHEAD levels behind the stream (pinned copy + event), so
+// the stream never drains between levels; the at most LOOKAHEAD no-op levels that follow the last
+// one cost a launch and (NCCL) an all-gather each.  Every rank stops after the same number of
+// enqueued levels, because the flag it polls is computed from all-reduced values.
+//
+// BFS level t (every rank / part):
+//   push  k_bfs_push: every frontier vertex u of the replicated bitmap FB_t walks its column-slice
+//         row "u -> owned targets" (built at create): a lane per short row, the warp for rows up
+//         to kHeavy edges, 1024-edge tasks (k_bfs_push_heavy) above; claims by atomicOr on the
+//         owned visited map; the rank's slice of FB_{t+1} is marked.
+//   pull  k_bfs_pull: the single-GPU list pull (bfs_pull.cuh) over the owned unvisited vertices:
+//         first in-neighbour probe, then cursors over the misses; early exit at the first parent.
+//   exchange: in-place all-gather of the FB_{t+1} slices (N/8 bytes) + all-reduce of (Va, Ea,
+//         edges) -> k_bfs_decide (Via/Eia, direction rule of select.cuh R6, records, done).
+// PageRank iteration (every vertex active): owned rows pull the replicated fp32
+//   contributions (rows above kHeavy edges as 1024-edge chunk tasks with fp64 partials), each rank
+//   writes its slice of the next contributions; all-gather (fp32, N*4 bytes) + all-reduce of the
+//   dangling mass.  Fixed iteration count: no host poll at all.
+// CC iteration (min-label propagation, DESIGN R8, with the pointer-jumping shortcut
+//   label[v] <- label[label[v]] that the replicated labels make local; Soman et al. [53]
+//   P:1429-1430): owned rows pull the replicated labels, each rank writes its slice; all-gather
+//   (N*4 bytes) + all-reduce of the change count -> k_cc_decide (done when nothing changed).
 #include <dlfcn.h>
 
 #include <algorithm>
@@ -20,6 +41,7 @@
 #include <cub/device/device_scan.cuh>
 #include <nccl.h>
 
+#include "bfs_pull.cuh"
 #include "launch.h"
 
 namespace gsw {
@@ -32,6 +54,8 @@ struct NcclApi {
     decltype(&ncclCommDestroy) commDestroy = nullptr;
     decltype(&ncclAllGather) allGather = nullptr;
     decltype(&ncclAllReduce) allReduce = nullptr;
+    decltype(&ncclGroupStart) groupStart = nullptr;
+    decltype(&ncclGroupEnd) groupEnd = nullptr;
     decltype(&ncclGetErrorString) errStr = nullptr;
 };
 static NcclApi g_nccl;
@@ -51,9 +75,11 @@ static bool nccl_load() {
     g_nccl.commDestroy = (decltype(g_nccl.commDestroy))dlsym(h, "ncclCommDestroy");
     g_nccl.allGather = (decltype(g_nccl.allGather))dlsym(h, "ncclAllGather");
     g_nccl.allReduce = (decltype(g_nccl.allReduce))dlsym(h, "ncclAllReduce");
+    g_nccl.groupStart = (decltype(g_nccl.groupStart))dlsym(h, "ncclGroupStart");
+    g_nccl.groupEnd = (decltype(g_nccl.groupEnd))dlsym(h, "ncclGroupEnd");
     g_nccl.errStr = (decltype(g_nccl.errStr))dlsym(h, "ncclGetErrorString");
     g_nccl.ok = g_nccl.getUniqueId && g_nccl.commInitRank && g_nccl.commDestroy && g_nccl.allGather &&
-                g_nccl.allReduce && g_nccl.errStr;
+                g_nccl.allReduce && g_nccl.groupStart && g_nccl.groupEnd && g_nccl.errStr;
     if (!g_nccl.ok) set_error("NCCL symbols missing");
     return g_nccl.ok;
 }
@@ -68,27 +94,70 @@ static bool nccl_load() {
     } while (0)
 
 // ------------------------------------------------------------------ partition state
+enum DistMode { DM_NCCL = 0, DM_LOOPBACK = 1, DM_HOST = 2 };
+
+constexpr uint32_t kHeavy = 1024;      // rows above this many edges become 1024-edge warp tasks
+constexpr int kMaxLevels = 1 << 16;    // per-level records kept on the device
+constexpr int kLookahead = 2;          // levels enqueued past the one whose done flag is polled
+
+struct DTask {
+    int row;
+    uint32_t beg, end;
+};
+
+// per-level record on the device (host converts it to gsw_iter_record)
+struct DRec {
+    long long Va, Ea, Via, Eia, edges;
+    int dir, pad;
+};
+
+// control block (device): identical on every rank after each decide
+struct DCtl {
+    unsigned long long tot[4];     // all-reduced {va, ea, edges, changes}
+    double dtot;                   // all-reduced f64 (PR dangling mass)
+    double pad0;
+    long long Via, Eia, nnz_g;     // unvisited vertices / their edges, global nnz
+    int dir, done, t, pad1;
+};
+
+// per-part counters, 64 B apart: {va, ea, edges, changes, f64 bits, -, -, -}
+constexpr int kLocStride = 8;
+
 struct DPart {
     int64_t vb = 0;           // first owned vertex (multiple of 64)
     int nloc = 0;             // owned vertices
     uint32_t nnz = 0;         // owned adjacency entries
     uint32_t *roff = nullptr; // nloc+1, rebased to 0
     const int32_t *rcol = nullptr;   // global neighbour ids
+    int32_t *rfirst = nullptr;// first in-neighbour of each owned row (-1: empty)
     uint32_t *soff = nullptr; // n_global+1: global source u -> owned targets
     int32_t *scol = nullptr;  // local target ids
     unsigned *vis = nullptr;  // visited words of the owned slice (S/32)
+    DTask *chunks = nullptr;  // heavy owned rows cut into kHeavy-edge chunks (create time)
+    unsigned *nchunks = nullptr;
+    DTask *ptasks = nullptr;  // push tasks of the current level
+    unsigned *nptasks = nullptr;
+    uint32_t ptask_cap = 0;
+    double *psum = nullptr;   // heavy-row partials (PR sums / CC minima as u32), nloc entries
+    unsigned long long *loc = nullptr;   // this part's counters (kLocStride u64)
 };
 
 struct DistState {
+    int mode = DM_NCCL;
     int nranks = 1, rank = 0;
-    bool loopback = false;
     int64_t n = 0, S = 0, npad = 0;
     std::vector<DPart> parts;
     unsigned *FB[2] = {nullptr, nullptr};   // replicated frontier bitmaps, npad/32 words
-    double *contrib[2] = {nullptr, nullptr};// replicated PR contributions, npad entries
-    unsigned long long *cnt = nullptr;      // per part {va, ea, edges}, then the totals
-    double *dang = nullptr;                 // per part dangling mass, then the total
+    uint32_t *rep[2] = {nullptr, nullptr};  // replicated per-vertex words: fp32 contributions / labels
+    unsigned long long *locs = nullptr;     // parts x kLocStride
+    DCtl *ctl = nullptr;
+    DRec *recs = nullptr;
     ncclComm_t comm = nullptr;
+    gsw_exchange hx{};                      // host-staged backend callbacks
+    unsigned char *hsend = nullptr, *hrecv = nullptr;   // pinned staging (host mode)
+    size_t hcap = 0;
+    int *hdone = nullptr;                   // pinned done flags, one per lookahead slot
+    cudaEvent_t evs[kLookahead + 1] = {};
 };
 
 int64_t dist_slice(int64_t n, int32_t p) {
@@ -99,8 +168,11 @@ int64_t dist_slice(int64_t n, int32_t p) {
 // ------------------------------------------------------------------ kernels
 namespace {
 
+constexpr int kDB = 256;    // threads per CTA of the partition kernels
+constexpr int kDW = kDB / 32;
+
 inline int grid_for(long long work, int sms) {
-    long long b = (work + kBlock - 1) / kBlock;
+    long long b = (work + kDB - 1) / kDB;
     return (int)std::max(1LL, std::min(b, (long long)sms * 8));
 }
 
@@ -110,7 +182,10 @@ __global__ void k_rebase_offsets(const int64_t *in, int64_t base, uint32_t *out,
 __global__ void k_rebase_offsets_u32(const uint32_t *in, uint32_t base, uint32_t *out, long long n1) {
     for (long long i = gtid(); i < n1; i += gthreads()) out[i] = in[i] - base;
 }
-// slice CSR: count global sources
+__global__ void k_first(const uint32_t *roff, const int32_t *rcol, int nloc, int32_t *first) {
+    for (long long v = gtid(); v < nloc; v += gthreads()) first[v] = roff[v + 1] > roff[v] ? rcol[roff[v]] : -1;
+}
+// column slice "global source -> owned targets": count, scan, fill
 __global__ void k_slice_count(const uint32_t *roff, const int32_t *rcol, int nloc, uint32_t *cnt) {
     for (long long v = gtid(); v < nloc; v += gthreads())
         for (uint32_t e = roff[v]; e < roff[v + 1]; ++e) atomicAdd(cnt + rcol[e], 1u);
@@ -119,227 +194,479 @@ __global__ void k_slice_fill(const uint32_t *roff, const int32_t *rcol, int nloc
     for (long long v = gtid(); v < nloc; v += gthreads())
         for (uint32_t e = roff[v]; e < roff[v + 1]; ++e) scol[atomicAdd(cursor + rcol[e], 1u)] = (int32_t)v;
 }
+// heavy owned rows -> kHeavy-edge chunks (order irrelevant: partials meet in atomics)
+__global__ void k_chunks(const uint32_t *roff, int nloc, DTask *tab, unsigned *cnt) {
+    for (long long v = gtid(); v < nloc; v += gthreads()) {
+        const uint32_t b = roff[v], e = roff[v + 1];
+        if (e - b > kHeavy) {
+            const unsigned k = (e - b + kHeavy - 1) / kHeavy;
+            const unsigned i = atomicAdd(cnt, k);
+            for (unsigned j = 0; j < k; ++j) tab[i + j] = DTask{(int)v, b + j * kHeavy, min(e, b + (j + 1) * kHeavy)};
+        }
+    }
+}
 
-struct BfsPartArgs {
+// CTA reduction of up to 3 u64 counters + 1 f64 into a part's counter slot (one atomic each)
+__device__ __forceinline__ void flush_loc(unsigned long long a, unsigned long long b, unsigned long long c,
+                                          double f, unsigned long long *loc) {
+    __shared__ unsigned long long s[kDW][3];
+    __shared__ double sf[kDW];
+    a = warp_sum(a); b = warp_sum(b); c = warp_sum(c); f = warp_sum(f);
+    if (lane_id() == 0) { s[threadIdx.x >> 5][0] = a; s[threadIdx.x >> 5][1] = b; s[threadIdx.x >> 5][2] = c; sf[threadIdx.x >> 5] = f; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long x = 0, y = 0, z = 0;
+        double ff = 0.0;
+        for (int w = 0; w < kDW; ++w) { x += s[w][0]; y += s[w][1]; z += s[w][2]; ff += sf[w]; }
+        if (x) atomicAdd(loc, x);
+        if (y) atomicAdd(loc + 1, y);
+        if (z) atomicAdd(loc + 2, z);
+        if (ff != 0.0) atomicAdd(reinterpret_cast<double *>(loc + 4), ff);
+    }
+}
+
+__global__ void k_sum_parts(const unsigned long long *locs, int parts, DCtl *ctl) {
+    if (threadIdx.x < 4) {
+        unsigned long long s = 0;
+        for (int p = 0; p < parts; ++p) s += locs[p * kLocStride + threadIdx.x];
+        ctl->tot[threadIdx.x] = s;
+    } else if (threadIdx.x == 4) {
+        double s = 0.0;
+        for (int p = 0; p < parts; ++p) s += reinterpret_cast<const double *>(locs + p * kLocStride)[4];
+        ctl->dtot = s;
+    }
+}
+__global__ void k_zero_locs(unsigned long long *locs, int parts) {
+    for (int i = threadIdx.x; i < parts * kLocStride; i += blockDim.x) locs[i] = 0ull;
+}
+
+// ---------------------------------------------------------------- BFS
+struct BfsP {
     const uint32_t *roff;
-    const int32_t *rcol;
+    const int32_t *rcol, *rfirst;
     const uint32_t *soff;
     const int32_t *scol;
     unsigned *vis;
     int *depth;               // owned slice
-    int64_t vb;
+    int64_t vb, npad;
     int nloc;
-    int64_t npad;
     const unsigned *fb;       // FB_t (global)
     unsigned *nfb;            // FB_{t+1} (global; this part writes its slice)
+    DTask *tasks;
+    unsigned *ntasks;
+    uint32_t task_cap;
+    unsigned long long *loc;
+    const DCtl *ctl;
     int lvl;
-    unsigned long long *cnt;  // {va, ea, edges}
 };
 
-__device__ __forceinline__ void add_counts(unsigned long long va, unsigned long long ea, unsigned long long ed,
-                                           unsigned long long *cnt) {
-    va = warp_sum(va); ea = warp_sum(ea); ed = warp_sum(ed);
-    if (lane_id() == 0 && (va | ed)) { atomicAdd(cnt, va); atomicAdd(cnt + 1, ea); atomicAdd(cnt + 2, ed); }
-}
-
-__global__ void k_bfs_init(BfsPartArgs a, int64_t src) {
+__global__ void k_bfs_init(BfsP a, int64_t src, unsigned *fb0) {
     const int W = (a.nloc + 31) >> 5;
     for (long long v = gtid(); v < a.nloc; v += gthreads()) a.depth[v] = (a.vb + v == src) ? 0 : -1;
     for (long long w = gtid(); w < W; w += gthreads()) {
         unsigned m = 0;
         for (int b = 0; b < 32; ++b) {
-            long long v = w * 32 + b;
-            bool done = v >= a.nloc || a.roff[v + 1] == a.roff[v] || a.vb + v == src;
+            const long long v = w * 32 + b;
+            const bool done = v >= a.nloc || a.roff[v + 1] == a.roff[v] || a.vb + v == src;   // padding, isolated, source
             m |= (done ? 1u : 0u) << b;
         }
         a.vis[w] = m;
     }
+    if (gtid() == 0 && src >= a.vb && src < a.vb + a.nloc) {
+        const int v = (int)(src - a.vb);
+        a.loc[0] = 1ull;
+        a.loc[1] = a.roff[v + 1] - a.roff[v];
+        atomicOr(fb0 + (src >> 5), 1u << (src & 31));
+    }
 }
 
-// push: warp per frontier word, lanes stride over the slice rows of its set bits
-__global__ void k_bfs_push(BfsPartArgs a) {
+// claim local target v for level lvl+1 (push): returns 1 if this call won it
+__device__ __forceinline__ bool push_claim(const BfsP &a, int v, unsigned long long &va, unsigned long long &ea) {
+    const unsigned bit = 1u << (v & 31);
+    if (a.vis[v >> 5] & bit) return false;
+    if (atomicOr(a.vis + (v >> 5), bit) & bit) return false;
+    a.depth[v] = a.lvl + 1;
+    atomicOr(a.nfb + ((a.vb + v) >> 5), bit);      // vb is a multiple of 64
+    va++;
+    ea += a.roff[v + 1] - a.roff[v];
+    return true;
+}
+
+// push, light part: a lane per frontier vertex of the warp's bitmap word (rows <= 32 edges, 4
+// columns in flight), the whole warp for rows of 33..kHeavy edges, tasks for longer rows
+__global__ void __launch_bounds__(kDB) k_bfs_push(BfsP a) {
+    if (a.ctl->done || a.ctl->dir != GSW_PUSH) return;
     const long long FW = a.npad >> 5;
+    const unsigned lane = lane_id();
     unsigned long long va = 0, ea = 0, ed = 0;
     for (long long w = gwarp(); w < FW; w += gwarps()) {
-        unsigned word = a.fb[w];
-        while (word) {
-            const int b = __ffs(word) - 1;
-            word &= word - 1;
-            const long long u = w * 32 + b;
-            const uint32_t s0 = a.soff[u], s1 = a.soff[u + 1];
-            for (uint32_t e = s0 + lane_id(); e < s1; e += 32) {
-                const int v = a.scol[e];
-                ed++;
-                const unsigned bit = 1u << (v & 31);
-                if (a.vis[v >> 5] & bit) continue;
-                if (atomicOr(a.vis + (v >> 5), bit) & bit) continue;
-                a.depth[v] = a.lvl + 1;
-                atomicOr(a.nfb + ((a.vb + v) >> 5), bit);      // vb is a multiple of 64
-                va++;
-                ea += a.roff[v + 1] - a.roff[v];
+        const unsigned word = a.fb[w];
+        if (!word) continue;
+        const bool mine = (word >> lane) & 1u;
+        const long long u = w * 32 + lane;
+        uint32_t s0 = 0, s1 = 0;
+        if (mine) { s0 = a.soff[u]; s1 = a.soff[u + 1]; }
+        const uint32_t L = s1 - s0;
+        if (mine && L > kHeavy) {
+            const unsigned k = (L + kHeavy - 1) / kHeavy;
+            const unsigned i = atomicAdd(a.ntasks, k);
+            for (unsigned j = 0; j < k && i + j < a.task_cap; ++j)
+                a.tasks[i + j] = DTask{(int)u, s0 + j * kHeavy, min(s1, s0 + (j + 1) * kHeavy)};
+        }
+        if (mine && L <= 32) {
+            for (uint32_t e = s0; e < s1; e += 4) {
+                int v[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) v[k] = e + k < s1 ? __ldg(a.scol + e + k) : -1;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) if (v[k] >= 0) { ed++; push_claim(a, v[k], va, ea); }
             }
         }
+        unsigned mid = __ballot_sync(0xffffffffu, mine && L > 32 && L <= kHeavy);
+        while (mid) {
+            const int j = __ffs(mid) - 1;
+            mid &= mid - 1;
+            const uint32_t b = __shfl_sync(0xffffffffu, s0, j), e = __shfl_sync(0xffffffffu, s1, j);
+            for (uint32_t k = b + lane; k < e; k += 32) { ed++; push_claim(a, __ldg(a.scol + k), va, ea); }
+        }
     }
-    add_counts(va, ea, ed, a.cnt);
+    flush_loc(va, ea, ed, 0.0, a.loc);
 }
 
-// pull: warp per owned 32-vertex word, lane = vertex, early exit at the first frontier parent
-__global__ void k_bfs_pull(BfsPartArgs a) {
-    const int W = (a.nloc + 31) >> 5;
+__global__ void __launch_bounds__(kDB) k_bfs_push_heavy(BfsP a) {
+    if (a.ctl->done || a.ctl->dir != GSW_PUSH) return;
+    const unsigned nt = min(*a.ntasks, a.task_cap);
     unsigned long long va = 0, ea = 0, ed = 0;
-    for (long long w = gwarp(); w < W; w += gwarps()) {
-        const unsigned vis = a.vis[w];
-        const long long v = w * 32 + lane_id();
-        bool found = false;
-        uint32_t deg = 0;
-        if (!((vis >> lane_id()) & 1u)) {
-            const uint32_t b = a.roff[v], e = a.roff[v + 1];
-            deg = e - b;
-            for (uint32_t k = b; k < e; ++k) {
-                const int u = a.rcol[k];
-                ed++;
-                if ((a.fb[u >> 5] >> (u & 31)) & 1u) { found = true; break; }
-            }
-        }
-        const unsigned hits = __ballot_sync(0xffffffffu, found);
-        if (found) { a.depth[v] = a.lvl + 1; va++; ea += deg; }
-        if (lane_id() == 0 && hits) {
-            a.vis[w] = vis | hits;
-            a.nfb[(a.vb >> 5) + w] = hits;
-        }
+    for (long long k = gwarp(); k < nt; k += gwarps()) {
+        const DTask tk = a.tasks[k];
+        for (uint32_t e = tk.beg + lane_id(); e < tk.end; e += 32) { ed++; push_claim(a, __ldg(a.scol + e), va, ea); }
     }
-    add_counts(va, ea, ed, a.cnt);
+    flush_loc(va, ea, ed, 0.0, a.loc);
 }
 
-__global__ void k_set_bit(unsigned *fb, int64_t v) { atomicOr(fb + (v >> 5), 1u << (v & 31)); }
-
-__global__ void k_sum_parts(unsigned long long *cnt, int parts) {
-    if (threadIdx.x < 3) {
-        unsigned long long s = 0;
-        for (int p = 0; p < parts; ++p) s += cnt[3 * p + threadIdx.x];
-        cnt[3 * parts + threadIdx.x] = s;
-    }
+__global__ void __launch_bounds__(kDB) k_bfs_pull(BfsP a) {
+    if (a.ctl->done || a.ctl->dir != GSW_PULL) return;
+    __shared__ int lists[(kPullList + kPullWordsPerWarp) * kDW];
+    LocalCnt c = bfs_pull_list(a.fb, a.vis, a.depth, a.roff, a.rcol, a.rfirst, a.roff, true, a.lvl,
+                               a.nfb + (a.vb >> 5), a.nloc, lists);
+    flush_loc(c.va, c.ea, c.edges, 0.0, a.loc);
 }
 
-struct PrPartArgs {
+// one thread: account level t (its expand just finished, tot = counts of AS_{t+1}), decide t+1
+__global__ void k_bfs_decide(DCtl *ctl, DRec *recs, unsigned long long *locs, int parts, int t, long long n,
+                             int force_dir) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const unsigned long long va = ctl->tot[0], ea = ctl->tot[1], ed = ctl->tot[2];
+    for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
+    if (ctl->done) return;
+    if (t >= 0 && t < kMaxLevels) recs[t].edges = (long long)ed;
+    if (va == 0) { ctl->done = 1; return; }
+    ctl->Via -= (long long)va;
+    ctl->Eia -= (long long)ea;
+    // the single-GPU direction split (select.cuh, R6) on the GLOBAL features
+    int dir = ((double)ea * 16.0 > (double)ctl->Eia && (double)va * 2048.0 > (double)n) ? GSW_PULL : GSW_PUSH;
+    if (force_dir != GSW_AUTO) dir = force_dir;
+    ctl->dir = dir;
+    ctl->t = t + 2;                                   // levels with a non-empty active set so far
+    if (t + 1 < kMaxLevels) recs[t + 1] = DRec{(long long)va, (long long)ea, ctl->Via, ctl->Eia, 0, dir, 0};
+}
+
+// ---------------------------------------------------------------- PageRank
+struct PrP {
     const uint32_t *roff;
     const int32_t *rcol;
     int64_t vb;
     int nloc;
-    const double *cur;        // replicated contributions
-    double *next;             // replicated next contributions (this part writes its slice)
-    const double *dtot;       // D_t
-    double *dpart;            // this part's dangling accumulator for D_{t+1}
+    const float *cur;         // replicated contributions pr_t(u)/deg(u)
+    float *next;              // replicated next contributions (this part writes its slice)
     double *out;              // owned slice output (last iteration) or nullptr
-    double base, d, invN;
+    const DTask *chunks;
+    const unsigned *nchunks;
+    double *psum;
+    unsigned long long *loc;
+    const DCtl *ctl;          // dtot = dangling mass of pr_t
+    double d, invN;
 };
 
-__global__ void k_pr_init(PrPartArgs a) {
+__global__ void k_pr_init(PrP a) {
     double dang = 0.0;
     for (long long v = gtid(); v < a.nloc; v += gthreads()) {
-        uint32_t dg = a.roff[v + 1] - a.roff[v];
-        a.next[a.vb + v] = dg ? a.invN / dg : 0.0;
+        const uint32_t dg = a.roff[v + 1] - a.roff[v];
+        a.next[a.vb + v] = dg ? (float)(a.invN / dg) : 0.f;
         if (!dg) dang += a.invN;
         if (a.out) a.out[v] = a.invN;
+        a.psum[v] = 0.0;
     }
-    dang = warp_sum(dang);
-    if (lane_id() == 0 && dang != 0.0) atomicAdd(a.dpart, dang);
+    flush_loc(0, 0, 0, dang, a.loc);
 }
 
-// warp per 32 owned rows: short rows one lane each, long rows warp-cooperative
-__global__ void k_pr_iter(PrPartArgs a) {
-    const double D = *a.dtot;
-    const double base = a.base + a.d * D * a.invN;
+__global__ void __launch_bounds__(kDB) k_pr_heavy(PrP a) {
+    const unsigned nc = *a.nchunks;
+    for (long long k = gwarp(); k < nc; k += gwarps()) {
+        const DTask tk = a.chunks[k];
+        double s = 0.0;
+        for (uint32_t e = tk.beg + lane_id(); e < tk.end; e += 32) s += (double)a.cur[__ldg(a.rcol + e)];
+        s = warp_sum(s);
+        if (lane_id() == 0) atomicAdd(a.psum + tk.row, s);
+    }
+}
+
+// a lane per row below 32 edges (4 gathers in flight), the warp for rows up to kHeavy, the
+// chunk partials for heavier rows
+__global__ void __launch_bounds__(kDB) k_pr_rows(PrP a) {
+    const double base = (1.0 - a.d) * a.invN + a.d * a.ctl->dtot * a.invN;
+    const unsigned lane = lane_id();
     double dang = 0.0;
     for (long long wb = gwarp() * 32; wb < a.nloc; wb += gwarps() * 32) {
-        const long long v = wb + lane_id();
+        const long long v = wb + lane;
         uint32_t b = 0, e = 0;
         if (v < a.nloc) { b = a.roff[v]; e = a.roff[v + 1]; }
+        const uint32_t L = e - b;
         double s = 0.0;
-        if (e - b < 32) for (uint32_t k = b; k < e; ++k) s += a.cur[a.rcol[k]];
-        unsigned longrows = __ballot_sync(0xffffffffu, v < a.nloc && e - b >= 32);
-        while (longrows) {
-            const int j = __ffs(longrows) - 1;
-            longrows &= longrows - 1;
+        if (v < a.nloc && L < 32) {
+            double s0 = 0.0, s1 = 0.0;
+            uint32_t k = b;
+            for (; k + 4 <= e; k += 4) {
+                const int u0 = __ldg(a.rcol + k), u1 = __ldg(a.rcol + k + 1), u2 = __ldg(a.rcol + k + 2), u3 = __ldg(a.rcol + k + 3);
+                s0 += (double)a.cur[u0] + (double)a.cur[u1];
+                s1 += (double)a.cur[u2] + (double)a.cur[u3];
+            }
+            for (; k < e; ++k) s0 += (double)a.cur[__ldg(a.rcol + k)];
+            s = s0 + s1;
+        } else if (v < a.nloc && L > kHeavy) {
+            s = a.psum[v];
+            a.psum[v] = 0.0;
+        }
+        unsigned mid = __ballot_sync(0xffffffffu, v < a.nloc && L >= 32 && L <= kHeavy);
+        while (mid) {
+            const int j = __ffs(mid) - 1;
+            mid &= mid - 1;
             const uint32_t bj = __shfl_sync(0xffffffffu, b, j), ej = __shfl_sync(0xffffffffu, e, j);
             double t = 0.0;
-            for (uint32_t k = bj + lane_id(); k < ej; k += 32) t += a.cur[a.rcol[k]];
+            for (uint32_t k = bj + lane; k < ej; k += 32) t += (double)a.cur[__ldg(a.rcol + k)];
             t = warp_sum(t);
-            if ((int)lane_id() == j) s = t;
+            if ((int)lane == j) s = t;
         }
         if (v < a.nloc) {
             const double p = base + a.d * s;
-            const uint32_t dg = e - b;
-            a.next[a.vb + v] = dg ? p / dg : 0.0;
-            if (!dg) dang += p;
+            a.next[a.vb + v] = L ? (float)(p / (double)L) : 0.f;
+            if (!L) dang += p;
             if (a.out) a.out[v] = p;
         }
     }
-    dang = warp_sum(dang);
-    if (lane_id() == 0 && dang != 0.0) atomicAdd(a.dpart, dang);
+    flush_loc(0, 0, 0, dang, a.loc);
 }
 
-__global__ void k_sum_dang(double *dang, int parts) {
-    if (threadIdx.x == 0) {
-        double s = 0.0;
-        for (int p = 0; p < parts; ++p) s += dang[p];
-        dang[parts] = s;
+// ---------------------------------------------------------------- CC
+struct CcP {
+    const uint32_t *roff;
+    const int32_t *rcol;
+    int64_t vb;
+    int nloc;
+    const uint32_t *cur;      // replicated labels
+    uint32_t *next;           // replicated next labels (this part writes its slice)
+    int32_t *out;             // owned slice output or nullptr
+    const DTask *chunks;
+    const unsigned *nchunks;
+    uint32_t *hmin;           // heavy-row minima (nloc), ~0 between iterations
+    unsigned long long *loc;
+    const DCtl *ctl;
+};
+
+__global__ void k_cc_init(uint32_t *lab, int64_t npad, uint32_t *hmin, int nloc) {
+    for (long long v = gtid(); v < npad; v += gthreads()) lab[v] = (uint32_t)v;
+    for (long long v = gtid(); v < nloc; v += gthreads()) hmin[v] = 0xffffffffu;
+}
+
+__global__ void __launch_bounds__(kDB) k_cc_heavy(CcP a) {
+    if (a.ctl->done) return;
+    const unsigned nc = *a.nchunks;
+    for (long long k = gwarp(); k < nc; k += gwarps()) {
+        const DTask tk = a.chunks[k];
+        uint32_t m = 0xffffffffu;
+        for (uint32_t e = tk.beg + lane_id(); e < tk.end; e += 32) m = min(m, a.cur[__ldg(a.rcol + e)]);
+        m = warp_min(m);
+        if (lane_id() == 0) atomicMin(a.hmin + tk.row, m);
     }
+}
+
+// label'[v] = min(label[v], min over neighbours), then the shortcut label'[v] = label[label'[v]]
+__global__ void __launch_bounds__(kDB) k_cc_rows(CcP a) {
+    if (a.ctl->done) return;
+    const unsigned lane = lane_id();
+    unsigned long long changed = 0;
+    for (long long wb = gwarp() * 32; wb < a.nloc; wb += gwarps() * 32) {
+        const long long v = wb + lane;
+        uint32_t b = 0, e = 0;
+        if (v < a.nloc) { b = a.roff[v]; e = a.roff[v + 1]; }
+        const uint32_t L = e - b;
+        uint32_t m = v < a.nloc ? a.cur[a.vb + v] : 0xffffffffu;
+        if (v < a.nloc && L < 32) {
+            uint32_t k = b;
+            for (; k + 4 <= e; k += 4) {
+                const int u0 = __ldg(a.rcol + k), u1 = __ldg(a.rcol + k + 1), u2 = __ldg(a.rcol + k + 2), u3 = __ldg(a.rcol + k + 3);
+                m = min(m, min(min(a.cur[u0], a.cur[u1]), min(a.cur[u2], a.cur[u3])));
+            }
+            for (; k < e; ++k) m = min(m, a.cur[__ldg(a.rcol + k)]);
+        } else if (v < a.nloc && L > kHeavy) {
+            m = min(m, a.hmin[v]);
+            a.hmin[v] = 0xffffffffu;
+        }
+        unsigned mid = __ballot_sync(0xffffffffu, v < a.nloc && L >= 32 && L <= kHeavy);
+        while (mid) {
+            const int j = __ffs(mid) - 1;
+            mid &= mid - 1;
+            const uint32_t bj = __shfl_sync(0xffffffffu, b, j), ej = __shfl_sync(0xffffffffu, e, j);
+            uint32_t t = 0xffffffffu;
+            for (uint32_t k = bj + lane; k < ej; k += 32) t = min(t, a.cur[__ldg(a.rcol + k)]);
+            t = warp_min(t);
+            if ((int)lane == j) m = min(m, t);
+        }
+        if (v < a.nloc) {
+            m = min(m, a.cur[m]);                     // pointer jumping on the replicated labels
+            a.next[a.vb + v] = m;
+            changed += m != a.cur[a.vb + v];
+            if (a.out) a.out[v] = (int32_t)m;
+        }
+    }
+    flush_loc(0, 0, 0, 0.0, a.loc);
+    changed = warp_sum(changed);
+    if (lane == 0 && changed) atomicAdd(a.loc + 3, changed);
+}
+
+__global__ void k_cc_decide(DCtl *ctl, unsigned long long *locs, int parts, int t) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const unsigned long long ch = ctl->tot[3];
+    for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
+    if (ctl->done) return;
+    ctl->t = t + 1;
+    if (ch == 0) ctl->done = 1;
 }
 
 }  // namespace
 
 // ------------------------------------------------------------------ workspace + creation
 static size_t al(size_t x) { return (x + 255) & ~size_t(255); }
+static size_t chunk_cap(uint64_t nnz) { return (size_t)(2 * nnz / kHeavy + 2); }
 
-static size_t dist_bytes(int64_t n, int64_t nnz_owned_total, int32_t nranks, int32_t nparts, bool own_copy_rows) {
+static size_t dist_bytes(int64_t n, int64_t nnz_total, int32_t nranks, int32_t nparts, int mode) {
     const int64_t S = dist_slice(n, nranks), npad = S * nranks;
     size_t b = 0;
     b += al((size_t)npad / 8) * 2;                           // FB[2]
-    b += al((size_t)npad * 8) * 2;                           // contrib[2]
-    b += al(64 * 8 * (nparts + 1)) + al(8 * (nparts + 1));  // counters
+    b += al((size_t)npad * 4) * 2;                           // rep[2]
+    b += al((size_t)kLocStride * 8 * nparts) + al(sizeof(DCtl)) + al(sizeof(DRec) * kMaxLevels);
     for (int p = 0; p < nparts; ++p) {
-        b += al((size_t)(S + 1) * 4);                        // roff
+        b += al((size_t)(S + 1) * 4) + al((size_t)S * 4);    // roff, rfirst
         b += al((size_t)(n + 1) * 4);                        // soff
-        b += al((size_t)S / 8);                              // vis
+        b += al((size_t)S / 8 + 8);                          // vis
+        b += al((size_t)S * 8);                              // psum
+        b += al(256) * 2;                                    // nchunks, nptasks
     }
-    b += al((size_t)nnz_owned_total * 4);                    // scol (all parts)
-    if (own_copy_rows) b += al((size_t)nnz_owned_total * 4); // rcol copy (NCCL mode)
-    else b += al((size_t)nnz_owned_total * 4) + al((size_t)(n + 1) * 4);   // full CSR (loopback)
+    // chunk and push-task tables: bounded by the part's nnz, summed over parts <= total nnz
+    b += (size_t)nparts * 2 * al(0) + 2 * al(chunk_cap((uint64_t)nnz_total) * sizeof(DTask)) + nparts * 512;
+    b += al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // scol (all parts)
+    b += al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // rcol copy
+    if (mode == DM_LOOPBACK) b += al((size_t)(n + 1) * 4);  // full u32 offsets
     size_t cub = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, cub, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(n + 1));
     b += al(cub) + al((size_t)(n + 1) * 4);                  // scan temp + cursor
-    b += al((size_t)(n + 1) * 8);                            // i64 staging
-    b += al((size_t)npad * 8) * 2;                           // output staging (depth / rank)
-    return b + (1 << 20);
+    b += al((size_t)(n + 1) * 8);                            // i64 staging of the caller's offsets
+    b += al((size_t)npad * 8);                               // output staging (depth / rank / labels)
+    return b + (2 << 20);
 }
 
-static gsw_status build_slice(gsw_graph g, DPart &p, int64_t n, Workspace &tmp_ws, int32_t *scol, void *cub_tmp,
-                              size_t cub_bytes, uint32_t *cursor) {
+static gsw_status build_slice(gsw_graph g, DPart &p, int64_t n, int32_t *scol, void *cub_tmp, size_t cub_bytes,
+                              uint32_t *cursor) {
     cudaStream_t s = g->stream;
     GSW_CUDA(cudaMemsetAsync(p.soff, 0, (size_t)(n + 1) * 4, s));
-    k_slice_count<<<grid_for(p.nloc, g->sms), kBlock, 0, s>>>(p.roff, p.rcol, p.nloc, p.soff);
+    k_slice_count<<<grid_for(p.nloc, g->sms), kDB, 0, s>>>(p.roff, p.rcol, p.nloc, p.soff);
     GSW_CUDA(cudaGetLastError());
     size_t cb = cub_bytes;
     GSW_CUDA(cub::DeviceScan::ExclusiveSum(cub_tmp, cb, p.soff, p.soff, (int)(n + 1), s));
     GSW_CUDA(cudaMemcpyAsync(cursor, p.soff, (size_t)(n + 1) * 4, cudaMemcpyDeviceToDevice, s));
-    k_slice_fill<<<grid_for(p.nloc, g->sms), kBlock, 0, s>>>(p.roff, p.rcol, p.nloc, cursor, scol);
+    k_slice_fill<<<grid_for(p.nloc, g->sms), kDB, 0, s>>>(p.roff, p.rcol, p.nloc, cursor, scol);
     GSW_CUDA(cudaGetLastError());
     p.scol = scol;
-    (void)tmp_ws;
     return GSW_OK;
 }
 
-gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int32_t nranks, int32_t rank,
-                       bool loopback, void *workspace, size_t ws_bytes, void *stream, gsw_graph *out) {
+// ---- exchange (the only place the three backends differ)
+static gsw_status host_stage(DistState *d, size_t bytes) {
+    if (bytes <= d->hcap) return GSW_OK;
+    if (d->hsend) cudaFreeHost(d->hsend);
+    if (d->hrecv) cudaFreeHost(d->hrecv);
+    d->hsend = d->hrecv = nullptr;
+    d->hcap = 0;
+    GSW_CUDA(cudaHostAlloc((void **)&d->hsend, bytes, cudaHostAllocDefault));
+    GSW_CUDA(cudaHostAlloc((void **)&d->hrecv, bytes * d->nranks, cudaHostAllocDefault));
+    d->hcap = bytes;
+    return GSW_OK;
+}
+
+// in-place all-gather of the rank slices of a replicated buffer (S elements of esize bytes each)
+static gsw_status ex_allgather(DistState *d, void *buf, size_t esize, cudaStream_t s) {
+    const size_t per = (size_t)d->S * esize;
+    if (d->mode == DM_LOOPBACK) return GSW_OK;                 // the replica is shared by the parts
+    if (d->mode == DM_NCCL) {
+        const ncclDataType_t ty = esize == 4 ? ncclUint32 : ncclUint8;
+        const size_t cnt = esize == 4 ? (size_t)d->S : per;
+        GSW_NCCL(g_nccl.allGather((char *)buf + (size_t)d->rank * per, buf, cnt, ty, d->comm, s));
+        return GSW_OK;
+    }
+    if (gsw_status e = host_stage(d, per)) return e;
+    GSW_CUDA(cudaMemcpyAsync(d->hsend, (char *)buf + (size_t)d->rank * per, per, cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    if (d->hx.allgather(d->hx.user, d->hsend, d->hrecv, per) != 0) { set_error("host exchange: allgather callback failed"); return GSW_ENCCL; }
+    GSW_CUDA(cudaMemcpyAsync(buf, d->hrecv, per * d->nranks, cudaMemcpyHostToDevice, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    return GSW_OK;
+}
+
+// sum the parts' / ranks' counters into ctl->tot and ctl->dtot
+static gsw_status ex_reduce(DistState *d, cudaStream_t s) {
+    if (d->mode == DM_LOOPBACK) {
+        k_sum_parts<<<1, 32, 0, s>>>(d->locs, (int)d->parts.size(), d->ctl);
+        GSW_CUDA(cudaGetLastError());
+        return GSW_OK;
+    }
+    if (d->mode == DM_NCCL) {
+        GSW_NCCL(g_nccl.groupStart());
+        GSW_NCCL(g_nccl.allReduce(d->locs, d->ctl->tot, 4, ncclUint64, ncclSum, d->comm, s));
+        GSW_NCCL(g_nccl.allReduce(d->locs + 4, &d->ctl->dtot, 1, ncclFloat64, ncclSum, d->comm, s));
+        GSW_NCCL(g_nccl.groupEnd());
+        return GSW_OK;
+    }
+    unsigned long long h[kLocStride];
+    GSW_CUDA(cudaMemcpyAsync(h, d->locs, sizeof(h), cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    double f;
+    std::memcpy(&f, h + 4, 8);
+    if (d->hx.allreduce_u64(d->hx.user, (uint64_t *)h, 4) != 0 || d->hx.allreduce_f64(d->hx.user, &f, 1) != 0) {
+        set_error("host exchange: allreduce callback failed");
+        return GSW_ENCCL;
+    }
+    std::memcpy(h + 4, &f, 8);
+    GSW_CUDA(cudaMemcpyAsync(d->ctl->tot, h, 32, cudaMemcpyHostToDevice, s));
+    GSW_CUDA(cudaMemcpyAsync(&d->ctl->dtot, h + 4, 8, cudaMemcpyHostToDevice, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    return GSW_OK;
+}
+
+gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, const gsw_exchange *hx, int32_t nranks,
+                       int32_t rank, int mode, void *workspace, size_t ws_bytes, void *stream, gsw_graph *out) {
     *out = nullptr;
     if (!rows || !rows->row_offsets || (rows->nnz > 0 && !rows->col_indices) || n <= 0 || nranks < 1 ||
         rank < 0 || rank >= nranks) {
         set_error("dist create: bad arguments");
         return GSW_EINVAL;
     }
+    if (mode == DM_HOST && (!hx || !hx->allgather || !hx->allreduce_u64 || !hx->allreduce_f64)) {
+        set_error("dist create: host exchange needs allgather / allreduce_u64 / allreduce_f64 callbacks");
+        return GSW_EINVAL;
+    }
     if (n >= (int64_t(1) << 31) - 64 || rows->nnz >= (int64_t(1) << 32)) { set_error("graph too large"); return GSW_EOVERFLOW; }
     const int64_t S = dist_slice(n, nranks);
+    const bool loopback = mode == DM_LOOPBACK;
     const int nparts = loopback ? nranks : 1;
     if (!loopback) {
         const int64_t own = std::max<int64_t>(0, std::min<int64_t>(n, (int64_t)(rank + 1) * S) - (int64_t)rank * S);
@@ -348,7 +675,7 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int3
         set_error("loopback mode takes the full graph");
         return GSW_EINVAL;
     }
-    const size_t need = dist_bytes(n, rows->nnz, nranks, nparts, !loopback);
+    const size_t need = dist_bytes(n, rows->nnz, nranks, nparts, mode);
     if (!workspace || is_device_ptr(workspace) != 1 || ws_bytes < need) {
         set_error("dist workspace must be a device buffer of >= " + std::to_string(need) + " bytes");
         return GSW_ENOMEM;
@@ -364,25 +691,41 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int3
     if (e != cudaSuccess) { delete g; return cuda_fail(e, "dist create setup"); }
     DistState *d = new DistState();
     g->dist = d;
-    d->nranks = nranks; d->rank = rank; d->loopback = loopback;
+    d->mode = mode;
+    d->nranks = nranks; d->rank = rank;
     d->n = n; d->S = S; d->npad = S * nranks;
+    if (hx) d->hx = *hx;
     g->g.n = (int)n;
     g->g.nnz = (uint32_t)rows->nnz;
+    auto fail = [&](gsw_status st) { gsw_graph_destroy(g); return st; };
+    for (auto &ev : d->evs)
+        if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "events"));
+    if (cudaHostAlloc((void **)&d->hdone, sizeof(int) * (kLookahead + 1), cudaHostAllocDefault) != cudaSuccess)
+        return fail(cuda_fail(cudaGetLastError(), "pinned flags"));
     Workspace ws{g->ws, ws_bytes, 0};
     d->FB[0] = (unsigned *)ws.take(d->npad / 8);
     d->FB[1] = (unsigned *)ws.take(d->npad / 8);
-    d->contrib[0] = (double *)ws.take(d->npad * 8);
-    d->contrib[1] = (double *)ws.take(d->npad * 8);
-    d->cnt = (unsigned long long *)ws.take(64 * 8 * (nparts + 1));
-    d->dang = (double *)ws.take(8 * (nparts + 1));
+    d->rep[0] = (uint32_t *)ws.take(d->npad * 4);
+    d->rep[1] = (uint32_t *)ws.take(d->npad * 4);
+    d->locs = (unsigned long long *)ws.take((size_t)kLocStride * 8 * nparts);
+    d->ctl = (DCtl *)ws.take(sizeof(DCtl));
+    d->recs = (DRec *)ws.take(sizeof(DRec) * kMaxLevels);
     int64_t *staging = (int64_t *)ws.take((size_t)(n + 1) * 8);
     size_t cub_bytes = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, cub_bytes, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(n + 1));
     void *cub_tmp = ws.take(cub_bytes);
     uint32_t *cursor = (uint32_t *)ws.take((size_t)(n + 1) * 4);
     int32_t *scol_all = (int32_t *)ws.take((size_t)std::max<int64_t>(rows->nnz, 1) * 4);
+    int32_t *col = (int32_t *)ws.take((size_t)std::max<int64_t>(rows->nnz, 1) * 4);
+    uint32_t *full_off = loopback ? (uint32_t *)ws.take((size_t)(n + 1) * 4) : nullptr;
+    DTask *chunk_all = (DTask *)ws.take(chunk_cap((uint64_t)rows->nnz) * sizeof(DTask));
+    DTask *task_all = (DTask *)ws.take(chunk_cap((uint64_t)rows->nnz) * sizeof(DTask));
+    if (!d->FB[1] || !d->rep[1] || !d->locs || !d->ctl || !d->recs || !staging || !cub_tmp || !cursor || !scol_all ||
+        !col || (loopback && !full_off) || !chunk_all || !task_all) {
+        set_error("dist workspace too small");
+        return fail(GSW_ENOMEM);
+    }
     cudaStream_t s = g->stream;
-    auto fail = [&](gsw_status st) { gsw_graph_destroy(g); return st; };
     // adjacency on the device
     const int64_t *off64 = rows->row_offsets;
     if (!is_device_ptr(off64)) {
@@ -390,21 +733,11 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int3
             return fail(cuda_fail(cudaGetLastError(), "copy offsets"));
         off64 = staging;
     }
-    int32_t *col = (int32_t *)ws.take((size_t)std::max<int64_t>(rows->nnz, 1) * 4);
-    uint32_t *full_off = loopback ? (uint32_t *)ws.take((size_t)(n + 1) * 4) : nullptr;
-    if (!d->FB[1] || !d->contrib[1] || !d->cnt || !d->dang || !staging || !cub_tmp || !cursor || !scol_all || !col ||
-        (loopback && !full_off)) {
-        set_error("dist workspace too small");
-        return fail(GSW_ENOMEM);
-    }
     if (rows->nnz > 0 && cudaMemcpyAsync(col, rows->col_indices, (size_t)rows->nnz * 4,
                                          is_device_ptr(rows->col_indices) ? cudaMemcpyDeviceToDevice
                                                                           : cudaMemcpyHostToDevice, s) != cudaSuccess)
         return fail(cuda_fail(cudaGetLastError(), "copy columns"));
-    if (loopback) {
-        k_rebase_offsets<<<grid_for(n + 1, g->sms), kBlock, 0, s>>>(off64, 0, full_off, n + 1);
-    }
-    // partitions
+    if (loopback) k_rebase_offsets<<<grid_for(n + 1, g->sms), kDB, 0, s>>>(off64, 0, full_off, n + 1);
     std::vector<int64_t> hoff;
     if (loopback) {
         hoff.resize(n + 1);
@@ -413,44 +746,78 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int3
             return fail(cuda_fail(cudaGetLastError(), "read offsets"));
     }
     int32_t *scol_cur = scol_all;
+    DTask *chunk_cur = chunk_all, *task_cur = task_all;
     for (int p = 0; p < nparts; ++p) {
         DPart P;
         const int r = loopback ? p : rank;
         P.vb = (int64_t)r * S;
         P.nloc = (int)std::max<int64_t>(0, std::min<int64_t>(n, P.vb + S) - P.vb);
         P.roff = (uint32_t *)ws.take((size_t)(S + 1) * 4);
+        P.rfirst = (int32_t *)ws.take((size_t)S * 4 + 4);
         P.soff = (uint32_t *)ws.take((size_t)(n + 1) * 4);
-        P.vis = (unsigned *)ws.take((size_t)S / 8);
-        if (!P.roff || !P.soff || !P.vis) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
+        P.vis = (unsigned *)ws.take((size_t)S / 8 + 8);
+        P.psum = (double *)ws.take((size_t)S * 8 + 8);
+        P.nchunks = (unsigned *)ws.take(256);
+        P.nptasks = (unsigned *)ws.take(256);
+        P.loc = d->locs + (size_t)p * kLocStride;
+        if (!P.roff || !P.rfirst || !P.soff || !P.vis || !P.psum || !P.nchunks || !P.nptasks) {
+            set_error("dist workspace too small");
+            return fail(GSW_ENOMEM);
+        }
         if (loopback) {
             const int64_t e0 = P.nloc ? hoff[P.vb] : 0, e1 = P.nloc ? hoff[P.vb + P.nloc] : 0;
             P.nnz = (uint32_t)(e1 - e0);
             P.rcol = col + e0;
-            if (P.nloc) k_rebase_offsets_u32<<<grid_for(P.nloc + 1, g->sms), kBlock, 0, s>>>(full_off + P.vb, (uint32_t)e0,
-                                                                                             P.roff, P.nloc + 1);
+            if (P.nloc)
+                k_rebase_offsets_u32<<<grid_for(P.nloc + 1, g->sms), kDB, 0, s>>>(full_off + P.vb, (uint32_t)e0, P.roff, P.nloc + 1);
         } else {
             P.nnz = (uint32_t)rows->nnz;
             P.rcol = col;
-            k_rebase_offsets<<<grid_for(P.nloc + 1, g->sms), kBlock, 0, s>>>(off64, 0, P.roff, P.nloc + 1);
+            k_rebase_offsets<<<grid_for(P.nloc + 1, g->sms), kDB, 0, s>>>(off64, 0, P.roff, P.nloc + 1);
         }
         if (cudaGetLastError() != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "rebase"));
-        Workspace none{nullptr, 0, 0};
-        gsw_status st = build_slice(g, P, n, none, scol_cur, cub_tmp, cub_bytes, cursor);
-        if (st != GSW_OK) return fail(st);
+        if (gsw_status st = build_slice(g, P, n, scol_cur, cub_tmp, cub_bytes, cursor)) return fail(st);
+        k_first<<<grid_for(P.nloc, g->sms), kDB, 0, s>>>(P.roff, P.rcol, P.nloc, P.rfirst);
+        P.chunks = chunk_cur;
+        P.ptasks = task_cur;
+        P.ptask_cap = (uint32_t)chunk_cap(P.nnz);
+        if (cudaMemsetAsync(P.nchunks, 0, 4, s) != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "memset"));
+        k_chunks<<<grid_for(P.nloc, g->sms), kDB, 0, s>>>(P.roff, P.nloc, P.chunks, P.nchunks);
+        if (cudaGetLastError() != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "chunks"));
         scol_cur += P.nnz;
+        chunk_cur += chunk_cap(P.nnz);
+        task_cur += chunk_cap(P.nnz);
         d->parts.push_back(P);
     }
-    // output staging lives after the partitions
-    g->scratch = (char *)ws.take((size_t)d->npad * 8 * 2);
-    g->scratch_bytes = (size_t)d->npad * 8 * 2;
+    g->scratch = (char *)ws.take((size_t)d->npad * 8);      // output staging (host outputs)
+    g->scratch_bytes = (size_t)d->npad * 8;
     if (!g->scratch) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
     if (cudaStreamSynchronize(s) != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "dist create"));
-    if (!loopback && nranks > 1) {
+    if (mode == DM_NCCL) {
         if (!nccl_load()) return fail(GSW_ENCCL);
+        if (!nccl_id) { set_error("NCCL mode needs the ncclUniqueId"); return fail(GSW_EINVAL); }
         ncclUniqueId id;
         std::memcpy(&id, nccl_id, sizeof(id));
         ncclResult_t r = g_nccl.commInitRank(&d->comm, nranks, id, rank);
         if (r != ncclSuccess) { set_error(std::string("ncclCommInitRank: ") + g_nccl.errStr(r)); return fail(GSW_ENCCL); }
+    }
+    // global nnz (once): every rank's owned entries, summed by the exchange
+    {
+        unsigned long long h[kLocStride] = {};
+        for (auto &P : d->parts) h[0] += P.nnz;            // loopback: part 0's slot carries the total
+        if (cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * nparts, s) != cudaSuccess ||
+            cudaMemcpyAsync(d->locs, h, sizeof(h), cudaMemcpyHostToDevice, s) != cudaSuccess)
+            return fail(cuda_fail(cudaGetLastError(), "nnz"));
+        if (gsw_status st = ex_reduce(d, s)) return fail(st);
+        unsigned long long tot[4];
+        if (cudaMemcpyAsync(tot, d->ctl->tot, 32, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+            cudaStreamSynchronize(s) != cudaSuccess)
+            return fail(cuda_fail(cudaGetLastError(), "nnz"));
+        DCtl c{};
+        c.nnz_g = (long long)tot[0];
+        if (cudaMemcpyAsync(d->ctl, &c, sizeof(c), cudaMemcpyHostToDevice, s) != cudaSuccess ||
+            cudaStreamSynchronize(s) != cudaSuccess)
+            return fail(cuda_fail(cudaGetLastError(), "ctl"));
     }
     *out = g;
     return GSW_OK;
@@ -459,34 +826,40 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, int3
 void dist_destroy(DistState *d) {
     if (!d) return;
     if (d->comm && g_nccl.ok) g_nccl.commDestroy(d->comm);
+    for (auto &ev : d->evs) if (ev) cudaEventDestroy(ev);
+    if (d->hdone) cudaFreeHost(d->hdone);
+    if (d->hsend) cudaFreeHost(d->hsend);
+    if (d->hrecv) cudaFreeHost(d->hrecv);
     delete d;
 }
 
-// ------------------------------------------------------------------ exchange
-static gsw_status allgather_u32(DistState *d, unsigned *buf, size_t words_per_rank, cudaStream_t s) {
-    if (d->loopback || d->nranks == 1) return GSW_OK;                 // shared replica / single rank
-    GSW_NCCL(g_nccl.allGather(buf + (size_t)d->rank * words_per_rank, buf, words_per_rank, ncclUint32, d->comm, s));
+// Pipelined termination: after enqueueing iteration t, poll the done flag of iteration
+// t - LOOKAHEAD (host mode: of t itself, its exchange has synchronised already).  Returns through
+// *stop whether the host should stop enqueueing.
+static gsw_status poll_done(DistState *d, int t, cudaStream_t s, bool *stop) {
+    const int R = kLookahead + 1;
+    GSW_CUDA(cudaMemcpyAsync(d->hdone + (t % R), &d->ctl->done, 4, cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaEventRecord(d->evs[t % R], s));
+    const int lag = d->mode == DM_HOST ? 0 : kLookahead;
+    *stop = false;
+    if (t >= lag) {
+        GSW_CUDA(cudaEventSynchronize(d->evs[(t - lag) % R]));
+        *stop = d->hdone[(t - lag) % R] != 0;
+    }
     return GSW_OK;
 }
-static gsw_status allgather_f64(DistState *d, double *buf, size_t per_rank, cudaStream_t s) {
-    if (d->loopback || d->nranks == 1) return GSW_OK;
-    GSW_NCCL(g_nccl.allGather(buf + (size_t)d->rank * per_rank, buf, per_rank, ncclFloat64, d->comm, s));
-    return GSW_OK;
+
+static void reset_ctl_host(DCtl &c, long long nnz_g, long long n) {
+    c = DCtl{};
+    c.nnz_g = nnz_g;
+    c.Via = n;
+    c.Eia = nnz_g;
+    c.dir = GSW_PUSH;
 }
-static gsw_status reduce_counts(DistState *d, cudaStream_t s) {
-    const int parts = (int)d->parts.size();
-    k_sum_parts<<<1, 32, 0, s>>>(d->cnt, parts);
-    GSW_CUDA(cudaGetLastError());
-    if (!d->loopback && d->nranks > 1)
-        GSW_NCCL(g_nccl.allReduce(d->cnt + 3 * parts, d->cnt + 3 * parts, 3, ncclUint64, ncclSum, d->comm, s));
-    return GSW_OK;
-}
-static gsw_status reduce_dang(DistState *d, cudaStream_t s) {
-    const int parts = (int)d->parts.size();
-    k_sum_dang<<<1, 32, 0, s>>>(d->dang, parts);
-    GSW_CUDA(cudaGetLastError());
-    if (!d->loopback && d->nranks > 1)
-        GSW_NCCL(g_nccl.allReduce(d->dang + parts, d->dang + parts, 1, ncclFloat64, ncclSum, d->comm, s));
+
+static gsw_status read_nnz_g(DistState *d, cudaStream_t s, long long *nnz_g) {
+    GSW_CUDA(cudaMemcpyAsync(nnz_g, &d->ctl->nnz_g, 8, cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
     return GSW_OK;
 }
 
@@ -496,106 +869,89 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
     cudaStream_t s = g->stream;
     if (source < 0 || source >= d->n) { set_error("gsw_bfs: source out of range"); return GSW_EINVAL; }
     if (!depth_out) { set_error("gsw_bfs: depth is NULL"); return GSW_EINVAL; }
+    const int fdir = g->forced.direction;
+    if (fdir != GSW_AUTO && fdir != GSW_PUSH && fdir != GSW_PULL) { set_error("gsw_bfs: bad forced direction"); return GSW_EUNSUPPORTED; }
     const int parts = (int)d->parts.size();
-    const int64_t out_len = d->loopback ? d->n : d->parts[0].nloc;
+    const int64_t out_len = d->mode == DM_LOOPBACK ? d->n : d->parts[0].nloc;
     const bool dev_out = is_device_ptr(depth_out) == 1;
     int *depth = dev_out ? depth_out : (int *)g->scratch;
-    const size_t FBW = (size_t)d->npad / 32;
-    std::vector<gsw_iter_record> recs;
+    const size_t FBB = (size_t)d->npad / 8;
+    long long nnz_g = 0;
+    if (gsw_status e = read_nnz_g(d, s, &nnz_g)) return e;
+    DCtl c0;
+    reset_ctl_host(c0, nnz_g, d->n);
     GSW_CUDA(cudaEventRecord(g->ev0, s));
-    GSW_CUDA(cudaMemsetAsync(d->FB[0], 0, FBW * 4, s));
-    std::vector<BfsPartArgs> pa(parts);
+    GSW_CUDA(cudaMemcpyAsync(d->ctl, &c0, sizeof(c0), cudaMemcpyHostToDevice, s));
+    GSW_CUDA(cudaMemsetAsync(d->FB[0], 0, FBB, s));
+    GSW_CUDA(cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * parts, s));
+    std::vector<BfsP> pa(parts);
     for (int p = 0; p < parts; ++p) {
         const DPart &P = d->parts[p];
-        pa[p] = BfsPartArgs{P.roff, P.rcol, P.soff, P.scol, P.vis, depth + (d->loopback ? P.vb : 0), P.vb, P.nloc,
-                            d->npad, nullptr, nullptr, 0, d->cnt + 3 * p};
-        if (P.nloc) k_bfs_init<<<grid_for(P.nloc, g->sms), kBlock, 0, s>>>(pa[p], source);
+        pa[p] = BfsP{P.roff, P.rcol, P.rfirst, P.soff, P.scol, P.vis, depth + (d->mode == DM_LOOPBACK ? P.vb : 0),
+                     P.vb, d->npad, P.nloc, nullptr, nullptr, P.ptasks, P.nptasks, P.ptask_cap, P.loc, d->ctl, 0};
+        k_bfs_init<<<grid_for(std::max(P.nloc, 1), g->sms), kDB, 0, s>>>(pa[p], source, d->FB[0]);
     }
-    k_set_bit<<<1, 1, 0, s>>>(d->FB[0], source);
     GSW_CUDA(cudaGetLastError());
-    // global features of level 0: Va = 1, Ea = deg(source)
-    unsigned long long tot[3] = {1, 0, 0};
-    {
-        // degree of the source: row length in the owning partition (host read of two offsets)
-        const int owner = d->loopback ? (int)(source / d->S) : -1;
-        unsigned long long dsrc = 0;
-        if (d->loopback || source / d->S == d->rank) {
-            const DPart &P = d->parts[d->loopback ? owner : 0];
-            uint32_t o[2];
-            GSW_CUDA(cudaMemcpyAsync(o, P.roff + (source - P.vb), 8, cudaMemcpyDeviceToHost, s));
-            GSW_CUDA(cudaStreamSynchronize(s));
-            dsrc = o[1] - o[0];
-        }
-        GSW_CUDA(cudaMemsetAsync(d->cnt, 0, 8 * 3 * (parts + 1), s));
-        GSW_CUDA(cudaMemcpyAsync(d->cnt + 1, &dsrc, 8, cudaMemcpyHostToDevice, s));
-        gsw_status r = reduce_counts(d, s);
-        if (r != GSW_OK) return r;
-        GSW_CUDA(cudaMemcpyAsync(tot, d->cnt + 3 * parts, 24, cudaMemcpyDeviceToHost, s));
-        GSW_CUDA(cudaStreamSynchronize(s));
-        tot[0] = 1;
-    }
-    long long Via = d->n - 1, Eia = (long long)g->g.nnz;   // per rank nnz is local: use the global sum below
-    {
-        // global nnz = sum of owned nnz over ranks
-        unsigned long long loc = 0;
-        for (auto &P : d->parts) loc += P.nnz;
-        GSW_CUDA(cudaMemsetAsync(d->cnt, 0, 8 * 3 * (parts + 1), s));
-        GSW_CUDA(cudaMemcpyAsync(d->cnt, &loc, 8, cudaMemcpyHostToDevice, s));
-        gsw_status r = reduce_counts(d, s);
-        if (r != GSW_OK) return r;
-        unsigned long long gn[3];
-        GSW_CUDA(cudaMemcpyAsync(gn, d->cnt + 3 * parts, 24, cudaMemcpyDeviceToHost, s));
-        GSW_CUDA(cudaStreamSynchronize(s));
-        Eia = (long long)gn[0] - (long long)tot[1];
-    }
-    unsigned long long edges_total = 0, bytes = 0;
+    if (gsw_status e = ex_allgather(d, d->FB[0], 1, s)) return e;      // the owner's source bit
+    // level-0 features (Va = 1, Ea = deg(source)) through the same exchange, then the decision
+    if (gsw_status e = ex_reduce(d, s)) return e;
+    k_bfs_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, -1, d->n, fdir);
+    GSW_CUDA(cudaGetLastError());
+    const int grid = g->sms * 8;
     int t = 0;
     for (;; ++t) {
-        const long long Va = (long long)tot[0], Ea = (long long)tot[1];
-        if (Va == 0) break;
-        if (t > 0) { Via -= Va; Eia -= Ea; }
-        // same direction split as the single-GPU selector (select.cuh, R6)
-        int dir = ((double)Ea * 16.0 > (double)Eia && (double)Va * 2048.0 > (double)d->n) ? GSW_PULL : GSW_PUSH;
-        if (g->forced.direction != GSW_AUTO) dir = g->forced.direction;
         unsigned *fb = d->FB[t & 1], *nfb = d->FB[(t + 1) & 1];
-        GSW_CUDA(cudaMemsetAsync(nfb, 0, FBW * 4, s));
-        GSW_CUDA(cudaMemsetAsync(d->cnt, 0, 8 * 3 * (parts + 1), s));
+        GSW_CUDA(cudaMemsetAsync(nfb, 0, FBB, s));
         for (int p = 0; p < parts; ++p) {
-            BfsPartArgs a = pa[p];
+            BfsP a = pa[p];
             a.fb = fb; a.nfb = nfb; a.lvl = t;
             if (!a.nloc) continue;
-            if (dir == GSW_PUSH) k_bfs_push<<<g->sms * 8, kBlock, 0, s>>>(a);
-            else k_bfs_pull<<<g->sms * 8, kBlock, 0, s>>>(a);
+            GSW_CUDA(cudaMemsetAsync(a.ntasks, 0, 4, s));
+            k_bfs_push<<<grid, kDB, 0, s>>>(a);
+            k_bfs_push_heavy<<<grid, kDB, 0, s>>>(a);
+            k_bfs_pull<<<grid, kDB, 0, s>>>(a);
         }
         GSW_CUDA(cudaGetLastError());
-        gsw_status r = allgather_u32(d, nfb, (size_t)d->S / 32, s);
-        if (r != GSW_OK) return r;
-        r = reduce_counts(d, s);
-        if (r != GSW_OK) return r;
-        gsw_iter_record rec{};
-        rec.iteration = t; rec.direction = dir; rec.format = GSW_BITMAP;
-        rec.load_balance = dir == GSW_PULL ? GSW_LB_THREAD : GSW_LB_WM; rec.fusion = GSW_FUSED;
-        rec.Va = Va; rec.Ea = Ea; rec.Via = Via; rec.Eia = Eia;
-        GSW_CUDA(cudaMemcpyAsync(tot, d->cnt + 3 * parts, 24, cudaMemcpyDeviceToHost, s));
-        GSW_CUDA(cudaStreamSynchronize(s));
-        rec.edges = (long long)tot[2];
-        edges_total += tot[2];
-        bytes += dir == GSW_PUSH ? 12ull * Va + 4ull * tot[2] + 8ull * tot[0]
-                                 : (unsigned long long)d->n / 4 + 4ull * tot[2] + 4ull * tot[0] + 8ull * Via;
-        recs.push_back(rec);
+        if (gsw_status e = ex_allgather(d, nfb, 1, s)) return e;
+        if (gsw_status e = ex_reduce(d, s)) return e;
+        k_bfs_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, t, d->n, fdir);
+        GSW_CUDA(cudaGetLastError());
+        bool stop = false;
+        if (gsw_status e = poll_done(d, t, s, &stop)) return e;
+        if (stop || t + 1 >= kMaxLevels) break;
     }
     GSW_CUDA(cudaEventRecord(g->ev1, s));
     if (!dev_out) GSW_CUDA(cudaMemcpyAsync(depth_out, depth, (size_t)out_len * 4, cudaMemcpyDeviceToHost, s));
+    DCtl cend;
+    GSW_CUDA(cudaMemcpyAsync(&cend, d->ctl, sizeof(cend), cudaMemcpyDeviceToHost, s));
     GSW_CUDA(cudaStreamSynchronize(s));
+    const int levels = std::min(cend.t, kMaxLevels);     // levels with a non-empty active set
+    std::vector<DRec> h(levels);
+    if (levels) GSW_CUDA(cudaMemcpy(h.data(), d->recs, sizeof(DRec) * levels, cudaMemcpyDeviceToHost));
     if (st) {
         float ms = 0.f;
         GSW_CUDA(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
-        st->iterations = t;
+        unsigned long long edges = 0, bytes = 0;
+        for (int i = 0; i < levels; ++i) {
+            const unsigned long long Va = h[i].Va, next = i + 1 < levels ? (unsigned long long)h[i + 1].Va : 0ull;
+            edges += h[i].edges;
+            // SURVEY 8(d) D0, summed over the ranks: push 12|F| + 4E + 8|F'|, pull N/4 + 8|U| + 4S + 4|F'|
+            bytes += h[i].dir == GSW_PUSH ? 12ull * Va + 4ull * h[i].edges + 8ull * next
+                                          : (unsigned long long)d->n / 4 + 8ull * (unsigned long long)std::max(0LL, h[i].Via) +
+                                                4ull * h[i].edges + 4ull * next;
+            if (st->records && i < st->max_records) {
+                gsw_iter_record &r = st->records[i];
+                r = gsw_iter_record{};
+                r.iteration = i; r.direction = h[i].dir; r.format = GSW_BITMAP;
+                r.load_balance = h[i].dir == GSW_PULL ? GSW_LB_THREAD : GSW_LB_TWC; r.fusion = GSW_FUSED;
+                r.Va = h[i].Va; r.Ea = h[i].Ea; r.Via = h[i].Via; r.Eia = h[i].Eia; r.edges = h[i].edges;
+                r.ctas = grid;
+            }
+        }
+        st->iterations = levels;
         st->gpu_ms = ms;
-        st->edges_touched = (int64_t)edges_total;
+        st->edges_touched = (int64_t)edges;
         st->bytes_alg = (int64_t)bytes;
-        if (st->records && st->max_records > 0)
-            std::memcpy(st->records, recs.data(), sizeof(gsw_iter_record) * std::min<size_t>(recs.size(), st->max_records));
     }
     return GSW_OK;
 }
@@ -606,43 +962,38 @@ gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out,
     cudaStream_t s = g->stream;
     if (!rank_out || iters < 0 || !(damping >= 0.0 && damping <= 1.0)) { set_error("gsw_pr: bad arguments"); return GSW_EINVAL; }
     const int parts = (int)d->parts.size();
-    const int64_t out_len = d->loopback ? d->n : d->parts[0].nloc;
+    const int64_t out_len = d->mode == DM_LOOPBACK ? d->n : d->parts[0].nloc;
     const bool dev_out = is_device_ptr(rank_out) == 1;
     double *out = dev_out ? rank_out : (double *)g->scratch;
     const double invN = 1.0 / (double)d->n;
+    float *C[2] = {reinterpret_cast<float *>(d->rep[0]), reinterpret_cast<float *>(d->rep[1])};
     GSW_CUDA(cudaEventRecord(g->ev0, s));
-    GSW_CUDA(cudaMemsetAsync(d->dang, 0, 8 * (parts + 1), s));
-    GSW_CUDA(cudaMemsetAsync(d->contrib[0], 0, (size_t)d->npad * 8, s));
-    for (int p = 0; p < parts; ++p) {
+    GSW_CUDA(cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * parts, s));
+    GSW_CUDA(cudaMemsetAsync(C[0], 0, (size_t)d->npad * 4, s));
+    auto args = [&](int p, const float *cur, float *next, bool last) {
         const DPart &P = d->parts[p];
-        PrPartArgs a{P.roff, P.rcol, P.vb, P.nloc, nullptr, d->contrib[0], nullptr, d->dang + p,
-                     iters == 0 ? out + (d->loopback ? P.vb : 0) : nullptr, 0.0, damping, invN};
-        if (P.nloc) k_pr_init<<<grid_for(P.nloc, g->sms), kBlock, 0, s>>>(a);
-    }
+        return PrP{P.roff, P.rcol, P.vb, P.nloc, cur, next, last ? out + (d->mode == DM_LOOPBACK ? P.vb : 0) : nullptr,
+                   P.chunks, P.nchunks, P.psum, P.loc, d->ctl, damping, invN};
+    };
+    for (int p = 0; p < parts; ++p)
+        k_pr_init<<<grid_for(std::max(d->parts[p].nloc, 1), g->sms), kDB, 0, s>>>(args(p, nullptr, C[0], iters == 0));
     GSW_CUDA(cudaGetLastError());
-    gsw_status r = allgather_f64(d, d->contrib[0], (size_t)d->S, s);
-    if (r != GSW_OK) return r;
-    r = reduce_dang(d, s);
-    if (r != GSW_OK) return r;
+    if (gsw_status e = ex_allgather(d, C[0], 4, s)) return e;
+    if (gsw_status e = ex_reduce(d, s)) return e;
+    const int grid = g->sms * 8;
     unsigned long long nnz_loc = 0;
     for (auto &P : d->parts) nnz_loc += P.nnz;
     for (int t = 0; t < iters; ++t) {
-        const double *cur = d->contrib[t & 1];
-        double *next = d->contrib[(t + 1) & 1];
-        // D_t sits at dang[parts]; the per-part accumulators are reused for D_{t+1}
-        GSW_CUDA(cudaMemsetAsync(d->dang, 0, 8 * parts, s));
+        GSW_CUDA(cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * parts, s));
         for (int p = 0; p < parts; ++p) {
-            const DPart &P = d->parts[p];
-            PrPartArgs a{P.roff, P.rcol, P.vb, P.nloc, cur, next, d->dang + parts, d->dang + p,
-                         t == iters - 1 ? out + (d->loopback ? P.vb : 0) : nullptr, (1.0 - damping) * invN, damping, invN};
-            // dtot is read before the per-part accumulators are summed into it by reduce_dang below
-            if (P.nloc) k_pr_iter<<<g->sms * 8, kBlock, 0, s>>>(a);
+            if (!d->parts[p].nloc) continue;
+            const PrP a = args(p, C[t & 1], C[(t + 1) & 1], t == iters - 1);
+            k_pr_heavy<<<grid, kDB, 0, s>>>(a);
+            k_pr_rows<<<grid, kDB, 0, s>>>(a);
         }
         GSW_CUDA(cudaGetLastError());
-        r = allgather_f64(d, next, (size_t)d->S, s);
-        if (r != GSW_OK) return r;
-        r = reduce_dang(d, s);
-        if (r != GSW_OK) return r;
+        if (gsw_status e = ex_allgather(d, C[(t + 1) & 1], 4, s)) return e;
+        if (gsw_status e = ex_reduce(d, s)) return e;
     }
     GSW_CUDA(cudaEventRecord(g->ev1, s));
     if (!dev_out) GSW_CUDA(cudaMemcpyAsync(rank_out, out, (size_t)out_len * 8, cudaMemcpyDeviceToHost, s));
@@ -653,13 +1004,78 @@ gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out,
         st->iterations = iters;
         st->gpu_ms = ms;
         st->edges_touched = (int64_t)nnz_loc * iters;
-        st->bytes_alg = (int64_t)((4ull * nnz_loc + 20ull * (unsigned long long)out_len) * iters);
+        // per iteration: 4 B per owned in-edge column + owned rows (offsets 4 B, contribution
+        // write 4 B) + the fp32 all-gather (N * 4 B received); gathers of the replicated
+        // contributions are L2 probes (D0) at C3 sizes
+        st->bytes_alg = (int64_t)((4ull * nnz_loc + 8ull * (unsigned long long)out_len + 4ull * d->npad) * iters);
     }
     return GSW_OK;
 }
 
-size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, bool own_copy) {
-    return dist_bytes(n, nnz, nranks, nparts, own_copy);
+// ------------------------------------------------------------------ distributed CC
+gsw_status dist_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
+    DistState *d = g->dist;
+    cudaStream_t s = g->stream;
+    if (!label_out) { set_error("gsw_cc: label is NULL"); return GSW_EINVAL; }
+    const int parts = (int)d->parts.size();
+    const int64_t out_len = d->mode == DM_LOOPBACK ? d->n : d->parts[0].nloc;
+    const bool dev_out = is_device_ptr(label_out) == 1;
+    int32_t *out = dev_out ? label_out : (int32_t *)g->scratch;
+    long long nnz_g = 0;
+    if (gsw_status e = read_nnz_g(d, s, &nnz_g)) return e;
+    DCtl c0;
+    reset_ctl_host(c0, nnz_g, d->n);
+    GSW_CUDA(cudaEventRecord(g->ev0, s));
+    GSW_CUDA(cudaMemcpyAsync(d->ctl, &c0, sizeof(c0), cudaMemcpyHostToDevice, s));
+    GSW_CUDA(cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * parts, s));
+    for (int p = 0; p < parts; ++p) {
+        const DPart &P = d->parts[p];
+        k_cc_init<<<grid_for(d->npad, g->sms), kDB, 0, s>>>(d->rep[0], p == 0 ? d->npad : 0,
+                                                            reinterpret_cast<uint32_t *>(P.psum), P.nloc);
+    }
+    GSW_CUDA(cudaGetLastError());
+    const int grid = g->sms * 8;
+    unsigned long long nnz_loc = 0;
+    for (auto &P : d->parts) nnz_loc += P.nnz;
+    int t = 0;
+    for (;; ++t) {
+        const uint32_t *cur = d->rep[t & 1];
+        uint32_t *next = d->rep[(t + 1) & 1];
+        for (int p = 0; p < parts; ++p) {
+            const DPart &P = d->parts[p];
+            if (!P.nloc) continue;
+            const CcP a{P.roff, P.rcol, P.vb, P.nloc, cur, next, out + (d->mode == DM_LOOPBACK ? P.vb : 0), P.chunks,
+                        P.nchunks, reinterpret_cast<uint32_t *>(P.psum), P.loc, d->ctl};
+            k_cc_heavy<<<grid, kDB, 0, s>>>(a);
+            k_cc_rows<<<grid, kDB, 0, s>>>(a);
+        }
+        GSW_CUDA(cudaGetLastError());
+        if (gsw_status e = ex_allgather(d, next, 4, s)) return e;
+        if (gsw_status e = ex_reduce(d, s)) return e;
+        k_cc_decide<<<1, 32, 0, s>>>(d->ctl, d->locs, parts, t);
+        GSW_CUDA(cudaGetLastError());
+        bool stop = false;
+        if (gsw_status e = poll_done(d, t, s, &stop)) return e;
+        if (stop || t + 1 >= kMaxLevels) break;
+    }
+    GSW_CUDA(cudaEventRecord(g->ev1, s));
+    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(label_out, out, (size_t)out_len * 4, cudaMemcpyDeviceToHost, s));
+    DCtl cend;
+    GSW_CUDA(cudaMemcpyAsync(&cend, d->ctl, sizeof(cend), cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    if (st) {
+        float ms = 0.f;
+        GSW_CUDA(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+        st->iterations = cend.t;                       // iterations until nothing changed
+        st->gpu_ms = ms;
+        st->edges_touched = (int64_t)nnz_loc * cend.t;
+        st->bytes_alg = (int64_t)((4ull * nnz_loc + 12ull * (unsigned long long)out_len + 4ull * d->npad) * cend.t);
+    }
+    return GSW_OK;
+}
+
+size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, int mode) {
+    return dist_bytes(n, nnz, nranks, nparts, mode);
 }
 
 gsw_status dist_unique_id(void *id128) {

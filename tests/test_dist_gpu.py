@@ -1,5 +1,7 @@
 """Multi-GPU path on one GPU: loopback partitions (the same partitioned kernels as
-NCCL mode, exchange in device memory) and NCCL mode with one rank.  BFS bit-exact, PR <= 1e-5."""
+NCCL mode, exchange in device memory), NCCL mode with one rank (the collectives really run), and
+the host-staged backend with 2-3 processes sharing the GPU over gloo.  BFS and CC bit-exact,
+PR <= 1e-5."""
 import numpy as np
 import pytest
 
@@ -56,8 +58,95 @@ def test_nccl_single_rank(gsw):
     x, _ = D.pr(0.85, 20)
     r = oracle.pr(g, 0.85, 20)
     assert (np.abs(x.cpu().numpy() - r) / r).max() <= 1e-5
+    lab, st = D.cc()
+    assert np.array_equal(lab.cpu().numpy(), oracle.cc(g))
     with pytest.raises(gsw.GswError):
-        D.cc()
+        D.sssp(s)
+    D2 = gsw.DistGraph(off, col, g.n, None, 1, 0)            # private communicator, no id needed
+    d, _ = D2.bfs(s)
+    assert np.array_equal(d.cpu().numpy(), oracle.bfs(g, s))
+
+
+@pytest.mark.parametrize("nparts", [1, 2, 3, 8])
+def test_loopback_cc(gsw, nparts):
+    for g in (gen.rmat(13, seed=4), gen.grid(37, 23), gen.from_edges(300, [(i, i + 1) for i in range(0, 299, 2)]),
+              gen.from_edges(400, [(0, i) for i in range(1, 300)] + [(i, i + 1) for i in range(300, 399)])):
+        lab, st = gsw.PartitionedGraph(g.off, g.col, nparts).cc()
+        assert np.array_equal(lab.cpu().numpy(), oracle.cc(g)), (nparts, g.name)
+
+
+def test_loopback_heavy_rows(gsw):
+    """Rows above the 1024-edge task size (push tasks, PR / CC chunk partials) across parts."""
+    n = 9000
+    edges = [(0, i) for i in range(1, 6000)] + [(1, i) for i in range(3000, 8999, 2)] + [(i, i + 1) for i in range(6000, 8999)]
+    g = gen.from_edges(n, edges)
+    for p in (1, 2, 4):
+        P = gsw.PartitionedGraph(g.off, g.col, p)
+        for force in (None, "push", "pull"):
+            P.force_config(direction=force)
+            for s in (0, 7000, 8998):
+                d, _ = P.bfs(s)
+                assert np.array_equal(d.cpu().numpy(), oracle.bfs(g, s)), (p, force, s)
+        P.force_config()
+        x, _ = P.pr(0.85, 20)
+        r = oracle.pr(g, 0.85, 20)
+        assert (np.abs(x.cpu().numpy() - r) / r).max() <= 1e-5
+        lab, _ = P.cc()
+        assert np.array_equal(lab.cpu().numpy(), oracle.cc(g))
+
+
+def _host_worker(rank, ws, port, q):
+    import os
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    try:
+        dist.init_process_group("gloo", rank=rank, world_size=ws)
+        import paper_conf_ppopp_menglts19_b200 as m
+        g = gen.rmat(13, seed=8)
+        off, col = m.owned_rows(g.off, g.col, rank, ws)
+        S = m.dist_slice(g.n, ws)
+        vb, ve = rank * S, min(g.n, (rank + 1) * S)
+        ex = m.TorchHostExchange()
+        D = m.HostDistGraph(off, col, g.n, ex, rank, device="cuda:0")
+        bad = []
+        for s in gen.sources(g, 3, seed=5):
+            d, st = D.bfs(s, records=64)
+            if not np.array_equal(d.cpu().numpy(), oracle.bfs(g, s)[vb:ve]):
+                bad.append(("bfs", s))
+            Va, _, _, _ = oracle.bfs_features(g, s)
+            if [r["Va"] for r in st["records"]] != Va.tolist():
+                bad.append(("bfs-Va", s))
+        x, _ = D.pr(0.85, 20)
+        r = oracle.pr(g, 0.85, 20)[vb:ve]
+        if (np.abs(x.cpu().numpy() - r) / r).max() > 1e-5:
+            bad.append("pr")
+        lab, _ = D.cc()
+        if not np.array_equal(lab.cpu().numpy(), oracle.cc(g)[vb:ve]):
+            bad.append("cc")
+        q.put((rank, bad))
+        dist.barrier()
+        dist.destroy_process_group()
+    except Exception as e:          # noqa: BLE001
+        q.put((rank, [repr(e)]))
+
+
+@pytest.mark.parametrize("ws", [2, 3])
+def test_host_staged_processes(gsw, ws):
+    """world_size 2 / 3 gloo processes, each driving the library's partitioned kernels on the same
+    GPU through gsw_graph_create_dist_host: owned slices match the oracle."""
+    import random
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 20000 + random.randint(0, 20000)
+    procs = [ctx.Process(target=_host_worker, args=(r, ws, port, q)) for r in range(ws)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=600) for _ in range(ws))
+    for p in procs:
+        p.join(timeout=120)
+    assert all(not v for v in res.values()), res
 
 
 def test_c3_loopback_8(gsw):
