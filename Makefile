@@ -11,7 +11,7 @@ LIB := $(PKG)/libgsw.so
 OBJDIR := build/obj
 OBJ := $(patsubst $(CSRC)/%.cu,$(OBJDIR)/%.o,$(CU))
 
-all: $(LIB) gen/libgswgen.so oracle/liboracle.so
+all: $(LIB) gen/libgswgen.so oracle/liboracle.so cpu_baselines/libompbase.so
 
 $(OBJDIR)/%.o: $(CSRC)/%.cu $(HDR)
 	@mkdir -p $(OBJDIR)
@@ -26,7 +26,10 @@ gen/libgswgen.so: gen/gen.c
 oracle/liboracle.so: oracle/oracle.c
 	gcc -O2 -fopenmp -fPIC -shared -o $@ $< -lm
 
+cpu_baselines/libompbase.so: cpu_baselines/omp_bfs.c
+	gcc -O3 -fopenmp -fPIC -shared -o $@ $<
+
 clean:
-	rm -rf build $(LIB) gen/libgswgen.so oracle/liboracle.so
+	rm -rf build $(LIB) gen/libgswgen.so oracle/liboracle.so cpu_baselines/libompbase.so
 
 .PHONY: all clean

@@ -177,12 +177,19 @@ def cpu_baseline_sample(g, roots, budget_s=12.0):
             "sample": f"{n} BFS roots on the full {g.name} graph, single-threaded oracle.bfs, {secs:.1f} s"}
 
 
-def run_extras(gsw, dev, G3, g3, peak):
+def run_extras(gsw, dev, G3, g3, peak, cpu=True):
     """The other BASELINE.json configs (device time of one autotuned call, best of 3, L2 flushed
-    before each): C3 CC, PageRank (20 iterations, d = 0.85) and Delta-PR (tol 1e-6), C2 SSSP, C4 BC (16 sources)."""
+    before each): C3 CC, PageRank (20 iterations, d = 0.85) and Delta-PR (tol 1e-6), C2 SSSP, C4 BC
+    (16 sources), C1 BFS over 64 roots.  Beside each, the CPU oracle timed on the host cores on a
+    bounded sample of the same workload (SURVEY 8(d) "oracle timing beside it"), and for BFS the
+    OpenMP level-synchronous baseline on all cores (cpu_baselines/)."""
     import torch
     import gen
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    if cpu:
+        import oracle
+        import cpu_baselines
+        oracle.set_threads(0)
 
     def best(fn):
         b = None
@@ -199,11 +206,25 @@ def run_extras(gsw, dev, G3, g3, peak):
         return {"value": value, "unit": unit, "gpu_ms": st["gpu_ms"], "iterations": st["iterations"],
                 "roofline_frac": sane_frac(gbs / peak, unit), "achieved_gbs": gbs}
 
+    def timed(fn):
+        t0 = time.perf_counter()
+        r = fn()
+        return r, time.perf_counter() - t0
+
     out = {}
     st = best(lambda: G3.cc())
     out["C3_cc"] = rec(g3.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
+    if cpu:
+        _, secs = timed(lambda: oracle.cc(g3))
+        out["C3_cc"]["cpu_baseline"] = {"value": g3.nnz / 2 / secs / 1e9, "unit": "GTEPS", "cores": 1,
+                                        "kind": "oracle", "sample": f"whole C3, union-find, {secs:.2f} s"}
     st = best(lambda: G3.pr(0.85, 20))
     out["C3_pr"] = rec(20 / (st["gpu_ms"] * 1e-3), "PR iters/s", st)
+    if cpu:
+        _, secs = timed(lambda: oracle.pr(g3, 0.85, 2))
+        out["C3_pr"]["cpu_baseline"] = {"value": 2 / secs, "unit": "PR iters/s", "cores": oracle.threads(),
+                                        "kind": "oracle", "sample": f"2 fp64 iterations, per-vertex loop over "
+                                                                    f"{oracle.threads()} OpenMP threads, {secs:.2f} s"}
     # Delta-PR (DESIGN R16): tol = 1e-6 in L1; GTEPS over the edges its Expand read
     st = best(lambda: G3.dpr(0.85, 1e-6))
     out["C3_dpr"] = rec(st["edges_touched"] / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS (edges read)", st)
@@ -212,21 +233,47 @@ def run_extras(gsw, dev, G3, g3, peak):
     st = best(lambda: G2.sssp(0))
     out["C2_sssp"] = rec(g2.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
     out["C2_sssp"]["us_per_round"] = st["gpu_ms"] * 1e3 / max(1, st["iterations"])
+    if cpu:
+        _, secs = timed(lambda: oracle.sssp(g2, 0))
+        out["C2_sssp"]["cpu_baseline"] = {"value": g2.nnz / 2 / secs / 1e9, "unit": "GTEPS", "cores": 1,
+                                          "kind": "oracle", "sample": f"binary-heap Dijkstra from vertex 0, {secs:.2f} s "
+                                                                      "(no parallel CPU variant: Dijkstra is serial)"}
     del G2, g2
     g4 = gen.config_graph("C4")
     G4 = gsw.Graph(g4.off, g4.col, device=dev)
     srcs = gen.sources(g4, 16)
     st = best(lambda: G4.bc(srcs))
     out["C4_bc"] = rec(16 * g4.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
+    if cpu:
+        _, secs = timed(lambda: oracle.bc(g4, srcs[:1]))
+        out["C4_bc"]["cpu_baseline"] = {"value": g4.nnz / 2 / secs / 1e9, "unit": "GTEPS", "cores": 1,
+                                        "kind": "oracle", "sample": f"Brandes from 1 of the 16 sources, {secs:.2f} s"}
     del G4, g4
     g1 = gen.config_graph("C1")
     G1 = gsw.Graph(g1.off, g1.col, device=dev)
-    tot_ms, tot_e = 0.0, 0
-    for s in gen.sources(g1, 16):
+    roots1 = gen.sources(g1, 64)
+    rates, tot_ms, tot_e = [], 0.0, 0
+    for s in roots1:
         d, st1 = G1.bfs(s)
+        e = m_cc(g1.deg, d.cpu().numpy())
+        rates.append(e / (st1["gpu_ms"] * 1e-3) / 1e9)
         tot_ms += st1["gpu_ms"]
-        tot_e += m_cc(g1.deg, d.cpu().numpy())
-    out["C1_bfs"] = {"value": tot_e / (tot_ms * 1e-3) / 1e9, "unit": "GTEPS", "gpu_ms_per_root": tot_ms / 16}
+        tot_e += e
+    hm = lambda r: len(r) / sum(1.0 / x for x in r)
+    out["C1_bfs"] = {"value": hm(rates), "unit": "GTEPS (harmonic mean, 64 roots)",
+                     "aggregate_gteps": tot_e / (tot_ms * 1e-3) / 1e9, "gpu_ms_per_root": tot_ms / 64}
+    if cpu:
+        rs, ro = [], []
+        for s in roots1:
+            d, secs = timed(lambda: oracle.bfs(g1, s))
+            rs.append(m_cc(g1.deg, d) / secs / 1e9)
+            d, secs = timed(lambda: cpu_baselines.bfs(g1, s))
+            ro.append(m_cc(g1.deg, d) / secs / 1e9)
+        out["C1_bfs"]["cpu_baseline"] = {"value": hm(rs), "unit": "GTEPS (harmonic mean, 64 roots)", "cores": 1,
+                                         "kind": "oracle", "sample": "the same 64 roots, oracle.bfs"}
+        out["C1_bfs"]["cpu_openmp"] = {"value": hm(ro), "unit": "GTEPS (harmonic mean, 64 roots)",
+                                       "cores": cpu_baselines.threads(), "kind": "openmp level-synchronous BFS",
+                                       "sample": "the same 64 roots, cpu_baselines.bfs"}
     return out
 
 
@@ -474,7 +521,7 @@ def run_gsw(args, ws, rank, local):
     if os.path.exists(tf):
         with open(tf) as f:
             traffic = json.load(f).get("dram_bytes_per_launch")
-    extra = (run_extras(gsw, dev, G, g, peak)
+    extra = (run_extras(gsw, dev, G, g, peak, cpu=not args.no_cpu_baseline)
              if (rank == 0 and ws == 1 and not args.quick and args.workload == "C3") else None)
 
     # ---- e2e: through the public API from pinned host buffers (graph H2D + BFS + depth D2H)

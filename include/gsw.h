@@ -243,6 +243,18 @@ gsw_status gsw_dist_loopback_workspace_size(int64_t n, int64_t nnz, int32_t npar
 gsw_status gsw_graph_create_partitioned(const gsw_csr *csr, int32_t nparts, void *workspace,
                                         size_t ws_bytes, void *cuda_stream, gsw_graph *out);
 
+/* ---------------------------------------------------------------------------------------------
+ * User-programmable front-end (Sec. 4.2, Fig. 11): the paper's
+ * filter / emit / comp / compAtomic functions as a header-only C++ policy template
+ * (include/gsw_app.cuh, gsw::app::run) driven by the same persistent engine, pattern candidates
+ * and selector.  These two entry points are BFS and SSSP written with it (csrc/app.cu); they
+ * return exactly what gsw_bfs / gsw_sssp return (same arguments, outputs and errors), including
+ * under gsw_force_config (direction / format / load balance / fusion; SSSP stepping STATIC /
+ * UNORDERED, otherwise the dynamic law).
+ * ------------------------------------------------------------------------------------------- */
+gsw_status gsw_app_bfs(gsw_graph g, int32_t source, int32_t *depth, gsw_run_stats *stats);
+gsw_status gsw_app_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *stats);
+
 /* Thread-local message for the last non-OK status of this thread. */
 const char *gsw_last_error(void);
 /* Library version string. */

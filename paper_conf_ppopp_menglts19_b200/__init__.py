@@ -194,6 +194,22 @@ class Graph:
                                   ctypes.byref(st)), "gsw_dpr")
         return out, _stats_dict(st, recs)
 
+    def app_bfs(self, source: int, out=None, records: int = 0):
+        """BFS written with the user-programmable front-end (include/gsw_app.cuh, gsw_app_bfs)."""
+        import torch
+        out = self._out(out, torch.int32)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_app_bfs(self._h, int(source), out.data_ptr(), ctypes.byref(st)), "gsw_app_bfs")
+        return out, _stats_dict(st, recs)
+
+    def app_sssp(self, source: int, out=None, records: int = 0):
+        """SSSP written with the user-programmable front-end (include/gsw_app.cuh, gsw_app_sssp)."""
+        import torch
+        out = self._out(out, torch.int32)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_app_sssp(self._h, int(source), out.data_ptr(), ctypes.byref(st)), "gsw_app_sssp")
+        return out, _stats_dict(st, recs)
+
     def bc(self, sources: Sequence[int], out=None, records: int = 0):
         import torch
         out = self._out(out, torch.float64)

@@ -83,6 +83,8 @@ SIGNATURES = {
     "gsw_pr": (ctypes.c_int, [_P, ctypes.c_double, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_dpr": (ctypes.c_int, [_P, ctypes.c_double, ctypes.c_double, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_bc": (ctypes.c_int, [_P, _P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
+    "gsw_app_bfs": (ctypes.c_int, [_P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
+    "gsw_app_sssp": (ctypes.c_int, [_P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_dist_slice": (ctypes.c_int64, [ctypes.c_int64, ctypes.c_int32]),
     "gsw_dist_unique_id": (ctypes.c_int, [_P]),
     "gsw_dist_workspace_size": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32,

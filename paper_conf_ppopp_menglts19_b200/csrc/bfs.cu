@@ -26,6 +26,8 @@ enum { MAT_NONE = 0, MAT_QUEUE = 1, MAT_SQUEUE = 2, MAT_BITMAP = 3 };
 struct BfsArgs {
     DevGraph g;
     const unsigned *iso;
+    const unsigned *iso_c;    // isolated bitmap in caller order (relabeled graphs)
+    int n_init;           // depth entries initialised: all n, or the non-isolated prefix after relabeling
     int src;              // caller id
     int *depth;           // internal order
     int *out;             // caller order (relabeled graphs), else nullptr
@@ -426,8 +428,12 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(const __grid_co
     int *depth = a.depth;
     const Adj adj_out{a.g.off, a.g.col}, adj_in{a.g.in_off, a.g.in_col};
 
+    if (is_book()) rc.ctl->t_start = globaltimer();
     // ---- init: depth, visited map, frontier bitmaps, counters, AS_0 = {src}
-    for (long long v = gtid(); v < n; v += gthreads()) depth[v] = (v == src) ? 0 : -1;
+    // (relabeled symmetric graphs: the isolated vertices are the internal tail and never leave -1;
+    // their depth entries are not written, the caller-order output takes -1 from iso_c)
+    for (long long v = gtid(); v < a.n_init; v += gthreads()) depth[v] = (v == src) ? 0 : -1;
+    if (gtid() == 0) depth[src] = 0;
     for (long long w = gtid(); w < W; w += gthreads()) {
         unsigned x = a.iso[w];
         if (w == (src >> 5)) x |= 1u << (src & 31);
@@ -441,11 +447,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(const __grid_co
         a.q[0][0] = src;
     }
     cta_queue_reset(qs);
-    grid_sync(bar, epoch);
-
-    Book book;
-    const bool solo_allowed = rc.solo_e > 0 && rc.force.direction == GSW_AUTO && rc.force.format == GSW_AUTO &&
-                              rc.force.load_balance == GSW_AUTO && rc.force.fusion == GSW_AUTO;
+    const bool all_auto = rc.force.direction == GSW_AUTO && rc.force.format == GSW_AUTO &&
+                          rc.force.load_balance == GSW_AUTO && rc.force.fusion == GSW_AUTO;
+    const bool solo_allowed = rc.solo_e > 0 && all_auto;
     bool last_small = false;
     long long Via = (long long)n - 1, Eia = (long long)a.g.nnz - dsrc;
     int mat = MAT_SQUEUE;
@@ -454,6 +458,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(const __grid_co
     int prev_dir = GSW_PUSH;
     long long prev_va = 0, prev_via = 0;
     int t = 0;
+    Book book;
+    grid_sync(bar, epoch);
+    if (is_book()) rc.ctl->t_phase = globaltimer();
     for (;; ++t) {
         IterCnt *cur = rc.cnt + (t % 3), *nxt = rc.cnt + ((t + 1) % 3);
         if (is_book()) book_start(book, rc, t, nxt);
@@ -595,8 +602,35 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(const __grid_co
         prev_va = (long long)va;
         prev_via = Via;
     }
-    if (a.out) gather_out(a.out, depth, a.g.inv, n);
-    if (is_book()) book_finish(book, rc, t);
+    if (is_book()) rc.ctl->t_expand = globaltimer();
+    if (a.out) {
+        // caller order: isolated vertices (iso_c) are -1 without touching depth (their entries were
+        // never initialised); the others gather depth[inv[j]], kG loads in flight per thread
+        constexpr int kG = 8;
+        const long long T0 = gtid(), NT = gthreads();
+        for (long long base = T0; base < n; base += kG * NT) {
+            int ix[kG], val[kG];
+            unsigned isw[kG];
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {          // independent loads: the isolated word and inv[j]
+                const long long j = base + k * NT;
+                isw[k] = j < n ? __ldg(a.iso_c + (j >> 5)) : ~0u;
+                ix[k] = j < n ? (int)__ldg(a.g.inv + j) : -1;
+            }
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+                const long long j = base + k * NT;
+                const bool iso = ((isw[k] >> (j & 31)) & 1u) && j != a.src;
+                val[k] = (ix[k] >= 0 && !iso) ? depth[ix[k]] : -1;
+            }
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+                const long long j = base + k * NT;
+                if (j < n) a.out[j] = val[k];
+            }
+        }
+    }
+    if (is_book()) { book_finish(book, rc, t); rc.ctl->t_end = globaltimer(); }
 }
 
 gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stats *st) {
@@ -608,8 +642,12 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     BfsArgs a{};
     a.g = g->g;
     a.iso = g->iso;
+    a.iso_c = g->iso_caller;
     a.src = source;
     const bool relabeled = g->g.inv != nullptr;
+    // relabeled (degree-descending) symmetric graphs keep their isolated vertices as the internal
+    // tail [n - isolated, n): only the prefix needs depth = -1 (the output reads iso_c for the rest)
+    a.n_init = (relabeled && g->symmetric && g->iso_caller) ? (int)(n - g->attrs.isolated) : n;
     a.depth = (dev_out && !relabeled) ? depth_out : (int *)ws.take((size_t)n * 4);
     a.out = relabeled ? (dev_out ? depth_out : (int *)ws.take((size_t)n * 4)) : nullptr;
     a.V = (unsigned *)ws.take((size_t)W * 4);

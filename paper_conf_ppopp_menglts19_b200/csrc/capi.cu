@@ -145,6 +145,16 @@ gsw_status gsw_graph_create(const gsw_csr *csr, const gsw_csr *csc, void *worksp
     int32_t *first = (int32_t *)gws.take((size_t)csr->n * 4 + 4);
     if (!first) { gsw_graph_destroy(g); set_error("workspace too small"); return GSW_ENOMEM; }
     if ((s = build_first_nbr(g, first)) != GSW_OK) { gsw_graph_destroy(g); return s; }
+    if (g->g.inv) {
+        g->iso_caller = (unsigned *)gws.take((size_t)((csr->n + 31) / 32) * 4);
+        if (!g->iso_caller) { gsw_graph_destroy(g); set_error("workspace too small"); return GSW_ENOMEM; }
+    }
+    g->ctl = gws.take(1024);
+    if (!g->ctl || cudaMemsetAsync(g->ctl, 0, 1024, g->stream) != cudaSuccess) {
+        gsw_graph_destroy(g);
+        set_error("workspace too small / control block");
+        return GSW_ENOMEM;
+    }
     void *tmp = (char *)g->scratch + (((csr->n + 1) * 16 + 4096 + 255) & ~int64_t(255));
     if ((s = compute_attrs(g, g->iso, tmp)) != GSW_OK) { gsw_graph_destroy(g); return s; }
     *out = g;

@@ -603,14 +603,14 @@ static gsw_status host_stage(DistState *d, size_t bytes) {
     return GSW_OK;
 }
 
-// in-place all-gather of the rank slices of a replicated buffer (S elements of esize bytes each)
-static gsw_status ex_allgather(DistState *d, void *buf, size_t esize, cudaStream_t s) {
-    const size_t per = (size_t)d->S * esize;
+// in-place all-gather of the rank slices of a replicated buffer: `per` bytes per rank (a frontier
+// bitmap: S/8; per-vertex words: 4 S)
+static gsw_status ex_allgather(DistState *d, void *buf, size_t per, cudaStream_t s) {
     if (d->mode == DM_LOOPBACK) return GSW_OK;                 // the replica is shared by the parts
     if (d->mode == DM_NCCL) {
-        const ncclDataType_t ty = esize == 4 ? ncclUint32 : ncclUint8;
-        const size_t cnt = esize == 4 ? (size_t)d->S : per;
-        GSW_NCCL(g_nccl.allGather((char *)buf + (size_t)d->rank * per, buf, cnt, ty, d->comm, s));
+        const bool words = per % 4 == 0;
+        GSW_NCCL(g_nccl.allGather((char *)buf + (size_t)d->rank * per, buf, words ? per / 4 : per,
+                                  words ? ncclUint32 : ncclUint8, d->comm, s));
         return GSW_OK;
     }
     if (gsw_status e = host_stage(d, per)) return e;
@@ -698,6 +698,16 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
     g->g.n = (int)n;
     g->g.nnz = (uint32_t)rows->nnz;
     auto fail = [&](gsw_status st) { gsw_graph_destroy(g); return st; };
+    // the communicator first: every rank arrives here at about the same time (the graph ingest
+    // below can take seconds at C5 scale, longer than NCCL's bootstrap waits for its peers)
+    if (mode == DM_NCCL) {
+        if (!nccl_load()) return fail(GSW_ENCCL);
+        if (!nccl_id) { set_error("NCCL mode needs the ncclUniqueId"); return fail(GSW_EINVAL); }
+        ncclUniqueId id;
+        std::memcpy(&id, nccl_id, sizeof(id));
+        ncclResult_t r = g_nccl.commInitRank(&d->comm, nranks, id, rank);
+        if (r != ncclSuccess) { set_error(std::string("ncclCommInitRank: ") + g_nccl.errStr(r)); return fail(GSW_ENCCL); }
+    }
     for (auto &ev : d->evs)
         if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "events"));
     if (cudaHostAlloc((void **)&d->hdone, sizeof(int) * (kLookahead + 1), cudaHostAllocDefault) != cudaSuccess)
@@ -793,14 +803,6 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
     g->scratch_bytes = (size_t)d->npad * 8;
     if (!g->scratch) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
     if (cudaStreamSynchronize(s) != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "dist create"));
-    if (mode == DM_NCCL) {
-        if (!nccl_load()) return fail(GSW_ENCCL);
-        if (!nccl_id) { set_error("NCCL mode needs the ncclUniqueId"); return fail(GSW_EINVAL); }
-        ncclUniqueId id;
-        std::memcpy(&id, nccl_id, sizeof(id));
-        ncclResult_t r = g_nccl.commInitRank(&d->comm, nranks, id, rank);
-        if (r != ncclSuccess) { set_error(std::string("ncclCommInitRank: ") + g_nccl.errStr(r)); return fail(GSW_ENCCL); }
-    }
     // global nnz (once): every rank's owned entries, summed by the exchange
     {
         unsigned long long h[kLocStride] = {};
@@ -892,7 +894,7 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
         k_bfs_init<<<grid_for(std::max(P.nloc, 1), g->sms), kDB, 0, s>>>(pa[p], source, d->FB[0]);
     }
     GSW_CUDA(cudaGetLastError());
-    if (gsw_status e = ex_allgather(d, d->FB[0], 1, s)) return e;      // the owner's source bit
+    if (gsw_status e = ex_allgather(d, d->FB[0], (size_t)d->S / 8, s)) return e;      // the owner's source bit
     // level-0 features (Va = 1, Ea = deg(source)) through the same exchange, then the decision
     if (gsw_status e = ex_reduce(d, s)) return e;
     k_bfs_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, -1, d->n, fdir);
@@ -912,7 +914,7 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
             k_bfs_pull<<<grid, kDB, 0, s>>>(a);
         }
         GSW_CUDA(cudaGetLastError());
-        if (gsw_status e = ex_allgather(d, nfb, 1, s)) return e;
+        if (gsw_status e = ex_allgather(d, nfb, (size_t)d->S / 8, s)) return e;
         if (gsw_status e = ex_reduce(d, s)) return e;
         k_bfs_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, t, d->n, fdir);
         GSW_CUDA(cudaGetLastError());
@@ -978,7 +980,7 @@ gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out,
     for (int p = 0; p < parts; ++p)
         k_pr_init<<<grid_for(std::max(d->parts[p].nloc, 1), g->sms), kDB, 0, s>>>(args(p, nullptr, C[0], iters == 0));
     GSW_CUDA(cudaGetLastError());
-    if (gsw_status e = ex_allgather(d, C[0], 4, s)) return e;
+    if (gsw_status e = ex_allgather(d, C[0], (size_t)d->S * 4, s)) return e;
     if (gsw_status e = ex_reduce(d, s)) return e;
     const int grid = g->sms * 8;
     unsigned long long nnz_loc = 0;
@@ -992,7 +994,7 @@ gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out,
             k_pr_rows<<<grid, kDB, 0, s>>>(a);
         }
         GSW_CUDA(cudaGetLastError());
-        if (gsw_status e = ex_allgather(d, C[(t + 1) & 1], 4, s)) return e;
+        if (gsw_status e = ex_allgather(d, C[(t + 1) & 1], (size_t)d->S * 4, s)) return e;
         if (gsw_status e = ex_reduce(d, s)) return e;
     }
     GSW_CUDA(cudaEventRecord(g->ev1, s));
@@ -1050,7 +1052,7 @@ gsw_status dist_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
             k_cc_rows<<<grid, kDB, 0, s>>>(a);
         }
         GSW_CUDA(cudaGetLastError());
-        if (gsw_status e = ex_allgather(d, next, 4, s)) return e;
+        if (gsw_status e = ex_allgather(d, next, (size_t)d->S * 4, s)) return e;
         if (gsw_status e = ex_reduce(d, s)) return e;
         k_cc_decide<<<1, 32, 0, s>>>(d->ctl, d->locs, parts, t);
         GSW_CUDA(cudaGetLastError());

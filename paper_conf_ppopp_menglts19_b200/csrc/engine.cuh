@@ -25,10 +25,11 @@ struct Hist {
 struct Ctl {
     unsigned arrive, gen, err, iters;
     unsigned long long edges_total, bytes_alg;
-    unsigned long long t_start, t_phase, t_expand;
+    unsigned long long t_start, t_phase, t_expand;   // kernel entry, loop start, output start (%globaltimer)
     float sum_tf, sum_te;
     unsigned stop;
-    unsigned pad[5];
+    unsigned pad;
+    unsigned long long t_end;                        // kernel end (GSW_PHASES=1 prints the split)
 };
 
 struct RunCommon {

@@ -19,6 +19,16 @@ __global__ void k_offsets_to_u32(const int64_t *in, uint32_t *out, long long n1)
     for (long long i = gtid(); i < n1; i += gthreads()) out[i] = (uint32_t)in[i];
 }
 
+// caller-order copy of the isolated bitmap: bit j = isolated(inv[j]) (padding bits set)
+__global__ void k_iso_caller(const uint32_t *inv, const unsigned *iso, int n, unsigned *isoc, int W) {
+    for (long long w = gwarp(); w < W; w += gwarps()) {
+        const int j = (int)(w * 32 + lane_id());
+        bool b = true;
+        if (j < n) { const uint32_t v = inv[j]; b = (iso[v >> 5] >> (v & 31)) & 1u; }
+        const unsigned m = __ballot_sync(0xffffffffu, b);
+        if (lane_id() == 0) isoc[w] = m;
+    }
+}
 // isolated bitmap: bit v = 1 if deg(v) == 0 or v >= n (padding bits)
 __global__ void k_isolated_bitmap(const uint32_t *off, int n, unsigned *iso, int W) {
     for (long long w = gwarp(); w < W; w += gwarps()) {
@@ -150,6 +160,8 @@ size_t graph_bytes(int64_t n, int64_t nnz, int has_w, int has_csc) {
     add(W * 4);  // isolated bitmap
     add(n * 4); add(n * 4);  // relabeling: perm, inv
     add(n * 4);              // first in-neighbour
+    add(W * 4);              // isolated bitmap in caller order
+    add(1024);               // persistent-kernel control block
     return b;
 }
 
@@ -208,7 +220,11 @@ gsw_status compute_attrs(gsw_graph g, unsigned *iso_bitmap, void *tmp) {
     const DevGraph &G = g->g;
     int n = G.n;
     int W = (n + 31) / 32;
-    k_isolated_bitmap<<<grid_for((long long)W * 32, g->sms), kBlock, 0, g->stream>>>(G.off, n, iso_bitmap, W);
+    // "isolated" for the traversals = no in-edges (never discovered; pre-marked visited); for the
+    // symmetric inputs of every config that is degree 0 (Table 1's isolated count, k_attrs)
+    k_isolated_bitmap<<<grid_for((long long)W * 32, g->sms), kBlock, 0, g->stream>>>(G.in_off, n, iso_bitmap, W);
+    if (G.inv && g->iso_caller)
+        k_iso_caller<<<grid_for((long long)W * 32, g->sms), kBlock, 0, g->stream>>>(G.inv, iso_bitmap, n, g->iso_caller, W);
     AttrAcc *acc = (AttrAcc *)tmp;
     AttrAcc init{};
     init.mind = 0xffffffffu;

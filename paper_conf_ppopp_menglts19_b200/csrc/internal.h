@@ -67,7 +67,11 @@ struct gsw_graph_s {
     cudaStream_t stream = nullptr;
     int device = 0, sms = 0;
     gsw_config forced{};
-    unsigned *iso = nullptr;      // isolated-vertex bitmap (deg 0 or padding), W words
+    unsigned *iso = nullptr;      // isolated-vertex bitmap (no in-edges, or padding), W words
+    unsigned *iso_caller = nullptr;  // the same bits in caller order (relabeled graphs), W words
+    void *ctl = nullptr;          // the persistent kernels' control block (grid barrier word,
+                                  // run totals), zeroed once at create: runs need no reset
+                                  // (the flip-bit barrier works from any counter value)
     // workspace regions
     char *ws = nullptr;
     size_t ws_bytes = 0;

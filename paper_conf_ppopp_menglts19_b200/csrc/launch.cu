@@ -1,5 +1,6 @@
 // launch.cu -- persistent cooperative launch + run bookkeeping shared by all algorithms.
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <map>
 #include <mutex>
@@ -36,7 +37,9 @@ static long long env_ll(const char *name, long long dflt) {
 
 gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li) {
     li.grid = g->sms * blocks_per_sm(kernel);
-    rc.ctl = (Ctl *)ws.take(sizeof(Ctl));
+    static_assert(sizeof(Ctl) <= 1024, "control block fits the handle's slot");
+    const bool own_ctl = g->ctl != nullptr;   // handle-owned block: zeroed at create, never reset
+    rc.ctl = own_ctl ? (Ctl *)g->ctl : (Ctl *)ws.take(sizeof(Ctl));
     rc.cnt = (IterCnt *)ws.take(3 * sizeof(IterCnt));
     rc.hist = (Hist *)ws.take(sizeof(Hist) * kMaxHist);
     rc.rec = (gsw_iter_record *)ws.take(sizeof(gsw_iter_record) * kMaxHist);
@@ -57,7 +60,7 @@ gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCom
     // solo tier (CTA 0 alone for tiny active sets); GSW_SOLO_E / GSW_SOLO_V override (calibration)
     rc.solo_e = env_ll("GSW_SOLO_E", kSoloE);
     rc.solo_v = env_ll("GSW_SOLO_V", kSoloV);
-    GSW_CUDA(cudaMemsetAsync(rc.ctl, 0, sizeof(Ctl), g->stream));
+    if (!own_ctl) GSW_CUDA(cudaMemsetAsync(rc.ctl, 0, sizeof(Ctl), g->stream));
     return GSW_OK;
 }
 
@@ -73,6 +76,9 @@ gsw_status finish_run(gsw_graph g, const RunCommon &rc, const LaunchInfo &li, gs
     GSW_CUDA(cudaMemcpyAsync(&h, rc.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, g->stream));
     GSW_CUDA(cudaStreamSynchronize(g->stream));
     if (h.err) { set_error("device error code " + std::to_string(h.err)); return GSW_ECUDA; }
+    if (h.t_end && std::getenv("GSW_PHASES"))
+        std::fprintf(stderr, "gsw phases: init %.2f us, iterations %.2f us, output %.2f us\n",
+                     (h.t_phase - h.t_start) * 1e-3, (h.t_expand - h.t_phase) * 1e-3, (h.t_end - h.t_expand) * 1e-3);
     if (st) {
         float ms = 0.f;
         GSW_CUDA(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
