@@ -29,6 +29,15 @@ oracle/liboracle.so: oracle/oracle.c
 cpu_baselines/libompbase.so: cpu_baselines/omp_bfs.c
 	gcc -O3 -fopenmp -fPIC -shared -o $@ $<
 
+# A/B variant of the library with another number of resident CTAs per SM for the persistent
+# kernels (register budget 65536 / (256 * MINB)): build/var_m$(MINB)/libgsw.so, loaded with
+# GSW_LIB_PATH=... for side-by-side timing
+MINB ?= 3
+variant:
+	@mkdir -p build/var_m$(MINB)
+	$(NVCC) $(NVFLAGS) -DGSW_MINB=$(MINB) -shared -o build/var_m$(MINB)/libgsw.so $(CU) -lcudart -ldl \
+	    2> build/var_m$(MINB)/ptxas.txt || (tail -20 build/var_m$(MINB)/ptxas.txt; exit 1)
+
 clean:
 	rm -rf build $(LIB) gen/libgswgen.so oracle/liboracle.so cpu_baselines/libompbase.so
 

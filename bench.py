@@ -277,6 +277,45 @@ def run_extras(gsw, dev, G3, g3, peak, cpu=True):
     return out
 
 
+def run_c5_extra(gsw, dev, peak, roots_n=2):
+    """C5 (Kronecker scale 26, 2.1e9 entries) on this one GPU, twice: the single-GPU persistent
+    engine (gsw.Graph) and the 1D-partitioned path at p = 1 (gsw.DistGraph: NCCL with one rank,
+    the same kernels and exchange code as bench.py --gpus N), so the N > 1 lines have their p = 1
+    point.  BFS over `roots_n` roots (device span, L2 flushed) and PageRank (20 iterations)."""
+    import torch
+    import gen
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    t0 = time.time()
+    g = gen.config_graph("C5")
+    gen_s = time.time() - t0
+    roots = gen.sources(g, roots_n)
+    deg = g.deg
+    out = {"gen_seconds": gen_s, "n": g.n, "nnz": g.nnz, "roots": roots}
+    for name, make in (("single_gpu", lambda: gsw.Graph(g.off, g.col, device=dev)),
+                       ("partitioned_p1", lambda: gsw.DistGraph(g.off, g.col, g.n, None, 1, 0, device=dev))):
+        G = make()
+        dd = torch.empty(g.n, dtype=torch.int32, device=dev)
+        G.bfs(roots[0], out=dd)                           # warm-up
+        ms, edges, bytes_alg = 0.0, 0, 0
+        for s in roots:
+            flush.fill_(1)
+            torch.cuda.synchronize()
+            _, st = G.bfs(s, out=dd)
+            ms += st["gpu_ms"]
+            bytes_alg += st["bytes_alg"]
+            edges += m_cc(deg, dd.cpu().numpy())
+        flush.fill_(2)
+        torch.cuda.synchronize()
+        _, stp = G.pr(0.85, 20)
+        gbs = bytes_alg / (ms * 1e-3) / 1e9
+        out[name] = {"bfs_gteps": edges / (ms * 1e-3) / 1e9, "bfs_ms_per_root": ms / len(roots),
+                     "bfs_roofline_frac": sane_frac(gbs / peak, f"C5 {name}"), "pr_iters_per_s": 20 / (stp["gpu_ms"] * 1e-3),
+                     "pr_gpu_ms": stp["gpu_ms"]}
+        del G, dd
+        torch.cuda.empty_cache()
+    return out
+
+
 def dist_sources(gsw, off_local, vb, n, count, dev, seed=7):
     """The SURVEY Q12 root stream (gen.sources) on a partitioned graph: candidate k is
     splitmix64((seed << 32) | k) mod n; its owner says whether it has edges; repeats and
@@ -393,9 +432,11 @@ def run_gsw_dist(args, ws, rank, local):
     e2e_ms, e2e_edges = 0.0, 0
     ke = 2
     for k in range(ke):
+        ids = [gsw.dist_unique_id() if rank == 0 else None]       # an ncclUniqueId serves one communicator
+        dist.broadcast_object_list(ids, src=0)
         dist.barrier()
         t0 = time.perf_counter()
-        D2 = gsw.DistGraph(pin_off, pin_col, n, obj[0], ws, rank, device=dev)
+        D2 = gsw.DistGraph(pin_off, pin_col, n, ids[0], ws, rank, device=dev)
         D2.bfs(roots[args.warmup + k], out=host_out)
         e2e_ms += mx((time.perf_counter() - t0) * 1e3)
         e2e_edges += int(sm(int(deg[host_out.numpy()[:D2.out_len] >= 0].sum()))) // 2
@@ -424,9 +465,9 @@ def run_gsw_dist(args, ws, rank, local):
             "timing": "device span of each gsw_bfs call on the library stream (CUDA events), max over ranks",
             "e2e": {"value": e2e_edges / (e2e_ms * 1e-3) / 1e9, "unit": "GTEPS",
                     "h2d_bytes_per_step": int(h2d_all), "d2h_bytes_per_step": int(d2h_all),
-                    "note": "per step, every rank: gsw_graph_create_dist from its pinned host slice (H2D + column-"
-                            "slice build) + gsw_bfs into pinned host depth (D2H); bytes summed over ranks; host wall "
-                            "clock of the slowest rank"},
+                    "note": "per step, every rank: gsw_graph_create_dist from its pinned host slice (NCCL "
+                            "communicator, H2D, column-slice build) + gsw_bfs into pinned host depth (D2H); bytes "
+                            "summed over ranks; host wall clock of the slowest rank"},
             "clocks": cs.summary(), "gen_seconds": gen_s, "create_seconds": create_s,
             "extra": {f"{workload}_pr": {"value": 20 / (pr_ms * 1e-3), "unit": "PR iters/s", "gpu_ms": pr_ms,
                                          "achieved_gbs_per_gpu": pr_bytes / (pr_ms * 1e-3) / 1e9,
@@ -523,6 +564,8 @@ def run_gsw(args, ws, rank, local):
             traffic = json.load(f).get("dram_bytes_per_launch")
     extra = (run_extras(gsw, dev, G, g, peak, cpu=not args.no_cpu_baseline)
              if (rank == 0 and ws == 1 and not args.quick and args.workload == "C3") else None)
+    if extra is not None and not args.no_c5:
+        extra["C5"] = run_c5_extra(gsw, dev, peak)
 
     # ---- e2e: through the public API from pinned host buffers (graph H2D + BFS + depth D2H)
     e2e = None
@@ -598,6 +641,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gsw", choices=["gsw", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-c5", action="store_true", help="skip the C5 (scale 26) single-GPU / p=1 extra")
     ap.add_argument("--quick", action="store_true", help="headline only (skip the other configs)")
     ap.add_argument("--workload", default="C3", choices=["C3", "C5"],
                     help="C3 (default, the north_star's headline) or C5 (R-MAT scale 26, 1 GPU)")

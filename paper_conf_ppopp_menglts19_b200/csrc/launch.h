@@ -12,7 +12,10 @@ struct LaunchInfo {
 };
 
 // Blocks per SM of every persistent kernel (kernels declare __launch_bounds__(kBlock, kMinBlocks)).
-constexpr int kMinBlocks = 4;
+#ifndef GSW_MINB
+#define GSW_MINB 4            // A/B builds: make variant MINB=3 (Makefile)
+#endif
+constexpr int kMinBlocks = GSW_MINB;
 
 gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li);
 gsw_status launch_persistent(gsw_graph g, const void *kernel, void **args, const LaunchInfo &li);

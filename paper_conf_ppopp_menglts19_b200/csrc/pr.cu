@@ -272,6 +272,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
 }
 
 gsw_status run_pr_stream(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st);
+gsw_status run_pr_blocked(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st);
+bool pr_blocked_wanted(gsw_graph g);
 
 gsw_status run_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st) {
     const int n = g->g.n;
@@ -285,6 +287,9 @@ gsw_status run_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_
         const gsw_config &fc = g->forced;
         const int dir = fc.direction != GSW_AUTO ? fc.direction : GSW_PULL;
         const int lb = fc.load_balance != GSW_AUTO ? fc.load_balance : GSW_LB_STRICT;
+        // AUTO on graphs whose contributions overflow L2: the source-blocked gather (pr_blocked.cu)
+        if (fc.direction == GSW_AUTO && fc.load_balance == GSW_AUTO && pr_blocked_wanted(g))
+            return run_pr_blocked(g, damping, iters, rank, st);
         if (dir == GSW_PULL && lb == GSW_LB_STRICT) return run_pr_stream(g, damping, iters, rank, st);
     }
     Workspace ws{g->scratch, g->scratch_bytes, 0};

@@ -8,9 +8,10 @@
 //   * one 1024-thread CTA per SM; the in-edge array is cut into tiles of kTile edges (8 per
 //     thread); tiles are dealt round-robin to CTAs, so work is equal by construction (hub rows
 //     span many tiles, short rows share a tile);
-//   * the tile's row offsets arrive in shared memory by a 1D TMA bulk copy (cp.async.bulk +
-//     mbarrier), double buffered one tile ahead; the column indices of the next tile are
-//     prefetched into registers (streaming loads, 16 B per lane) while the current one is reduced;
+//   * the column indices of the next warp-tile are prefetched into registers (streaming 16-byte
+//     loads, ld.global.cs) while the current one is reduced, together with the first 32 row
+//     offsets and the tile geometry; the remaining row offsets of a tile are staged in a per-warp
+//     shared-memory buffer (plain loads -- an earlier plan for a TMA bulk copy was not kept);
 //   * contributions pr_t(u)/deg_out(u) are stored as fp32 (accumulation stays fp64); the first K
 //     of them -- the highest-degree vertices after graph.cu's degree-ordered relabeling, ~55% of
 //     all gathers on R-MAT -- are cached in shared memory for the whole iteration, the rest are

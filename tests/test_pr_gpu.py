@@ -105,3 +105,18 @@ def test_stream_tiles(gsw, monkeypatch, relabel, cache):
         x, st = G.pr(0.85, iters, records=64)
         _close(x.cpu().numpy(), oracle.pr(g, 0.85, iters))
         assert st["records"][0]["load_balance"] == gsw.LB_STRICT
+
+
+@pytest.mark.parametrize("blocks", ["1", "2", "3", "8"])
+def test_source_blocked(gsw, monkeypatch, blocks):
+    """The source-blocked gather (pr_blocked.cu; AUTO when pr/deg overflows L2, i.e. C5): forced
+    on small graphs with 1-8 source blocks, heavy rows (> 4096 in-edges) as chunk tasks, with
+    and without relabeling, 0 / 1 / 20 iterations."""
+    monkeypatch.setenv("GSW_PR_BLOCKED", "1")
+    monkeypatch.setenv("GSW_PR_BLOCKS", blocks)
+    for g in (_stream_graph(), gen.rmat(13, seed=2), gen.from_edges(10, [(0, 1), (2, 3)])):
+        G = gsw.Graph(g.off, g.col)
+        for iters in (0, 1, 20):
+            x, st = G.pr(0.85, iters)
+            _close(x.cpu().numpy(), oracle.pr(g, 0.85, iters))
+            assert st["iterations"] == iters
