@@ -155,7 +155,7 @@ union BcSmem {
     LbRedSmem pull;
 };
 
-__global__ void __launch_bounds__(kBlock, kMinBlocks) bc_kernel(BcArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocksBc) bc_kernel(BcArgs a) {
     __shared__ BcSmem sm;
     __shared__ uint32_t red[kWarps + 1];
     __shared__ CtaQStore qs;              // staged appends to the BFS stack S
@@ -364,7 +364,7 @@ gsw_status run_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc_
     int *dsrc = (int *)ws.take((size_t)std::max(nsrc, 1) * 4);
     a.sources = dsrc;
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)bc_kernel, a.rc, li);
+    gsw_status s = prepare_common(g, ws, (const void *)bc_kernel, a.rc, li, kMinBlocksBc);
     if (s != GSW_OK) return s;
     if (!a.bc || !a.depth || !a.sigma || !a.omega || !a.dacc || !a.V || !a.S || !a.lvl_off || !a.scan || !a.err || !dsrc ||
         !a.heavy[1] || !a.hblk[1] || !a.heavy_cnt) {

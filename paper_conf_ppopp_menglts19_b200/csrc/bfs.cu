@@ -416,7 +416,7 @@ __device__ __noinline__ void bfs_solo(const BfsArgs &a, SoloSmem &ss, int t, lon
     }
 }
 
-__global__ void __launch_bounds__(kBlock, kMinBlocks) bfs_kernel(const __grid_constant__ BfsArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocksBfs) bfs_kernel(const __grid_constant__ BfsArgs a) {
     __shared__ BfsSmem bsm;
     LbSmem &sm = bsm.lb;
     __shared__ CtaQStore qs;
@@ -657,7 +657,7 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
     a.iso_count = g->attrs.isolated;
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)bfs_kernel, a.rc, li);
+    gsw_status s = prepare_common(g, ws, (const void *)bfs_kernel, a.rc, li, kMinBlocksBfs);
     if (s != GSW_OK) return s;
     // BFS selector: hand-set rules (default) or the learned trees (GSW_SELECTOR=trees)
     if (const char *sel = std::getenv("GSW_SELECTOR")) a.rc.base.selector = std::strcmp(sel, "trees") == 0 ? 1 : 0;

@@ -117,7 +117,7 @@ union CcSmem {
     LbRedSmem pull;
 };
 
-__global__ void __launch_bounds__(kBlock, kMinBlocks) cc_kernel(CcArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocksCc) cc_kernel(CcArgs a) {
     __shared__ CcSmem sm;
     __shared__ uint32_t red[kWarps + 1];
     const RunCommon &rc = a.rc;
@@ -260,7 +260,7 @@ gsw_status run_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     a.hblk = (unsigned *)ws.take((nh + 1) * 4);
     a.heavy_cnt = (unsigned *)ws.take(256);
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)cc_kernel, a.rc, li);
+    gsw_status s = prepare_common(g, ws, (const void *)cc_kernel, a.rc, li, kMinBlocksCc);
     if (s != GSW_OK) return s;
     if (!a.label || !a.chg || !a.fb[2] || !a.q || !a.scan || !a.heavy || !a.hblk || !a.heavy_cnt) { set_error("workspace too small"); return GSW_ENOMEM; }
     void *args[] = {&a};

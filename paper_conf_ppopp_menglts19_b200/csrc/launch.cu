@@ -9,7 +9,7 @@
 
 namespace gsw {
 
-static int blocks_per_sm(const void *kernel) {
+static int blocks_per_sm(const void *kernel, int max_per_sm) {
     static std::mutex mu;
     static std::map<const void *, int> cache;
     std::lock_guard<std::mutex> lk(mu);
@@ -20,7 +20,7 @@ static int blocks_per_sm(const void *kernel) {
         cudaGetLastError();
         nb = 1;
     }
-    nb = std::max(1, std::min(nb, kMinBlocks));
+    nb = std::max(1, std::min(nb, max_per_sm));   // the kernel's launch-bounds minimum (launch.h)
     // optional shared-memory carveout hint (percent), for L1-vs-smem A/B measurements
     if (const char *c = std::getenv("GSW_CARVEOUT")) {
         if (cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, std::atoi(c)) != cudaSuccess)
@@ -35,8 +35,9 @@ static long long env_ll(const char *name, long long dflt) {
     return (v && *v) ? std::atoll(v) : dflt;
 }
 
-gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li) {
-    li.grid = g->sms * blocks_per_sm(kernel);
+gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li,
+                          int max_per_sm) {
+    li.grid = g->sms * blocks_per_sm(kernel, max_per_sm);
     static_assert(sizeof(Ctl) <= 1024, "control block fits the handle's slot");
     const bool own_ctl = g->ctl != nullptr;   // handle-owned block: zeroed at create, never reset
     rc.ctl = own_ctl ? (Ctl *)g->ctl : (Ctl *)ws.take(sizeof(Ctl));

@@ -12,12 +12,23 @@ struct LaunchInfo {
 };
 
 // Blocks per SM of every persistent kernel (kernels declare __launch_bounds__(kBlock, kMinBlocks)).
-#ifndef GSW_MINB
-#define GSW_MINB 4            // A/B builds: make variant MINB=3 (Makefile)
+// Resident CTAs per SM of each persistent kernel (its __launch_bounds__ minimum, hence its
+// register budget 65536 / (256 * k)).  Measured on B200 (profiles/r2/minblocks_ab.txt): the
+// latency-bound level loops of BFS and SSSP run faster with fewer, fatter CTAs (the grid barrier
+// has fewer arrivals and ptxas stops spilling), CC's bandwidth-heavy pulls with more.
+// GSW_MINB=k (make variant MINB=k) forces one value for every kernel (A/B builds).
+constexpr int kMaxBlocksPerSm = 4;
+#ifdef GSW_MINB
+constexpr int kMinBlocks = GSW_MINB, kMinBlocksBfs = GSW_MINB, kMinBlocksSssp = GSW_MINB, kMinBlocksCc = GSW_MINB,
+              kMinBlocksBc = GSW_MINB, kMinBlocksPr = GSW_MINB, kMinBlocksApp = GSW_MINB;
+#else
+constexpr int kMinBlocks = 4;
+constexpr int kMinBlocksBfs = 2, kMinBlocksSssp = 2, kMinBlocksCc = 4, kMinBlocksBc = 4, kMinBlocksPr = 4,
+              kMinBlocksApp = 2;
 #endif
-constexpr int kMinBlocks = GSW_MINB;
 
-gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li);
+gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li,
+                          int max_per_sm);
 gsw_status launch_persistent(gsw_graph g, const void *kernel, void **args, const LaunchInfo &li);
 gsw_status finish_run(gsw_graph g, const RunCommon &rc, const LaunchInfo &li, gsw_run_stats *st);
 

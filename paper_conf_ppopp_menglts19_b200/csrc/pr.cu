@@ -176,7 +176,7 @@ __device__ __forceinline__ void flush_dangling(double v, double *dst) {
     }
 }
 
-__global__ void __launch_bounds__(kBlock, kMinBlocks) pr_kernel(PrArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocksPr) pr_kernel(PrArgs a) {
     __shared__ PrSmem sm;
     __shared__ uint32_t red[kWarps + 1];
     const RunCommon &rc = a.rc;
@@ -309,7 +309,7 @@ gsw_status run_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_
     a.hblk = (unsigned *)ws.take((nh + 1) * 4);
     a.heavy_cnt = (unsigned *)ws.take(256);
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)pr_kernel, a.rc, li);
+    gsw_status s = prepare_common(g, ws, (const void *)pr_kernel, a.rc, li, kMinBlocksPr);
     if (s != GSW_OK) return s;
     if (!a.out || !a.contrib[1] || !a.sum || !a.dsum || !a.scan || !a.heavy || !a.hblk || !a.heavy_cnt) { set_error("workspace too small"); return GSW_ENOMEM; }
     void *args[] = {&a};

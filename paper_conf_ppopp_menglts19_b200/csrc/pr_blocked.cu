@@ -1,6 +1,8 @@
-// pr_blocked.cu -- PageRank pull with the gather blocked by SOURCE range, for graphs whose
-// contribution array does not fit in L2 ("L2 blocking of the PR gather by source
-// range is the B200 lever" at C5, where pr/deg of 67M vertices is 268 MB against a 126 MB L2).
+// pr_blocked.cu -- PageRank pull with row tiers and (optionally) the gather blocked by SOURCE range,
+// for graphs whose contribution array does not fit in L2 ("L2 blocking of the PR
+// gather by source range is the B200 lever" at C5, where pr/deg of 67M vertices is 268 MB against
+// a 126 MB L2).  Measured, the blocking does not pay on B200 (see run_pr_blocked: B = 1 wins), but
+// the row-tiered kernel is 2.35x the edge-tiled stream kernel at C5, so it is AUTO's choice there.
 //
 // Same iteration as pr.cu / pr_stream.cu (reading R7):
 //   pr_{t+1}(v) = (1-d)/N + d * ( sum_{u in N_in(v)} pr_t(u)/deg_out(u) + D_t/N ),  D_t = dangling mass
@@ -212,9 +214,14 @@ gsw_status run_pr_blocked(gsw_graph g, double damping, int32_t iters, double *ra
     int l2 = 0;
     cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, g->device);
     cudaGetLastError();
-    const double budget = std::max(1.0, (double)(l2 > 0 ? l2 : (64 << 20)) / 3.0);   // bytes of contributions per block
-    int B = (int)std::ceil((double)n * 4.0 / budget);
-    if (const char *e = std::getenv("GSW_PR_BLOCKS")) B = std::atoi(e);                  // tests / calibration
+    // Source blocks: measured on C5 (profiles/r2/minblocks_ab_m1_m2_c5pr_blocks.txt, r2k): B = 1
+    // 116 it/s, 2: 108, 3: 101, 4: 96, 6: 87, 8: 79 -- the split reads and the partial's
+    // read-modify-write per pass cost more than the L2 hits of the narrower gather save, so the
+    // default is one block (the row tiers alone are 2.35x the stream kernel at C5: 49 it/s).
+    // GSW_PR_BLOCKS=B keeps the blocked passes selectable (tests, calibration on other GPUs).
+    (void)l2;
+    int B = 1;
+    if (const char *e = std::getenv("GSW_PR_BLOCKS")) B = std::atoi(e);
     B = std::max(1, std::min(B, kMaxBlocks));
     PbArgs a{};
     a.n = n;

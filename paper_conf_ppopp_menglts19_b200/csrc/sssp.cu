@@ -459,7 +459,7 @@ union SsSmem {
 };
 static_assert(sizeof(SsSoloSmem) <= sizeof(LbSmem), "the solo tier must not grow the kernel's shared memory");
 
-__global__ void __launch_bounds__(kBlock, kMinBlocks) sssp_kernel(const __grid_constant__ SsspArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocksSssp) sssp_kernel(const __grid_constant__ SsspArgs a) {
     __shared__ SsSmem sm;
     __shared__ uint32_t red[kWarps + 1];
     __shared__ CtaQStore qs0, qs1;        // staged appends: near queue, far queue
@@ -786,7 +786,7 @@ gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_sta
     a.law = kDefaultLaw;
     if (const char *law = getenv("GSW_SSSP_LAW")) a.law = atoi(law);
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)sssp_kernel, a.rc, li);
+    gsw_status s = prepare_common(g, ws, (const void *)sssp_kernel, a.rc, li, kMinBlocksSssp);
     if (s != GSW_OK) return s;
     if (!a.dist || !a.nb[2] || !a.q[1] || !a.fq[1] || !a.chg || !a.farbit || !a.flen || !a.split || !a.scan) {
         set_error("workspace too small");
