@@ -365,32 +365,46 @@ def run_gsw_dist(args, ws, rank, local):
     import torch.distributed as dist
     import paper_conf_ppopp_menglts19_b200 as gsw
 
+    host_ex = args.exchange == "host"
+    if host_ex:
+        local = 0        # --exchange host: every rank on GPU 0 (tests the N > 1 logic on one GPU)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if "RANK" not in os.environ:
         os.environ.update(RANK="0", WORLD_SIZE="1", LOCAL_RANK="0", MASTER_ADDR="127.0.0.1",
                           MASTER_PORT=str(29500 + os.getpid() % 1000))
-    dist.init_process_group("nccl", device_id=dev)
+    if host_ex:
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("nccl", device_id=dev)
+    rdev = torch.device("cpu") if host_ex else dev        # device of the bench's own reductions
     workload = args.workload if args.workload != "C3" or args.dist_workload_forced else "C5"
     n, vb, off, col, gen_s = partition_input(workload, rank, ws)
     nroots = args.steps + args.warmup
-    roots = dist_sources(gsw, off, vb, n, nroots, dev)
-    obj = [gsw.dist_unique_id() if rank == 0 else None]
-    dist.broadcast_object_list(obj, src=0)
+    roots = dist_sources(gsw, off, vb, n, nroots, rdev)
+    ex = gsw.TorchHostExchange() if host_ex else None
+
+    def make_graph(o, c):
+        if host_ex:
+            return gsw.HostDistGraph(o, c, n, ex, rank, device=dev)
+        ids = [gsw.dist_unique_id() if rank == 0 else None]       # an ncclUniqueId serves one communicator
+        dist.broadcast_object_list(ids, src=0)
+        return gsw.DistGraph(o, c, n, ids[0], ws, rank, device=dev)
+
     t0 = time.time()
-    D = gsw.DistGraph(off, col, n, obj[0], ws, rank, device=dev)
+    D = make_graph(off, col)
     create_s = time.time() - t0
     deg = np.diff(off)
     out = torch.empty(max(D.out_len, 1), dtype=torch.int32, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
     def mx(x):
-        t = torch.tensor([float(x)], device=dev, dtype=torch.float64)
+        t = torch.tensor([float(x)], device=rdev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
     def sm(x):
-        t = torch.tensor([float(x)], device=dev, dtype=torch.float64)
+        t = torch.tensor([float(x)], device=rdev, dtype=torch.float64)
         dist.all_reduce(t)
         return float(t.item())
 
@@ -432,11 +446,9 @@ def run_gsw_dist(args, ws, rank, local):
     e2e_ms, e2e_edges = 0.0, 0
     ke = 2
     for k in range(ke):
-        ids = [gsw.dist_unique_id() if rank == 0 else None]       # an ncclUniqueId serves one communicator
-        dist.broadcast_object_list(ids, src=0)
         dist.barrier()
         t0 = time.perf_counter()
-        D2 = gsw.DistGraph(pin_off, pin_col, n, ids[0], ws, rank, device=dev)
+        D2 = make_graph(pin_off, pin_col)
         D2.bfs(roots[args.warmup + k], out=host_out)
         e2e_ms += mx((time.perf_counter() - t0) * 1e3)
         e2e_edges += int(sm(int(deg[host_out.numpy()[:D2.out_len] >= 0].sum()))) // 2
@@ -455,7 +467,8 @@ def run_gsw_dist(args, ws, rank, local):
                                    f"(slice {gsw.dist_slice(n, ws)}), per-level NCCL bitmap all-gather, roots per "
                                    "SURVEY Q12",
                        "l2": "flushed between steps (256 MiB write outside the timed span)",
-                       "parallelism": f"1D vertex partition x{ws} (NCCL over NVLink)"},
+                       "parallelism": f"1D vertex partition x{ws} " + ("(host-staged exchange over gloo, all ranks on GPU 0: "
+                                                                "a logic test, not a measurement)" if host_ex else "(NCCL over NVLink)")},
             "roofline": {"bound": "hbm", "achieved": per_gpu_gbs, "peak": peak, "unit": "GB/s",
                          "frac": sane_frac(per_gpu_gbs / peak, "dist BFS"), "traffic": None,
                          "peak_source": peak_src,
@@ -648,6 +661,9 @@ def main():
     ap.add_argument("--force-dist", action="store_true", help="run the partitioned NCCL path even at N=1")
     ap.add_argument("--partitioned", action="store_true",
                     help="the 1D vertex-partitioned graph with NCCL exchange (SURVEY 8(e)); default for N > 1")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "host"],
+                    help="partitioned path: NCCL (one GPU per rank) or the host-staged backend over gloo with every "
+                         "rank on GPU 0 (exercises the N > 1 code on one GPU; not a performance number)")
     ap.add_argument("--replicas", action="store_true",
                     help="N > 1: root-sharded replicas of C3 instead of the partitioned C5 (or exercise them at N=1)")
     args = ap.parse_args()

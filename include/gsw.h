@@ -196,9 +196,14 @@ gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc,
  *     the contribution slices (n*4 bytes) + all-reduce of the dangling mass.
  *   CC iteration: min-label propagation with the pointer-jumping shortcut label[label[v]] on the
  *     replicated labels; all-gather of the label slices + all-reduce of the change count.
+ *   SSSP round (weighted graphs): near/far with a static step delta0 (gsw_config.delta0, else
+ *     32*wbar/dbar; forced UNORDERED = Bellman-Ford): the near set is all-gathered as a bitmap,
+ *     frontier vertices relax their column slices into owned distances (atomicMin), and the
+ *     distance slices are all-gathered after every round.
  * The host never waits per iteration (NCCL / loopback): it polls the device's done flag two
- * iterations behind the stream.  Supported on distributed handles: gsw_bfs, gsw_pr, gsw_cc
- * (others return GSW_EUNSUPPORTED); gsw_force_config's direction pins the BFS direction.
+ * iterations behind the stream.  Supported on distributed handles: gsw_bfs, gsw_pr, gsw_cc,
+ * gsw_sssp (others return GSW_EUNSUPPORTED); gsw_force_config's direction pins the BFS direction,
+ * its stepping (UNORDERED) and delta0 the SSSP step.
  * Outputs of NCCL / host-staged handles cover the OWNED slice only; loopback outputs all n.
  * Three exchange backends run the same kernels:
  *   NCCL (one process per GPU; NCCL is dlopen'ed, a missing library gives GSW_ENCCL),
@@ -212,6 +217,10 @@ int64_t gsw_dist_slice(int64_t n, int32_t nranks);
 gsw_status gsw_dist_unique_id(void *id128);
 /* Workspace bytes for a partition of n_global vertices with nnz_owned adjacency entries. */
 gsw_status gsw_dist_workspace_size(int64_t n_global, int64_t nnz_owned, int32_t nranks, size_t *bytes);
+/* The same with edge weights (needed by gsw_sssp on partitioned handles) and/or for loopback mode
+ * (loopback != 0: nnz_owned is the whole graph's nnz, nranks the number of virtual parts). */
+gsw_status gsw_dist_workspace_size_weighted(int64_t n_global, int64_t nnz_owned, int32_t nranks, int32_t has_weights,
+                                            int32_t loopback, size_t *bytes);
 /* NCCL mode (one process per GPU).  owned: the rows of the owned slice -- owned->n = number of
  * owned vertices, row_offsets start at 0, col_indices are GLOBAL ids (symmetric graph).
  * nccl_id128 may be NULL only when nranks == 1 (a private communicator is created; the

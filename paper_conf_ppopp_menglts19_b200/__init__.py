@@ -248,12 +248,13 @@ class DistGraph(_Handle):
     symmetric graph (global column ids).  Collective: every rank constructs it in the same order."""
 
     def __init__(self, owned_offsets, owned_cols, n_global: int, nccl_id: bytes, nranks: int, rank: int,
-                 device: str | int = "cuda", stream=None):
+                 device: str | int = "cuda", stream=None, weights=None):
         import torch
         lib = _lib.load()
         self.device = torch.device(device)
         off = _as(owned_offsets, np.int64, torch.int64)
         col = _as(owned_cols, np.int32, torch.int32)
+        w = None if weights is None else _as(weights, np.uint32, torch.int32)
         self.n = int(n_global)
         self.out_len = int(off.shape[0]) - 1
         self.nnz = int(col.shape[0])
@@ -262,10 +263,11 @@ class DistGraph(_Handle):
             self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
             po, ko, _ = _ptr_of(off)
             pc, kc, _ = _ptr_of(col) if self.nnz else (None, None, False)
-            csr = _lib.gsw_csr(self.out_len, self.nnz, po, pc, None)
+            pw, kw, _ = _ptr_of(w) if w is not None else (None, None, False)
+            csr = _lib.gsw_csr(self.out_len, self.nnz, po, pc, pw)
             nbytes = ctypes.c_size_t()
-            check(lib.gsw_dist_workspace_size(self.n, self.nnz, self.nranks, ctypes.byref(nbytes)),
-                  "gsw_dist_workspace_size")
+            check(lib.gsw_dist_workspace_size_weighted(self.n, self.nnz, self.nranks, int(w is not None), 0,
+                                                       ctypes.byref(nbytes)), "gsw_dist_workspace_size_weighted")
             self.workspace = torch.empty(nbytes.value, dtype=torch.uint8, device=self.device)
             idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
             h = ctypes.c_void_p()
@@ -273,7 +275,7 @@ class DistGraph(_Handle):
                                             self.workspace.data_ptr(), nbytes.value, self.stream.cuda_stream,
                                             ctypes.byref(h)), "gsw_graph_create_dist")
             self._h = h
-            del ko, kc
+            del ko, kc, kw
 
 
 class TorchHostExchange:
@@ -323,12 +325,13 @@ class HostDistGraph(_Handle):
     (a TorchHostExchange) instead of NCCL.  The kernels are the same partitioned kernels."""
 
     def __init__(self, owned_offsets, owned_cols, n_global: int, exchange: "TorchHostExchange", rank: int,
-                 device: str | int = "cuda", stream=None):
+                 device: str | int = "cuda", stream=None, weights=None):
         import torch
         lib = _lib.load()
         self.device = torch.device(device)
         off = _as(owned_offsets, np.int64, torch.int64)
         col = _as(owned_cols, np.int32, torch.int32)
+        w = None if weights is None else _as(weights, np.uint32, torch.int32)
         self.n = int(n_global)
         self.out_len = int(off.shape[0]) - 1
         self.nnz = int(col.shape[0])
@@ -338,10 +341,11 @@ class HostDistGraph(_Handle):
             self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
             po, ko, _ = _ptr_of(off)
             pc, kc, _ = _ptr_of(col) if self.nnz else (None, None, False)
-            csr = _lib.gsw_csr(self.out_len, self.nnz, po, pc, None)
+            pw, kw, _ = _ptr_of(w) if w is not None else (None, None, False)
+            csr = _lib.gsw_csr(self.out_len, self.nnz, po, pc, pw)
             nbytes = ctypes.c_size_t()
-            check(lib.gsw_dist_workspace_size(self.n, self.nnz, self.nranks, ctypes.byref(nbytes)),
-                  "gsw_dist_workspace_size")
+            check(lib.gsw_dist_workspace_size_weighted(self.n, self.nnz, self.nranks, int(w is not None), 0,
+                                                       ctypes.byref(nbytes)), "gsw_dist_workspace_size_weighted")
             self.workspace = torch.empty(nbytes.value, dtype=torch.uint8, device=self.device)
             h = ctypes.c_void_p()
             check(lib.gsw_graph_create_dist_host(ctypes.byref(csr), self.n, ctypes.byref(exchange.struct),
@@ -356,12 +360,14 @@ class PartitionedGraph(_Handle):
     """Loopback mode: `nparts` virtual ranks of the full graph on this GPU, running the same
     partitioned kernels as DistGraph with the exchange done in device memory."""
 
-    def __init__(self, row_offsets, col_indices, nparts: int, device: str | int = "cuda", stream=None):
+    def __init__(self, row_offsets, col_indices, nparts: int, device: str | int = "cuda", stream=None,
+                 weights=None):
         import torch
         lib = _lib.load()
         self.device = torch.device(device)
         off = _as(row_offsets, np.int64, torch.int64)
         col = _as(col_indices, np.int32, torch.int32)
+        w = None if weights is None else _as(weights, np.uint32, torch.int32)
         self.n = int(off.shape[0]) - 1
         self.out_len = self.n
         self.nnz = int(col.shape[0])
@@ -370,24 +376,27 @@ class PartitionedGraph(_Handle):
             self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
             po, ko, _ = _ptr_of(off)
             pc, kc, _ = _ptr_of(col) if self.nnz else (None, None, False)
-            csr = _lib.gsw_csr(self.n, self.nnz, po, pc, None)
+            pw, kw, _ = _ptr_of(w) if w is not None else (None, None, False)
+            csr = _lib.gsw_csr(self.n, self.nnz, po, pc, pw)
             nbytes = ctypes.c_size_t()
-            check(lib.gsw_dist_loopback_workspace_size(self.n, self.nnz, self.nparts, ctypes.byref(nbytes)),
-                  "gsw_dist_loopback_workspace_size")
+            check(lib.gsw_dist_workspace_size_weighted(self.n, self.nnz, self.nparts, int(w is not None), 1,
+                                                       ctypes.byref(nbytes)), "gsw_dist_workspace_size_weighted")
             self.workspace = torch.empty(nbytes.value, dtype=torch.uint8, device=self.device)
             h = ctypes.c_void_p()
             check(lib.gsw_graph_create_partitioned(ctypes.byref(csr), self.nparts, self.workspace.data_ptr(),
                                                    nbytes.value, self.stream.cuda_stream, ctypes.byref(h)),
                   "gsw_graph_create_partitioned")
             self._h = h
-            del ko, kc
+            del ko, kc, kw
 
 
-def owned_rows(row_offsets, col_indices, rank: int, nranks: int):
-    """Rows [rank*S, min(n, (rank+1)*S)) of a CSR as (offsets rebased to 0, global columns)."""
+def owned_rows(row_offsets, col_indices, rank: int, nranks: int, weights=None):
+    """Rows [rank*S, min(n, (rank+1)*S)) of a CSR as (offsets rebased to 0, global columns[, weights])."""
     off = np.asarray(row_offsets, dtype=np.int64)
     n = off.shape[0] - 1
     S = dist_slice(n, nranks)
     vb, ve = min(n, rank * S), min(n, (rank + 1) * S)
     loc = off[vb:ve + 1] - off[vb]
-    return loc, np.asarray(col_indices)[off[vb]:off[ve]]
+    if weights is None:
+        return loc, np.asarray(col_indices)[off[vb]:off[ve]]
+    return loc, np.asarray(col_indices)[off[vb]:off[ve]], np.asarray(weights)[off[vb]:off[ve]]

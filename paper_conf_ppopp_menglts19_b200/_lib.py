@@ -91,6 +91,8 @@ SIGNATURES = {
                                                ctypes.POINTER(ctypes.c_size_t)]),
     "gsw_graph_create_dist": (ctypes.c_int, [ctypes.POINTER(gsw_csr), ctypes.c_int64, _P, ctypes.c_int32,
                                              ctypes.c_int32, _P, ctypes.c_size_t, _P, ctypes.POINTER(_P)]),
+    "gsw_dist_workspace_size_weighted": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                                        ctypes.c_int32, ctypes.POINTER(ctypes.c_size_t)]),
     "gsw_graph_create_dist_host": (ctypes.c_int, [ctypes.POINTER(gsw_csr), ctypes.c_int64,
                                                   ctypes.POINTER(gsw_exchange), ctypes.c_int32, ctypes.c_int32, _P,
                                                   ctypes.c_size_t, _P, ctypes.POINTER(_P)]),

@@ -34,7 +34,8 @@ void dist_destroy(DistState *d);
 gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stats *st);
 gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out, gsw_run_stats *st);
 gsw_status dist_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st);
-size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, int mode);
+gsw_status dist_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_stats *st);
+size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, int mode, bool weighted);
 enum { kModeNccl = 0, kModeLoopback = 1, kModeHost = 2 };   // dist.cu DistMode
 gsw_status dist_unique_id(void *id128);
 
@@ -206,7 +207,7 @@ gsw_status gsw_bfs(gsw_graph g, int32_t source, int32_t *depth, gsw_run_stats *s
 
 gsw_status gsw_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
-    if (gsw_status s = no_dist(g, "gsw_sssp")) return s;
+    if (g->dist) return dist_sssp(g, source, dist, stats);
     return run_sssp(g, source, dist, stats);
 }
 
@@ -240,13 +241,21 @@ gsw_status gsw_dist_unique_id(void *id128) { return dist_unique_id(id128); }
 
 gsw_status gsw_dist_workspace_size(int64_t n_global, int64_t nnz_owned, int32_t nranks, size_t *bytes) {
     if (!bytes || n_global <= 0 || nnz_owned < 0 || nranks < 1) { set_error("gsw_dist_workspace_size: bad arguments"); return GSW_EINVAL; }
-    *bytes = dist_workspace(n_global, nnz_owned, nranks, 1, kModeNccl);
+    *bytes = dist_workspace(n_global, nnz_owned, nranks, 1, kModeNccl, false);
+    return GSW_OK;
+}
+
+gsw_status gsw_dist_workspace_size_weighted(int64_t n_global, int64_t nnz_owned, int32_t nranks, int32_t has_weights,
+                                            int32_t loopback, size_t *bytes) {
+    if (!bytes || n_global <= 0 || nnz_owned < 0 || nranks < 1) { set_error("gsw_dist_workspace_size_weighted: bad arguments"); return GSW_EINVAL; }
+    *bytes = dist_workspace(n_global, nnz_owned, nranks, loopback ? nranks : 1, loopback ? kModeLoopback : kModeNccl,
+                            has_weights != 0);
     return GSW_OK;
 }
 
 gsw_status gsw_dist_loopback_workspace_size(int64_t n, int64_t nnz, int32_t nparts, size_t *bytes) {
     if (!bytes || n <= 0 || nnz < 0 || nparts < 1) { set_error("gsw_dist_loopback_workspace_size: bad arguments"); return GSW_EINVAL; }
-    *bytes = dist_workspace(n, nnz, nparts, nparts, kModeLoopback);
+    *bytes = dist_workspace(n, nnz, nparts, nparts, kModeLoopback, false);
     return GSW_OK;
 }
 

@@ -118,6 +118,7 @@ struct DCtl {
     double pad0;
     long long Via, Eia, nnz_g;     // unvisited vertices / their edges, global nnz
     int dir, done, t, pad1;
+    unsigned long long theta, delta;   // SSSP priority threshold and its step (P4)
 };
 
 // per-part counters, 64 B apart: {va, ea, edges, changes, f64 bits, -, -, -}
@@ -132,7 +133,10 @@ struct DPart {
     int32_t *rfirst = nullptr;// first in-neighbour of each owned row (-1: empty)
     uint32_t *soff = nullptr; // n_global+1: global source u -> owned targets
     int32_t *scol = nullptr;  // local target ids
-    unsigned *vis = nullptr;  // visited words of the owned slice (S/32)
+    unsigned *vis = nullptr;  // visited words of the owned slice (S/32); SSSP: improved in the last push
+    unsigned *far = nullptr;  // SSSP far set of the owned slice (S/32)
+    const uint32_t *rw = nullptr;   // weights of the owned rows (weighted graphs)
+    uint32_t *sw = nullptr;   // weights of the column slice
     DTask *chunks = nullptr;  // heavy owned rows cut into kHeavy-edge chunks (create time)
     unsigned *nchunks = nullptr;
     DTask *ptasks = nullptr;  // push tasks of the current level
@@ -153,6 +157,9 @@ struct DistState {
     DCtl *ctl = nullptr;
     DRec *recs = nullptr;
     ncclComm_t comm = nullptr;
+    unsigned *ntasks = nullptr;             // parts x 32: push-task counters (zeroed by k_bfs_decide)
+    bool weighted = false;
+    double wbar = 0.0;                      // mean edge weight (SSSP static step c * wbar / dbar)
     gsw_exchange hx{};                      // host-staged backend callbacks
     unsigned char *hsend = nullptr, *hrecv = nullptr;   // pinned staging (host mode)
     size_t hcap = 0;
@@ -190,9 +197,21 @@ __global__ void k_slice_count(const uint32_t *roff, const int32_t *rcol, int nlo
     for (long long v = gtid(); v < nloc; v += gthreads())
         for (uint32_t e = roff[v]; e < roff[v + 1]; ++e) atomicAdd(cnt + rcol[e], 1u);
 }
-__global__ void k_slice_fill(const uint32_t *roff, const int32_t *rcol, int nloc, uint32_t *cursor, int32_t *scol) {
+__global__ void k_slice_fill(const uint32_t *roff, const int32_t *rcol, const uint32_t *rw, int nloc, uint32_t *cursor,
+                             int32_t *scol, uint32_t *sw) {
     for (long long v = gtid(); v < nloc; v += gthreads())
-        for (uint32_t e = roff[v]; e < roff[v + 1]; ++e) scol[atomicAdd(cursor + rcol[e], 1u)] = (int32_t)v;
+        for (uint32_t e = roff[v]; e < roff[v + 1]; ++e) {
+            const uint32_t k = atomicAdd(cursor + rcol[e], 1u);
+            scol[k] = (int32_t)v;
+            if (sw) sw[k] = rw[e];     // symmetric graph: w(u, v) = w(v, u)
+        }
+}
+// sum of the owned rows' weights (for wbar)
+__global__ void k_wsum(const uint32_t *w, uint32_t m, unsigned long long *out) {
+    unsigned long long s = 0;
+    for (long long e = gtid(); e < m; e += gthreads()) s += w[e];
+    s = warp_sum(s);
+    if (lane_id() == 0 && s) atomicAdd(out, s);
 }
 // heavy owned rows -> kHeavy-edge chunks (order irrelevant: partials meet in atomics)
 __global__ void k_chunks(const uint32_t *roff, int nloc, DTask *tab, unsigned *cnt) {
@@ -294,8 +313,7 @@ __device__ __forceinline__ bool push_claim(const BfsP &a, int v, unsigned long l
 
 // push, light part: a lane per frontier vertex of the warp's bitmap word (rows <= 32 edges, 4
 // columns in flight), the whole warp for rows of 33..kHeavy edges, tasks for longer rows
-__global__ void __launch_bounds__(kDB) k_bfs_push(BfsP a) {
-    if (a.ctl->done || a.ctl->dir != GSW_PUSH) return;
+__device__ __noinline__ void bfs_push_body(const BfsP &a) {
     const long long FW = a.npad >> 5;
     const unsigned lane = lane_id();
     unsigned long long va = 0, ea = 0, ed = 0;
@@ -344,18 +362,28 @@ __global__ void __launch_bounds__(kDB) k_bfs_push_heavy(BfsP a) {
     flush_loc(va, ea, ed, 0.0, a.loc);
 }
 
-__global__ void __launch_bounds__(kDB) k_bfs_pull(BfsP a) {
-    if (a.ctl->done || a.ctl->dir != GSW_PULL) return;
+// one launch per level and part: the direction decided on the device (k_bfs_decide) selects the
+// push or the pull body; heavy push rows are finished by k_bfs_push_heavy
+__global__ void __launch_bounds__(kDB) k_bfs_level(BfsP a) {
+    if (a.ctl->done) return;
+    if (a.ctl->dir == GSW_PUSH) {
+        bfs_push_body(a);
+        return;
+    }
     __shared__ int lists[(kPullList + kPullWordsPerWarp) * kDW];
     LocalCnt c = bfs_pull_list(a.fb, a.vis, a.depth, a.roff, a.rcol, a.rfirst, a.roff, true, a.lvl,
                                a.nfb + (a.vb >> 5), a.nloc, lists);
     flush_loc(c.va, c.ea, c.edges, 0.0, a.loc);
 }
 
-// one thread: account level t (its expand just finished, tot = counts of AS_{t+1}), decide t+1
+// account level t (its expand and exchange finished, tot = counts of AS_{t+1}) and decide t+1
+// (block 0 / thread 0); every thread also clears the bitmap level t+1 will write (FB_t, read by
+// level t) and thread 0 the parts' push-task counters, so a level needs no separate memsets
 __global__ void k_bfs_decide(DCtl *ctl, DRec *recs, unsigned long long *locs, int parts, int t, long long n,
-                             int force_dir) {
+                             int force_dir, unsigned *clear, long long clear_words, unsigned *ntasks) {
+    for (long long w = gtid(); w < clear_words; w += gthreads()) clear[w] = 0u;
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    for (int p = 0; p < parts; ++p) ntasks[p * 32] = 0u;
     const unsigned long long va = ctl->tot[0], ea = ctl->tot[1], ed = ctl->tot[2];
     for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
     if (ctl->done) return;
@@ -369,6 +397,142 @@ __global__ void k_bfs_decide(DCtl *ctl, DRec *recs, unsigned long long *locs, in
     ctl->dir = dir;
     ctl->t = t + 2;                                   // levels with a non-empty active set so far
     if (t + 1 < kMaxLevels) recs[t + 1] = DRec{(long long)va, (long long)ea, ctl->Via, ctl->Eia, 0, dir, 0};
+}
+
+// ---------------------------------------------------------------- SSSP (near/far stepping)
+// Replicated distances (rep[0], npad u32): rank r relaxes only edges into its owned slice and
+// writes only that slice; the slices are all-gathered after every push, so the next round reads
+// dist[u] of any frontier vertex locally.
+struct SsspP {
+    const uint32_t *roff;
+    const uint32_t *soff;
+    const int32_t *scol;
+    const uint32_t *sw;
+    unsigned *imp;            // owned: improved by the last push
+    unsigned *far;            // owned: improved but above theta (deferred)
+    unsigned *dist;           // replicated distances
+    int64_t vb, npad;
+    int nloc;
+    const unsigned *fb;       // the near set N_t (global bitmap)
+    unsigned *nfb;            // this part's slice of N_t is written by classify
+    DTask *tasks;
+    unsigned *ntasks;
+    uint32_t task_cap;
+    unsigned long long *loc;
+    const DCtl *ctl;
+};
+
+__global__ void k_sssp_init(SsspP a, int64_t src) {
+    const int W = (a.nloc + 31) >> 5;
+    for (long long v = gtid(); v < a.nloc; v += gthreads()) a.dist[a.vb + v] = (a.vb + v == src) ? 0u : 0xffffffffu;
+    for (long long w = gtid(); w < W; w += gthreads()) {
+        unsigned m = 0;
+        if (src >= a.vb + w * 32 && src < a.vb + w * 32 + 32 && src < a.vb + a.nloc) m = 1u << ((src - a.vb) & 31);
+        a.imp[w] = m;
+        a.far[w] = 0u;
+    }
+}
+
+// Filter of round t: improved or deferred vertices below theta form N_t (this part's slice of the
+// replicated bitmap), the rest stays in the far set; counts |N_t|, its edges, |far|
+__global__ void __launch_bounds__(kDB) k_sssp_classify(SsspP a) {
+    if (a.ctl->done) return;
+    const unsigned long long theta = a.ctl->theta;
+    const int W = (a.nloc + 31) >> 5;
+    unsigned long long va = 0, ea = 0, nf = 0;
+    for (long long w = gwarp(); w < W; w += gwarps()) {
+        const unsigned cand = a.imp[w] | a.far[w];
+        const int v = (int)(w * 32 + lane_id());
+        const bool c = (cand >> lane_id()) & 1u;
+        bool nr = false;
+        if (c) {
+            nr = (unsigned long long)a.dist[a.vb + v] < theta;
+            if (nr) { va++; ea += a.roff[v + 1] - a.roff[v]; } else nf++;
+        }
+        const unsigned nm = __ballot_sync(0xffffffffu, nr);
+        if (lane_id() == 0) {
+            a.nfb[(a.vb >> 5) + w] = nm;
+            a.far[w] = cand & ~nm;
+            a.imp[w] = 0u;
+        }
+    }
+    flush_loc(va, ea, 0, 0.0, a.loc);
+    nf = warp_sum(nf);
+    if (lane_id() == 0 && nf) atomicAdd(a.loc + 3, nf);
+}
+
+__device__ __forceinline__ void sssp_relax(const SsspP &a, int v, unsigned nd) {
+    unsigned *dv = a.dist + a.vb + v;
+    if (nd < *dv && nd < atomicMin(dv, nd)) atomicOr(a.imp + (v >> 5), 1u << (v & 31));
+}
+
+// Expand of round t: every vertex of N_t relaxes its column-slice row (owned targets)
+__global__ void __launch_bounds__(kDB) k_sssp_push(SsspP a) {
+    if (a.ctl->done) return;
+    const long long FW = a.npad >> 5;
+    const unsigned lane = lane_id();
+    unsigned long long ed = 0;
+    for (long long w = gwarp(); w < FW; w += gwarps()) {
+        const unsigned word = a.fb[w];
+        if (!word) continue;
+        const bool mine = (word >> lane) & 1u;
+        const long long u = w * 32 + lane;
+        uint32_t s0 = 0, s1 = 0;
+        unsigned du = 0;
+        if (mine) { s0 = a.soff[u]; s1 = a.soff[u + 1]; du = a.dist[u]; }
+        const uint32_t L = s1 - s0;
+        if (mine && L > kHeavy) {
+            const unsigned k = (L + kHeavy - 1) / kHeavy;
+            const unsigned i = atomicAdd(a.ntasks, k);
+            for (unsigned j = 0; j < k && i + j < a.task_cap; ++j)
+                a.tasks[i + j] = DTask{(int)u, s0 + j * kHeavy, min(s1, s0 + (j + 1) * kHeavy)};
+        }
+        if (mine && L <= 32)
+            for (uint32_t e = s0; e < s1; ++e) { ed++; sssp_relax(a, __ldg(a.scol + e), du + __ldg(a.sw + e)); }
+        unsigned mid = __ballot_sync(0xffffffffu, mine && L > 32 && L <= kHeavy);
+        while (mid) {
+            const int j = __ffs(mid) - 1;
+            mid &= mid - 1;
+            const uint32_t b = __shfl_sync(0xffffffffu, s0, j), e = __shfl_sync(0xffffffffu, s1, j);
+            const unsigned dj = __shfl_sync(0xffffffffu, du, j);
+            for (uint32_t k = b + lane; k < e; k += 32) { ed++; sssp_relax(a, __ldg(a.scol + k), dj + __ldg(a.sw + k)); }
+        }
+    }
+    flush_loc(0, 0, ed, 0.0, a.loc);
+}
+
+__global__ void __launch_bounds__(kDB) k_sssp_push_heavy(SsspP a) {
+    if (a.ctl->done) return;
+    const unsigned nt = min(*a.ntasks, a.task_cap);
+    unsigned long long ed = 0;
+    for (long long k = gwarp(); k < nt; k += gwarps()) {
+        const DTask tk = a.tasks[k];
+        const unsigned du = a.dist[tk.row];
+        for (uint32_t e = tk.beg + lane_id(); e < tk.end; e += 32) { ed++; sssp_relax(a, __ldg(a.scol + e), du + __ldg(a.sw + e)); }
+    }
+    flush_loc(0, 0, ed, 0.0, a.loc);
+}
+
+// after classify's exchange: empty near set -> advance theta (static delta-stepping, P4) or stop
+// when the far set is empty too; records the round; zeroes the counters and push-task counters
+__global__ void k_sssp_decide(DCtl *ctl, DRec *recs, unsigned long long *locs, int parts, int t, unsigned *ntasks) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const unsigned long long va = ctl->tot[0], ea = ctl->tot[1], nf = ctl->tot[3];
+    for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
+    for (int p = 0; p < parts; ++p) ntasks[p * 32] = 0u;
+    if (ctl->done) return;
+    if (va == 0) {
+        if (nf == 0) { ctl->done = 1; return; }
+        ctl->theta = ctl->theta + ctl->delta;
+    }
+    if (t < kMaxLevels) recs[t] = DRec{(long long)va, (long long)ea, (long long)nf, 0, 0, GSW_PUSH, (int)min(ctl->theta, 0xffffffffull)};
+    ctl->t = t + 1;
+}
+// edges of round t, read after the push's counters were reduced
+__global__ void k_sssp_edges(DCtl *ctl, DRec *recs, unsigned long long *locs, int parts, int t) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    if (t < kMaxLevels && !ctl->done) recs[t].edges = (long long)ctl->tot[2];
+    for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
 }
 
 // ---------------------------------------------------------------- PageRank
@@ -549,16 +713,16 @@ __global__ void k_cc_decide(DCtl *ctl, unsigned long long *locs, int parts, int 
 static size_t al(size_t x) { return (x + 255) & ~size_t(255); }
 static size_t chunk_cap(uint64_t nnz) { return (size_t)(2 * nnz / kHeavy + 2); }
 
-static size_t dist_bytes(int64_t n, int64_t nnz_total, int32_t nranks, int32_t nparts, int mode) {
+static size_t dist_bytes(int64_t n, int64_t nnz_total, int32_t nranks, int32_t nparts, int mode, bool weighted) {
     const int64_t S = dist_slice(n, nranks), npad = S * nranks;
     size_t b = 0;
     b += al((size_t)npad / 8) * 2;                           // FB[2]
     b += al((size_t)npad * 4) * 2;                           // rep[2]
-    b += al((size_t)kLocStride * 8 * nparts) + al(sizeof(DCtl)) + al(sizeof(DRec) * kMaxLevels);
+    b += al((size_t)kLocStride * 8 * nparts) + al(sizeof(DCtl)) + al(sizeof(DRec) * kMaxLevels) + al((size_t)128 * nparts);
     for (int p = 0; p < nparts; ++p) {
         b += al((size_t)(S + 1) * 4) + al((size_t)S * 4);    // roff, rfirst
         b += al((size_t)(n + 1) * 4);                        // soff
-        b += al((size_t)S / 8 + 8);                          // vis
+        b += al((size_t)S / 8 + 8) * 2;                      // vis, far
         b += al((size_t)S * 8);                              // psum
         b += al(256) * 2;                                    // nchunks, nptasks
     }
@@ -566,6 +730,7 @@ static size_t dist_bytes(int64_t n, int64_t nnz_total, int32_t nranks, int32_t n
     b += (size_t)nparts * 2 * al(0) + 2 * al(chunk_cap((uint64_t)nnz_total) * sizeof(DTask)) + nparts * 512;
     b += al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // scol (all parts)
     b += al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // rcol copy
+    if (weighted) b += 2 * al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // row + slice weights
     if (mode == DM_LOOPBACK) b += al((size_t)(n + 1) * 4);  // full u32 offsets
     size_t cub = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, cub, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(n + 1));
@@ -584,7 +749,7 @@ static gsw_status build_slice(gsw_graph g, DPart &p, int64_t n, int32_t *scol, v
     size_t cb = cub_bytes;
     GSW_CUDA(cub::DeviceScan::ExclusiveSum(cub_tmp, cb, p.soff, p.soff, (int)(n + 1), s));
     GSW_CUDA(cudaMemcpyAsync(cursor, p.soff, (size_t)(n + 1) * 4, cudaMemcpyDeviceToDevice, s));
-    k_slice_fill<<<grid_for(p.nloc, g->sms), kDB, 0, s>>>(p.roff, p.rcol, p.nloc, cursor, scol);
+    k_slice_fill<<<grid_for(p.nloc, g->sms), kDB, 0, s>>>(p.roff, p.rcol, p.rw, p.nloc, cursor, scol, p.sw);
     GSW_CUDA(cudaGetLastError());
     p.scol = scol;
     return GSW_OK;
@@ -675,7 +840,7 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
         set_error("loopback mode takes the full graph");
         return GSW_EINVAL;
     }
-    const size_t need = dist_bytes(n, rows->nnz, nranks, nparts, mode);
+    const size_t need = dist_bytes(n, rows->nnz, nranks, nparts, mode, rows->weights != nullptr);
     if (!workspace || is_device_ptr(workspace) != 1 || ws_bytes < need) {
         set_error("dist workspace must be a device buffer of >= " + std::to_string(need) + " bytes");
         return GSW_ENOMEM;
@@ -720,6 +885,7 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
     d->locs = (unsigned long long *)ws.take((size_t)kLocStride * 8 * nparts);
     d->ctl = (DCtl *)ws.take(sizeof(DCtl));
     d->recs = (DRec *)ws.take(sizeof(DRec) * kMaxLevels);
+    d->ntasks = (unsigned *)ws.take((size_t)128 * nparts);
     int64_t *staging = (int64_t *)ws.take((size_t)(n + 1) * 8);
     size_t cub_bytes = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, cub_bytes, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(n + 1));
@@ -728,9 +894,13 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
     int32_t *scol_all = (int32_t *)ws.take((size_t)std::max<int64_t>(rows->nnz, 1) * 4);
     int32_t *col = (int32_t *)ws.take((size_t)std::max<int64_t>(rows->nnz, 1) * 4);
     uint32_t *full_off = loopback ? (uint32_t *)ws.take((size_t)(n + 1) * 4) : nullptr;
+    d->weighted = rows->weights != nullptr;
+    uint32_t *wrow = d->weighted ? (uint32_t *)ws.take((size_t)std::max<int64_t>(rows->nnz, 1) * 4) : nullptr;
+    uint32_t *wslice = d->weighted ? (uint32_t *)ws.take((size_t)std::max<int64_t>(rows->nnz, 1) * 4) : nullptr;
+    if (d->weighted && (!wrow || !wslice)) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
     DTask *chunk_all = (DTask *)ws.take(chunk_cap((uint64_t)rows->nnz) * sizeof(DTask));
     DTask *task_all = (DTask *)ws.take(chunk_cap((uint64_t)rows->nnz) * sizeof(DTask));
-    if (!d->FB[1] || !d->rep[1] || !d->locs || !d->ctl || !d->recs || !staging || !cub_tmp || !cursor || !scol_all ||
+    if (!d->FB[1] || !d->rep[1] || !d->locs || !d->ctl || !d->recs || !d->ntasks || !staging || !cub_tmp || !cursor || !scol_all ||
         !col || (loopback && !full_off) || !chunk_all || !task_all) {
         set_error("dist workspace too small");
         return fail(GSW_ENOMEM);
@@ -747,6 +917,10 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
                                          is_device_ptr(rows->col_indices) ? cudaMemcpyDeviceToDevice
                                                                           : cudaMemcpyHostToDevice, s) != cudaSuccess)
         return fail(cuda_fail(cudaGetLastError(), "copy columns"));
+    if (d->weighted && rows->nnz > 0 &&
+        cudaMemcpyAsync(wrow, rows->weights, (size_t)rows->nnz * 4,
+                        is_device_ptr(rows->weights) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, s) != cudaSuccess)
+        return fail(cuda_fail(cudaGetLastError(), "copy weights"));
     if (loopback) k_rebase_offsets<<<grid_for(n + 1, g->sms), kDB, 0, s>>>(off64, 0, full_off, n + 1);
     std::vector<int64_t> hoff;
     if (loopback) {
@@ -766,11 +940,12 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
         P.rfirst = (int32_t *)ws.take((size_t)S * 4 + 4);
         P.soff = (uint32_t *)ws.take((size_t)(n + 1) * 4);
         P.vis = (unsigned *)ws.take((size_t)S / 8 + 8);
+        P.far = (unsigned *)ws.take((size_t)S / 8 + 8);
         P.psum = (double *)ws.take((size_t)S * 8 + 8);
         P.nchunks = (unsigned *)ws.take(256);
-        P.nptasks = (unsigned *)ws.take(256);
+        P.nptasks = d->ntasks ? d->ntasks + 32 * p : nullptr;
         P.loc = d->locs + (size_t)p * kLocStride;
-        if (!P.roff || !P.rfirst || !P.soff || !P.vis || !P.psum || !P.nchunks || !P.nptasks) {
+        if (!P.roff || !P.rfirst || !P.soff || !P.vis || !P.far || !P.psum || !P.nchunks || !P.nptasks) {
             set_error("dist workspace too small");
             return fail(GSW_ENOMEM);
         }
@@ -778,11 +953,13 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
             const int64_t e0 = P.nloc ? hoff[P.vb] : 0, e1 = P.nloc ? hoff[P.vb + P.nloc] : 0;
             P.nnz = (uint32_t)(e1 - e0);
             P.rcol = col + e0;
+            if (wrow) { P.rw = wrow + e0; P.sw = wslice + e0; }
             if (P.nloc)
                 k_rebase_offsets_u32<<<grid_for(P.nloc + 1, g->sms), kDB, 0, s>>>(full_off + P.vb, (uint32_t)e0, P.roff, P.nloc + 1);
         } else {
             P.nnz = (uint32_t)rows->nnz;
             P.rcol = col;
+            if (wrow) { P.rw = wrow; P.sw = wslice; }
             k_rebase_offsets<<<grid_for(P.nloc + 1, g->sms), kDB, 0, s>>>(off64, 0, P.roff, P.nloc + 1);
         }
         if (cudaGetLastError() != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "rebase"));
@@ -810,6 +987,7 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
         if (cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * nparts, s) != cudaSuccess ||
             cudaMemcpyAsync(d->locs, h, sizeof(h), cudaMemcpyHostToDevice, s) != cudaSuccess)
             return fail(cuda_fail(cudaGetLastError(), "nnz"));
+        if (wrow && rows->nnz > 0) k_wsum<<<grid_for(rows->nnz, g->sms), kDB, 0, s>>>(wrow, (uint32_t)rows->nnz, d->locs + 1);
         if (gsw_status st = ex_reduce(d, s)) return fail(st);
         unsigned long long tot[4];
         if (cudaMemcpyAsync(tot, d->ctl->tot, 32, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
@@ -817,6 +995,7 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
             return fail(cuda_fail(cudaGetLastError(), "nnz"));
         DCtl c{};
         c.nnz_g = (long long)tot[0];
+        d->wbar = tot[0] ? (double)tot[1] / (double)tot[0] : 1.0;
         if (cudaMemcpyAsync(d->ctl, &c, sizeof(c), cudaMemcpyHostToDevice, s) != cudaSuccess ||
             cudaStreamSynchronize(s) != cudaSuccess)
             return fail(cuda_fail(cudaGetLastError(), "ctl"));
@@ -897,26 +1076,24 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
     if (gsw_status e = ex_allgather(d, d->FB[0], (size_t)d->S / 8, s)) return e;      // the owner's source bit
     // level-0 features (Va = 1, Ea = deg(source)) through the same exchange, then the decision
     if (gsw_status e = ex_reduce(d, s)) return e;
-    k_bfs_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, -1, d->n, fdir);
-    GSW_CUDA(cudaGetLastError());
     const int grid = g->sms * 8;
+    const long long FBW = d->npad / 32;
+    k_bfs_decide<<<g->sms, kDB, 0, s>>>(d->ctl, d->recs, d->locs, parts, -1, d->n, fdir, d->FB[1], FBW, d->ntasks);
+    GSW_CUDA(cudaGetLastError());
     int t = 0;
     for (;; ++t) {
         unsigned *fb = d->FB[t & 1], *nfb = d->FB[(t + 1) & 1];
-        GSW_CUDA(cudaMemsetAsync(nfb, 0, FBB, s));
         for (int p = 0; p < parts; ++p) {
             BfsP a = pa[p];
             a.fb = fb; a.nfb = nfb; a.lvl = t;
             if (!a.nloc) continue;
-            GSW_CUDA(cudaMemsetAsync(a.ntasks, 0, 4, s));
-            k_bfs_push<<<grid, kDB, 0, s>>>(a);
-            k_bfs_push_heavy<<<grid, kDB, 0, s>>>(a);
-            k_bfs_pull<<<grid, kDB, 0, s>>>(a);
+            k_bfs_level<<<grid, kDB, 0, s>>>(a);
+            k_bfs_push_heavy<<<g->sms * 2, kDB, 0, s>>>(a);
         }
         GSW_CUDA(cudaGetLastError());
         if (gsw_status e = ex_allgather(d, nfb, (size_t)d->S / 8, s)) return e;
         if (gsw_status e = ex_reduce(d, s)) return e;
-        k_bfs_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, t, d->n, fdir);
+        k_bfs_decide<<<g->sms, kDB, 0, s>>>(d->ctl, d->recs, d->locs, parts, t, d->n, fdir, fb, FBW, d->ntasks);
         GSW_CUDA(cudaGetLastError());
         bool stop = false;
         if (gsw_status e = poll_done(d, t, s, &stop)) return e;
@@ -951,6 +1128,108 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
             }
         }
         st->iterations = levels;
+        st->gpu_ms = ms;
+        st->edges_touched = (int64_t)edges;
+        st->bytes_alg = (int64_t)bytes;
+    }
+    return GSW_OK;
+}
+
+// ------------------------------------------------------------------ distributed SSSP
+// Near/far rounds with a static step (P4 "static" candidate; forced UNORDERED = Bellman-Ford,
+// theta = infinity): classify -> all-gather of the near-set slices + counts -> decide (theta,
+// done) -> push over the column slices (atomicMin on owned distances) -> all-gather of the
+// distance slices.  The dynamic law of the single-GPU kernel is not used here.
+gsw_status dist_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_stats *st) {
+    DistState *d = g->dist;
+    cudaStream_t s = g->stream;
+    if (source < 0 || source >= d->n) { set_error("gsw_sssp: source out of range"); return GSW_EINVAL; }
+    if (!dist_out) { set_error("gsw_sssp: dist is NULL"); return GSW_EINVAL; }
+    if (!d->weighted) { set_error("gsw_sssp: the partitioned graph has no weights"); return GSW_EINVAL; }
+    const int parts = (int)d->parts.size();
+    const int64_t out_len = d->mode == DM_LOOPBACK ? d->n : d->parts[0].nloc;
+    const bool dev_out = is_device_ptr(dist_out) == 1;
+    unsigned *distv = d->rep[0];
+    long long nnz_g = 0;
+    if (gsw_status e = read_nnz_g(d, s, &nnz_g)) return e;
+    DCtl c0;
+    reset_ctl_host(c0, nnz_g, d->n);
+    const gsw_config &fc = g->forced;
+    const double dbar = (double)nnz_g / (double)d->n;
+    const double d0 = fc.delta0 ? (double)fc.delta0 : 32.0 * d->wbar / std::max(dbar, 1e-9);   // P:660-661, R6b
+    c0.delta = (unsigned long long)std::max(1.0, std::min(d0, 2147483647.0));
+    c0.theta = fc.stepping == GSW_STEP_UNORDERED ? 0xffffffffull : c0.delta;
+    GSW_CUDA(cudaEventRecord(g->ev0, s));
+    GSW_CUDA(cudaMemcpyAsync(d->ctl, &c0, sizeof(c0), cudaMemcpyHostToDevice, s));
+    GSW_CUDA(cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * parts, s));
+    GSW_CUDA(cudaMemsetAsync(d->ntasks, 0, (size_t)128 * parts, s));
+    GSW_CUDA(cudaMemsetAsync(d->FB[0], 0, (size_t)d->npad / 8, s));   // padding words stay 0 (never classified)
+    std::vector<SsspP> pa(parts);
+    for (int p = 0; p < parts; ++p) {
+        const DPart &P = d->parts[p];
+        pa[p] = SsspP{P.roff, P.soff, P.scol, P.sw, P.vis, P.far, distv, P.vb, d->npad, P.nloc, nullptr, nullptr,
+                      P.ptasks, P.nptasks, P.ptask_cap, P.loc, d->ctl};
+        k_sssp_init<<<grid_for(std::max(P.nloc, 1), g->sms), kDB, 0, s>>>(pa[p], source);
+    }
+    GSW_CUDA(cudaGetLastError());
+    if (gsw_status e = ex_allgather(d, distv, (size_t)d->S * 4, s)) return e;
+    const int grid = g->sms * 8;
+    unsigned *nb = d->FB[0];
+    int t = 0;
+    for (;; ++t) {
+        for (int p = 0; p < parts; ++p) {
+            SsspP a = pa[p];
+            a.fb = nb; a.nfb = nb;
+            if (a.nloc) k_sssp_classify<<<grid, kDB, 0, s>>>(a);
+        }
+        GSW_CUDA(cudaGetLastError());
+        if (gsw_status e = ex_allgather(d, nb, (size_t)d->S / 8, s)) return e;
+        if (gsw_status e = ex_reduce(d, s)) return e;
+        k_sssp_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, t, d->ntasks);
+        for (int p = 0; p < parts; ++p) {
+            SsspP a = pa[p];
+            a.fb = nb; a.nfb = nb;
+            if (!a.nloc) continue;
+            k_sssp_push<<<grid, kDB, 0, s>>>(a);
+            k_sssp_push_heavy<<<g->sms * 2, kDB, 0, s>>>(a);
+        }
+        GSW_CUDA(cudaGetLastError());
+        if (gsw_status e = ex_allgather(d, distv, (size_t)d->S * 4, s)) return e;
+        if (gsw_status e = ex_reduce(d, s)) return e;
+        k_sssp_edges<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, t);
+        GSW_CUDA(cudaGetLastError());
+        bool stop = false;
+        if (gsw_status e = poll_done(d, t, s, &stop)) return e;
+        if (stop || t + 1 >= (1 << 24)) break;
+    }
+    GSW_CUDA(cudaEventRecord(g->ev1, s));
+    const unsigned *own = distv + (d->mode == DM_LOOPBACK ? 0 : d->parts[0].vb);
+    GSW_CUDA(cudaMemcpyAsync(dist_out, own, (size_t)out_len * 4, dev_out ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s));
+    DCtl cend;
+    GSW_CUDA(cudaMemcpyAsync(&cend, d->ctl, sizeof(cend), cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    const int rounds = cend.t;
+    if (st) {
+        float ms = 0.f;
+        GSW_CUDA(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+        const int nrec = std::min(rounds, kMaxLevels);
+        std::vector<DRec> h(nrec);
+        if (nrec) GSW_CUDA(cudaMemcpy(h.data(), d->recs, sizeof(DRec) * nrec, cudaMemcpyDeviceToHost));
+        unsigned long long edges = 0, bytes = 0;
+        for (int i = 0; i < nrec; ++i) {
+            edges += h[i].edges;
+            bytes += 12ull * h[i].Va + 8ull * h[i].edges + 8ull * (i + 1 < nrec ? h[i + 1].Va : 0);
+            if (st->records && i < st->max_records) {
+                gsw_iter_record &r = st->records[i];
+                r = gsw_iter_record{};
+                r.iteration = i; r.direction = GSW_PUSH; r.format = GSW_BITMAP; r.load_balance = GSW_LB_TWC;
+                r.stepping = fc.stepping == GSW_STEP_UNORDERED ? GSW_STEP_UNORDERED : GSW_STEP_STATIC;
+                r.fusion = GSW_STANDALONE;
+                r.Va = h[i].Va; r.Ea = h[i].Ea; r.edges = h[i].edges; r.theta = (uint32_t)h[i].pad;
+                r.ctas = grid;
+            }
+        }
+        st->iterations = rounds;
         st->gpu_ms = ms;
         st->edges_touched = (int64_t)edges;
         st->bytes_alg = (int64_t)bytes;
@@ -1076,8 +1355,8 @@ gsw_status dist_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     return GSW_OK;
 }
 
-size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, int mode) {
-    return dist_bytes(n, nnz, nranks, nparts, mode);
+size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, int mode, bool weighted) {
+    return dist_bytes(n, nnz, nranks, nparts, mode, weighted);
 }
 
 gsw_status dist_unique_id(void *id128) {

@@ -1,8 +1,9 @@
 // pr_blocked.cu -- PageRank pull with row tiers and (optionally) the gather blocked by SOURCE range,
 // for graphs whose contribution array does not fit in L2 ("L2 blocking of the PR
 // gather by source range is the B200 lever" at C5, where pr/deg of 67M vertices is 268 MB against
-// a 126 MB L2).  Measured, the blocking does not pay on B200 (see run_pr_blocked: B = 1 wins), but
-// the row-tiered kernel is 2.35x the edge-tiled stream kernel at C5, so it is AUTO's choice there.
+// a 126 MB L2).  Measured, the blocking does not pay on B200 (see run_pr_blocked: B = 1 wins), and
+// once the stream kernel's hub cache was sized for L1 the row tiers lost their lead at C5 too
+// (116 vs 120 it/s): a measured alternative, selected with GSW_PR_BLOCKED=1.
 //
 // Same iteration as pr.cu / pr_stream.cu (reading R7):
 //   pr_{t+1}(v) = (1-d)/N + d * ( sum_{u in N_in(v)} pr_t(u)/deg_out(u) + D_t/N ),  D_t = dangling mass
@@ -200,11 +201,13 @@ __global__ void __launch_bounds__(kPB) k_pb_final(PbArgs a, int t, bool last) {
 
 // Blocking is worth it once the fp32 contributions exceed half of L2; GSW_PR_BLOCKED=1 forces it
 // (parity tests on small graphs), =0 disables it.
+// Not AUTO's choice any more: with the hub cache sized for L1 (pr_stream.cu) the stream kernel
+// reaches 120 it/s on C5 against 116 for this one (profiles/r2/pr_cache_sweep.txt), so the
+// row-tier / source-blocked kernel is kept as a measured alternative, selected by GSW_PR_BLOCKED=1.
 bool pr_blocked_wanted(gsw_graph g) {
+    (void)g;
     if (const char *e = std::getenv("GSW_PR_BLOCKED")) return std::atoi(e) != 0;
-    int l2 = 0;
-    if (cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, g->device) != cudaSuccess) { cudaGetLastError(); return false; }
-    return (double)g->g.n * 4.0 > 0.5 * (double)l2;
+    return false;
 }
 
 gsw_status run_pr_blocked(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st) {

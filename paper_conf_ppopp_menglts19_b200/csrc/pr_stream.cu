@@ -365,7 +365,16 @@ static int stream_cache_entries(gsw_graph g, size_t *smem_bytes) {
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, g->device);
     const size_t static_bytes = sizeof(uint32_t) * kSWarps * kWBuf + 2048;   // warp buffers, scratch
     long long avail = (long long)optin - (long long)static_bytes - 16;
-    long long K = avail > 0 ? (avail / 16) * 4 : 0;
+    // Cache size (profiles/r2/pr_cache_sweep.txt, tools/pr_ab.py): every shared-memory byte the hub
+    // cache takes is an L1 byte the gathers lose (one CTA per SM; the carveout steps 132 / 164 /
+    // 196 / 228 KB), and the whole opt-in size (~46K entries, L1 ~28 KB) was the worst choice:
+    // C3 11.5 ms vs 7.6 ms at 28,672 entries (2,629 it/s), C4 19.3 vs 12.4 ms, C1 0.43 vs 0.37 ms.
+    // Graphs whose contributions overflow L2 (C5) want a smaller cache still: 12,288 entries
+    // 166 ms vs 179 ms at 28,672 (and 402 ms at the maximum).
+    int l2 = 0;
+    if (cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, g->device) != cudaSuccess) { cudaGetLastError(); l2 = 0; }
+    const long long want = (l2 > 0 && (double)g->g.n * 4.0 > 0.5 * (double)l2) ? 12288 : 28672;
+    long long K = std::min<long long>(want, avail > 0 ? (avail / 16) * 4 : 0);
     K = std::min<long long>(K, ((long long)g->g.n / 4) * 4);
     if (const char *e = getenv("GSW_PR_CACHE")) K = std::min<long long>(K, (atoll(e) / 4) * 4);   // tests
     if (K < 0) K = 0;

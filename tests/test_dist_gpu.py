@@ -61,7 +61,7 @@ def test_nccl_single_rank(gsw):
     lab, st = D.cc()
     assert np.array_equal(lab.cpu().numpy(), oracle.cc(g))
     with pytest.raises(gsw.GswError):
-        D.sssp(s)
+        D.sssp(s)                                             # no weights on this handle
     D2 = gsw.DistGraph(off, col, g.n, None, 1, 0)            # private communicator, no id needed
     d, _ = D2.bfs(s)
     assert np.array_equal(d.cpu().numpy(), oracle.bfs(g, s))
@@ -124,6 +124,13 @@ def _host_worker(rank, ws, port, q):
         lab, _ = D.cc()
         if not np.array_equal(lab.cpu().numpy(), oracle.cc(g)[vb:ve]):
             bad.append("cc")
+        gw = gen.with_hash_weights(g, 11, 64)
+        wo, wc, ww = m.owned_rows(gw.off, gw.col, rank, ws, weights=gw.w)
+        Dw = m.HostDistGraph(wo, wc, g.n, ex, rank, device="cuda:0", weights=ww)
+        s0 = gen.sources(g, 1, seed=6)[0]
+        dd, _ = Dw.sssp(s0)
+        if not np.array_equal(dd.cpu().numpy().view(np.uint32), oracle.sssp(gw, s0)[vb:ve]):
+            bad.append("sssp")
         q.put((rank, bad))
         dist.barrier()
         dist.destroy_process_group()
@@ -155,3 +162,32 @@ def test_c3_loopback_8(gsw):
     s = gen.sources(g, 1)[0]
     d, _ = P.bfs(s)
     assert np.array_equal(d.cpu().numpy(), oracle.bfs(g, s))
+
+
+@pytest.mark.parametrize("nparts", [1, 2, 3, 8])
+def test_loopback_sssp(gsw, nparts):
+    """Partitioned SSSP (near/far with a static step, forced UNORDERED = Bellman-Ford): bit-exact
+    distances against the Dijkstra oracle on scale-free, grid and path inputs."""
+    for g in (gen.with_hash_weights(gen.rmat(12, seed=4), 3, 64), gen.with_hash_weights(gen.grid(41, 23), 12345, 64),
+              gen.with_hash_weights(gen.from_edges(200, [(i, i + 1) for i in range(199)]), 5, 64)):
+        P = gsw.PartitionedGraph(g.off, g.col, nparts, weights=g.w)
+        for step in (None, "unordered"):
+            P.force_config(stepping=step)
+            for s in gen.sources(g, 2, seed=3):
+                d, st = P.sssp(s, records=64)
+                assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.sssp(g, s)), (nparts, g.name, step, s)
+        P.force_config(delta0=1)
+        s = gen.sources(g, 1, seed=9)[0]
+        d, _ = P.sssp(s)
+        assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.sssp(g, s))
+
+
+def test_nccl_single_rank_sssp(gsw):
+    g = gen.with_hash_weights(gen.rmat(12, seed=5), 7, 64)
+    off, col, w = gsw.owned_rows(g.off, g.col, 0, 1, weights=g.w)
+    D = gsw.DistGraph(off, col, g.n, None, 1, 0, weights=w)
+    s = gen.sources(g, 1)[0]
+    d, _ = D.sssp(s)
+    assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.sssp(g, s))
+    with pytest.raises(gsw.GswError):
+        gsw.DistGraph(*gsw.owned_rows(g.off, g.col, 0, 1), g.n, None, 1, 0).sssp(s)   # no weights
