@@ -350,6 +350,9 @@ def partition_input(workload, rank, ws):
     n = 1 << scale
     S = gsw.dist_slice(n, ws)
     vb, ve = min(n, rank * S), min(n, (rank + 1) * S)
+    # torchrun sets OMP_NUM_THREADS=1; give this rank its share of the node's cores for generation
+    local_ws = int(os.environ.get("LOCAL_WORLD_SIZE", ws))
+    gen.set_threads(max(1, (os.cpu_count() or 1) // max(1, local_ws)))
     t0 = time.time()
     off, col = gen.rmat_slice(scale, vb, ve, 16, seed=1)
     return n, vb, off, col, time.time() - t0

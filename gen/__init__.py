@@ -51,6 +51,8 @@ def _load():
                                      ctypes.c_uint64, ctypes.POINTER(_Csr)]
         lib.gen_hash_weights.argtypes = [ctypes.POINTER(_Csr), ctypes.c_uint64, ctypes.c_uint32]
         lib.gen_free.argtypes = [ctypes.POINTER(_Csr)]
+        lib.gen_set_threads.argtypes = [ctypes.c_int]
+        lib.gen_set_threads.restype = None
         lib.gen_splitmix64.argtypes = [ctypes.c_uint64]
         lib.gen_splitmix64.restype = ctypes.c_uint64
         _lib = lib
@@ -141,6 +143,11 @@ def with_hash_weights(g: Graph, seed: int = 12345, maxw: int = 64) -> Graph:
     # free only the weight buffer (off/col belong to numpy)
     ctypes.CDLL(None).free(ctypes.cast(c.w, ctypes.c_void_p))
     return Graph(g.n, g.off, g.col, w, g.name + f"_w{maxw}")
+
+
+def set_threads(k: int) -> None:
+    """OpenMP threads of the C generators (0 = all cores); draws do not depend on it."""
+    _load().gen_set_threads(int(k))
 
 
 def splitmix64(x: int) -> int:

@@ -42,6 +42,19 @@ static inline double u01(uint64_t r) { return (double)(r >> 11) * (1.0 / 9007199
 
 uint64_t gen_splitmix64(uint64_t x) { return splitmix64(x); }
 
+/* OpenMP threads of the generators (0 = all cores).  torchrun exports OMP_NUM_THREADS=1 to every
+ * rank; bench.py gives each rank its share of the host cores for its slice of C5 instead. */
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+void gen_set_threads(int k) {
+#ifdef _OPENMP
+    omp_set_num_threads(k > 0 ? k : omp_get_num_procs());
+#else
+    (void)k;
+#endif
+}
+
 typedef struct {
     int64_t n, nnz;
     int64_t *off;   /* n+1 */

@@ -29,22 +29,54 @@ LBS = ["thread", "twc", "wm", "cm", "strict"]
 FUS = ["standalone", "fused"]
 
 
-def corpus(gen):
+def corpus(gen, size="full"):
+    """~110 synthetic graphs (none of them C1-C5: other seeds and sizes).  size="small" keeps the
+    round-1 list of 24."""
     out = []
-    for scale, ef, abc, seed in [(14, 8, (.57, .19, .19), 11), (14, 32, (.57, .19, .19), 12),
-                                 (15, 16, (.45, .25, .15), 13), (15, 16, (.70, .10, .10), 14),
-                                 (16, 8, (.57, .19, .19), 15), (16, 16, (.45, .15, .15), 16),
-                                 (17, 16, (.57, .19, .19), 17), (17, 4, (.57, .19, .19), 18),
-                                 (18, 16, (.57, .19, .19), 19), (18, 8, (.65, .15, .15), 20),
-                                 (19, 16, (.57, .19, .19), 21), (19, 32, (.50, .20, .20), 22),
-                                 (20, 16, (.57, .19, .19), 23), (20, 8, (.60, .15, .15), 24),
-                                 (21, 16, (.57, .19, .19), 25), (21, 24, (.50, .20, .20), 26)]:
-        out.append(gen.rmat(scale, ef, *abc, seed=seed))
-    for w, h in [(192, 192), (400, 100), (700, 700), (1400, 1000)]:
+    if size == "small":
+        for scale, ef, abc, seed in [(14, 8, (.57, .19, .19), 11), (14, 32, (.57, .19, .19), 12),
+                                     (15, 16, (.45, .25, .15), 13), (15, 16, (.70, .10, .10), 14),
+                                     (16, 8, (.57, .19, .19), 15), (16, 16, (.45, .15, .15), 16),
+                                     (17, 16, (.57, .19, .19), 17), (17, 4, (.57, .19, .19), 18),
+                                     (18, 16, (.57, .19, .19), 19), (18, 8, (.65, .15, .15), 20),
+                                     (19, 16, (.57, .19, .19), 21), (19, 32, (.50, .20, .20), 22),
+                                     (20, 16, (.57, .19, .19), 23), (20, 8, (.60, .15, .15), 24),
+                                     (21, 16, (.57, .19, .19), 25), (21, 24, (.50, .20, .20), 26)]:
+            out.append(gen.rmat(scale, ef, *abc, seed=seed))
+        for w, h in [(192, 192), (400, 100), (700, 700), (1400, 1000)]:
+            out.append(gen.grid(w, h))
+        for n, pairs, gamma, seed in [(200_000, 2_000_000, 2.1, 31), (300_000, 3_000_000, 2.5, 32),
+                                      (500_000, 4_000_000, 2.3, 33), (2_000_000, 24_000_000, 2.3, 34)]:
+            out.append(gen.chung_lu(n, pairs, gamma=gamma, i0=50.0, seed=seed))
+        return out
+    skews = [(.45, .15, .15), (.50, .20, .20), (.57, .19, .19), (.60, .15, .15), (.65, .15, .15), (.70, .10, .10)]
+    seed = 100
+    # R-MAT / Kronecker: scales 12-20 x edge factors 4-48 x six skews (72 graphs)
+    for scale in (12, 13, 14, 15, 16, 17, 18, 19, 20):
+        for k, ef in enumerate((4, 8, 16, 24, 32, 48, 6, 12)):
+            if scale >= 19 and ef > 16:
+                continue
+            seed += 1
+            out.append(gen.rmat(scale, ef, *skews[(scale + k) % len(skews)], seed=seed))
+    # road-like grids of several sizes and aspect ratios (16)
+    for w, h in [(64, 64), (128, 32), (150, 150), (256, 256), (300, 80), (400, 400), (512, 128), (600, 600),
+                 (800, 200), (1000, 1000), (1200, 300), (1400, 1400), (2000, 120), (90, 3000), (1700, 900),
+                 (2400, 500)]:
         out.append(gen.grid(w, h))
-    for n, pairs, gamma, seed in [(200_000, 2_000_000, 2.1, 31), (300_000, 3_000_000, 2.5, 32),
-                                  (500_000, 4_000_000, 2.3, 33), (2_000_000, 24_000_000, 2.3, 34)]:
-        out.append(gen.chung_lu(n, pairs, gamma=gamma, i0=50.0, seed=seed))
+    # Chung-Lu power laws (24)
+    for k, (n, pairs, gamma) in enumerate([(50_000, 300_000, 2.1), (50_000, 800_000, 2.6), (80_000, 500_000, 2.3),
+                                           (100_000, 1_000_000, 2.0), (100_000, 600_000, 2.8),
+                                           (150_000, 2_000_000, 2.2), (200_000, 1_500_000, 2.5),
+                                           (250_000, 3_000_000, 2.1), (300_000, 2_000_000, 2.9),
+                                           (400_000, 5_000_000, 2.3), (500_000, 3_000_000, 2.7),
+                                           (600_000, 8_000_000, 2.2), (700_000, 5_000_000, 2.5),
+                                           (800_000, 10_000_000, 2.4), (1_000_000, 6_000_000, 2.8),
+                                           (1_000_000, 15_000_000, 2.1), (1_200_000, 10_000_000, 2.3),
+                                           (1_500_000, 12_000_000, 2.6), (1_500_000, 20_000_000, 2.2),
+                                           (2_000_000, 16_000_000, 2.4), (2_000_000, 30_000_000, 2.1),
+                                           (2_500_000, 20_000_000, 2.5), (3_000_000, 25_000_000, 2.3),
+                                           (3_000_000, 40_000_000, 2.2)]):
+        out.append(gen.chung_lu(n, pairs, gamma=gamma, i0=20.0 + 10 * (k % 5), seed=200 + k))
     return out
 
 
@@ -52,6 +84,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--json", required=True)
     ap.add_argument("--roots", type=int, default=2)
+    ap.add_argument("--size", default="full", choices=["full", "small"])
     a = ap.parse_args()
     import torch
     import gen
@@ -59,7 +92,7 @@ def main():
     variants = list(itertools.product(DIRS, FMTS, LBS, FUS))
     rows = []
     t0 = time.time()
-    for g in corpus(gen):
+    for g in corpus(gen, a.size):
         G = gsw.Graph(g.off, g.col)
         attrs = G.attributes()
         for s in gen.sources(g, a.roots, seed=99):
