@@ -196,13 +196,16 @@ gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc,
  *     the contribution slices (n*4 bytes) + all-reduce of the dangling mass.
  *   CC iteration: min-label propagation with the pointer-jumping shortcut label[label[v]] on the
  *     replicated labels; all-gather of the label slices + all-reduce of the change count.
+ *   BC source (Brandes): forward levels pull sigma over in-neighbours at the previous depth,
+ *     backward levels pull omega = (1 + delta) / sigma over successors; the owned slices of the
+ *     replicated depth / sigma / omega arrays are all-gathered after every level.
  *   SSSP round (weighted graphs): near/far with a static step delta0 (gsw_config.delta0, else
  *     32*wbar/dbar; forced UNORDERED = Bellman-Ford): the near set is all-gathered as a bitmap,
  *     frontier vertices relax their column slices into owned distances (atomicMin), and the
  *     distance slices are all-gathered after every round.
  * The host never waits per iteration (NCCL / loopback): it polls the device's done flag two
  * iterations behind the stream.  Supported on distributed handles: gsw_bfs, gsw_pr, gsw_cc,
- * gsw_sssp (others return GSW_EUNSUPPORTED); gsw_force_config's direction pins the BFS direction,
+ * gsw_sssp, gsw_bc (gsw_dpr, gsw_app_* return GSW_EUNSUPPORTED); gsw_force_config's direction pins the BFS direction,
  * its stepping (UNORDERED) and delta0 the SSSP step.
  * Outputs of NCCL / host-staged handles cover the OWNED slice only; loopback outputs all n.
  * Three exchange backends run the same kernels:

@@ -35,6 +35,7 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
 gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out, gsw_run_stats *st);
 gsw_status dist_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st);
 gsw_status dist_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_stats *st);
+gsw_status dist_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc_out, gsw_run_stats *st);
 size_t dist_workspace(int64_t n, int64_t nnz, int32_t nranks, int32_t nparts, int mode, bool weighted);
 enum { kModeNccl = 0, kModeLoopback = 1, kModeHost = 2 };   // dist.cu DistMode
 gsw_status dist_unique_id(void *id128);
@@ -231,7 +232,7 @@ gsw_status gsw_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, d
 
 gsw_status gsw_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
-    if (gsw_status s = no_dist(g, "gsw_bc")) return s;
+    if (g->dist) return dist_bc(g, sources, nsrc, bc, stats);
     return run_bc(g, sources, nsrc, bc, stats);
 }
 

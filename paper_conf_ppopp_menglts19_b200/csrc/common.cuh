@@ -51,14 +51,12 @@ __device__ __forceinline__ unsigned lanemask_lt() {
 }
 
 // ------------------------------------------------------------------ grid barrier
-// Monotone arrival counter + generation word.  The last CTA to arrive for generation g sees
-// prev == g*gridDim - 1 and publishes g with a release store; the others spin with acquire
-// loads.  Co-residency of all CTAs is guaranteed by cudaLaunchCooperativeKernel.  A spin longer
-// than kBarrierTimeoutNs sets an error code and traps, so a bug becomes a launch failure rather
-// than a hung GPU.
+// One arrival word with the flip-bit protocol of grid_sync below (every CTA adds to the same
+// counter; the waiters poll for the flip of its top bit).  Co-residency of all CTAs is guaranteed
+// by cudaLaunchCooperativeKernel.  A spin longer than kBarrierTimeoutNs sets an error code and
+// traps, so a bug becomes a launch failure rather than a hung GPU.
 struct GridBarrier {
     unsigned *arrive;
-    unsigned *gen;
     unsigned *err;
 };
 constexpr uint64_t kBarrierTimeoutNs = 20ull * 1000 * 1000 * 1000;

@@ -158,6 +158,9 @@ struct DistState {
     DRec *recs = nullptr;
     ncclComm_t comm = nullptr;
     unsigned *ntasks = nullptr;             // parts x 32: push-task counters (zeroed by k_bfs_decide)
+    int *bdepth = nullptr;                  // BC: replicated depth (npad)
+    unsigned long long *bsigma = nullptr;   // BC: replicated path counts (npad)
+    double *bomega = nullptr;               // BC: replicated (1 + delta) / sigma (npad)
     bool weighted = false;
     double wbar = 0.0;                      // mean edge weight (SSSP static step c * wbar / dbar)
     gsw_exchange hx{};                      // host-staged backend callbacks
@@ -535,6 +538,175 @@ __global__ void k_sssp_edges(DCtl *ctl, DRec *recs, unsigned long long *locs, in
     for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
 }
 
+// ---------------------------------------------------------------- BC (Brandes, per source)
+// Replicated depth / sigma / omega: forward level l pulls, for every owned unvisited v, the sum of
+// sigma over its in-neighbours at depth l (every parent counts: no early exit); the backward level
+// l pulls, for owned v at depth l, delta = sigma(v) * sum over successors w (depth l+1) of
+// omega(w) = (1 + delta(w)) / sigma(w).  The owned slices are all-gathered after every level.
+struct BcP {
+    const uint32_t *roff;
+    const int32_t *rcol;
+    int64_t vb;
+    int nloc;
+    int *depth;
+    unsigned long long *sigma;
+    double *omega;
+    double *bc;               // owned slice, accumulated over sources
+    const DTask *chunks;
+    const unsigned *nchunks;
+    double *hacc;             // heavy-row partials (nloc): sigma as u64 bits, or the omega sum
+    unsigned long long *loc;
+    const DCtl *ctl;
+    int src;
+};
+
+__global__ void k_bc_init(int *depth, unsigned long long *sigma, int64_t npad, int src) {
+    for (long long v = gtid(); v < npad; v += gthreads()) {
+        depth[v] = v == src ? 0 : -1;
+        sigma[v] = v == src ? 1ull : 0ull;
+    }
+}
+
+// forward: heavy rows' partial sigma sums over in-neighbours at depth l
+__global__ void __launch_bounds__(kDB) k_bc_fwd_heavy(BcP a, int l) {
+    if (a.ctl->done) return;
+    unsigned long long *acc = reinterpret_cast<unsigned long long *>(a.hacc);
+    const unsigned nc = *a.nchunks;
+    for (long long k = gwarp(); k < nc; k += gwarps()) {
+        const DTask tk = a.chunks[k];
+        if (a.depth[a.vb + tk.row] != -1) continue;
+        unsigned long long s = 0;
+        for (uint32_t e = tk.beg + lane_id(); e < tk.end; e += 32) {
+            const int u = __ldg(a.rcol + e);
+            if (a.depth[u] == l) s += a.sigma[u];
+        }
+        s = warp_sum(s);
+        if (lane_id() == 0 && s) atomicAdd(acc + tk.row, s);
+    }
+}
+
+__global__ void __launch_bounds__(kDB) k_bc_fwd(BcP a, int l) {
+    if (a.ctl->done) return;
+    unsigned long long *acc = reinterpret_cast<unsigned long long *>(a.hacc);
+    const unsigned lane = lane_id();
+    unsigned long long va = 0, ea = 0, ed = 0;
+    for (long long wb = gwarp() * 32; wb < a.nloc; wb += gwarps() * 32) {
+        const long long v = wb + lane;
+        uint32_t b = 0, e = 0;
+        bool open = false;
+        if (v < a.nloc) { open = a.depth[a.vb + v] == -1; if (open) { b = a.roff[v]; e = a.roff[v + 1]; } }
+        const uint32_t L = e - b;
+        unsigned long long sg = 0;
+        if (open && L < 32) {
+            for (uint32_t k = b; k < e; ++k) {
+                const int u = __ldg(a.rcol + k);
+                if (a.depth[u] == l) sg += a.sigma[u];
+            }
+            ed += L;
+        } else if (open && L > kHeavy) {
+            sg = acc[v];
+            acc[v] = 0ull;
+            ed += L;
+        }
+        unsigned mid = __ballot_sync(0xffffffffu, open && L >= 32 && L <= kHeavy);
+        while (mid) {
+            const int j = __ffs(mid) - 1;
+            mid &= mid - 1;
+            const uint32_t bj = __shfl_sync(0xffffffffu, b, j), ej = __shfl_sync(0xffffffffu, e, j);
+            unsigned long long t = 0;
+            for (uint32_t k = bj + lane; k < ej; k += 32) {
+                const int u = __ldg(a.rcol + k);
+                if (a.depth[u] == l) t += a.sigma[u];
+            }
+            t = warp_sum(t);
+            if ((int)lane == j) { sg = t; ed += ej - bj; }
+        }
+        if (open && sg) {           // v joins level l+1 (plain stores: owned, and read only next level)
+            a.depth[a.vb + v] = l + 1;
+            a.sigma[a.vb + v] = sg;
+            va++;
+            ea += L;
+        }
+    }
+    flush_loc(va, ea, ed, 0.0, a.loc);
+}
+
+// omega = 1 / sigma for every reached vertex (delta = 0 below the deepest level); local on the
+// replicated arrays
+__global__ void k_bc_omega0(const int *depth, const unsigned long long *sigma, double *omega, int64_t npad) {
+    for (long long v = gtid(); v < npad; v += gthreads())
+        omega[v] = depth[v] >= 0 && sigma[v] ? 1.0 / (double)sigma[v] : 0.0;
+}
+
+__global__ void __launch_bounds__(kDB) k_bc_bwd_heavy(BcP a, int l) {
+    const unsigned nc = *a.nchunks;
+    for (long long k = gwarp(); k < nc; k += gwarps()) {
+        const DTask tk = a.chunks[k];
+        if (a.depth[a.vb + tk.row] != l) continue;
+        double s = 0.0;
+        for (uint32_t e = tk.beg + lane_id(); e < tk.end; e += 32) {
+            const int w = __ldg(a.rcol + e);
+            if (a.depth[w] == l + 1) s += a.omega[w];
+        }
+        s = warp_sum(s);
+        if (lane_id() == 0 && s != 0.0) atomicAdd(a.hacc + tk.row, s);
+    }
+}
+
+__global__ void __launch_bounds__(kDB) k_bc_bwd(BcP a, int l) {
+    const unsigned lane = lane_id();
+    for (long long wb = gwarp() * 32; wb < a.nloc; wb += gwarps() * 32) {
+        const long long v = wb + lane;
+        uint32_t b = 0, e = 0;
+        bool on = false;
+        if (v < a.nloc) { on = a.depth[a.vb + v] == l; if (on) { b = a.roff[v]; e = a.roff[v + 1]; } }
+        const uint32_t L = e - b;
+        double s = 0.0;
+        if (on && L < 32) {
+            for (uint32_t k = b; k < e; ++k) {
+                const int w = __ldg(a.rcol + k);
+                if (a.depth[w] == l + 1) s += a.omega[w];
+            }
+        } else if (on && L > kHeavy) {
+            s = a.hacc[v];
+            a.hacc[v] = 0.0;
+        }
+        unsigned mid = __ballot_sync(0xffffffffu, on && L >= 32 && L <= kHeavy);
+        while (mid) {
+            const int j = __ffs(mid) - 1;
+            mid &= mid - 1;
+            const uint32_t bj = __shfl_sync(0xffffffffu, b, j), ej = __shfl_sync(0xffffffffu, e, j);
+            double t = 0.0;
+            for (uint32_t k = bj + lane; k < ej; k += 32) {
+                const int w = __ldg(a.rcol + k);
+                if (a.depth[w] == l + 1) t += a.omega[w];
+            }
+            t = warp_sum(t);
+            if ((int)lane == j) s = t;
+        }
+        if (on) {
+            const double sg = (double)a.sigma[a.vb + v];
+            const double delta = sg * s;
+            a.omega[a.vb + v] = (1.0 + delta) / sg;
+            if (a.vb + v != a.src) a.bc[v] += delta;
+        }
+    }
+}
+
+__global__ void k_bc_decide(DCtl *ctl, DRec *recs, unsigned long long *locs, int parts, int t) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const unsigned long long va = ctl->tot[0];
+    for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
+    if (ctl->done) return;
+    if (va == 0) { ctl->done = 1; return; }
+    ctl->t = t + 2;                    // levels with a non-empty set so far (level 0 = the source)
+    (void)recs;
+}
+
+__global__ void k_zero_f64(double *x, long long n) {
+    for (long long i = gtid(); i < n; i += gthreads()) x[i] = 0.0;
+}
+
 // ---------------------------------------------------------------- PageRank
 struct PrP {
     const uint32_t *roff;
@@ -717,6 +889,7 @@ static size_t dist_bytes(int64_t n, int64_t nnz_total, int32_t nranks, int32_t n
     const int64_t S = dist_slice(n, nranks), npad = S * nranks;
     size_t b = 0;
     b += al((size_t)npad / 8) * 2;                           // FB[2]
+    b += al((size_t)npad * 4) + 2 * al((size_t)npad * 8);    // BC: depth, sigma, omega (replicated)
     b += al((size_t)npad * 4) * 2;                           // rep[2]
     b += al((size_t)kLocStride * 8 * nparts) + al(sizeof(DCtl)) + al(sizeof(DRec) * kMaxLevels) + al((size_t)128 * nparts);
     for (int p = 0; p < nparts; ++p) {
@@ -886,6 +1059,9 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
     d->ctl = (DCtl *)ws.take(sizeof(DCtl));
     d->recs = (DRec *)ws.take(sizeof(DRec) * kMaxLevels);
     d->ntasks = (unsigned *)ws.take((size_t)128 * nparts);
+    d->bdepth = (int *)ws.take((size_t)d->npad * 4);
+    d->bsigma = (unsigned long long *)ws.take((size_t)d->npad * 8);
+    d->bomega = (double *)ws.take((size_t)d->npad * 8);
     int64_t *staging = (int64_t *)ws.take((size_t)(n + 1) * 8);
     size_t cub_bytes = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, cub_bytes, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(n + 1));
@@ -900,7 +1076,7 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
     if (d->weighted && (!wrow || !wslice)) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
     DTask *chunk_all = (DTask *)ws.take(chunk_cap((uint64_t)rows->nnz) * sizeof(DTask));
     DTask *task_all = (DTask *)ws.take(chunk_cap((uint64_t)rows->nnz) * sizeof(DTask));
-    if (!d->FB[1] || !d->rep[1] || !d->locs || !d->ctl || !d->recs || !d->ntasks || !staging || !cub_tmp || !cursor || !scol_all ||
+    if (!d->FB[1] || !d->rep[1] || !d->locs || !d->ctl || !d->recs || !d->ntasks || !d->bomega || !staging || !cub_tmp || !cursor || !scol_all ||
         !col || (loopback && !full_off) || !chunk_all || !task_all) {
         set_error("dist workspace too small");
         return fail(GSW_ENOMEM);
@@ -1233,6 +1409,92 @@ gsw_status dist_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_st
         st->gpu_ms = ms;
         st->edges_touched = (int64_t)edges;
         st->bytes_alg = (int64_t)bytes;
+    }
+    return GSW_OK;
+}
+
+// ------------------------------------------------------------------ distributed BC
+gsw_status dist_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc_out, gsw_run_stats *st) {
+    DistState *d = g->dist;
+    cudaStream_t s = g->stream;
+    if (!bc_out) { set_error("gsw_bc: bc is NULL"); return GSW_EINVAL; }
+    if (nsrc < 0 || (nsrc > 0 && !sources)) { set_error("gsw_bc: bad sources"); return GSW_EINVAL; }
+    if (is_device_ptr(sources) == 1) { set_error("gsw_bc: sources must be a host array"); return GSW_EINVAL; }
+    for (int i = 0; i < nsrc; ++i)
+        if (sources[i] < 0 || sources[i] >= d->n) { set_error("gsw_bc: source out of range"); return GSW_EINVAL; }
+    const int parts = (int)d->parts.size();
+    const int64_t out_len = d->mode == DM_LOOPBACK ? d->n : d->parts[0].nloc;
+    const bool dev_out = is_device_ptr(bc_out) == 1;
+    double *bc = dev_out ? bc_out : (double *)g->scratch;
+    long long nnz_g = 0;
+    if (gsw_status e = read_nnz_g(d, s, &nnz_g)) return e;
+    const int grid = g->sms * 8;
+    GSW_CUDA(cudaEventRecord(g->ev0, s));
+    k_zero_f64<<<grid_for(out_len, g->sms), kDB, 0, s>>>(bc, out_len);
+    for (auto &P : d->parts) k_zero_f64<<<grid_for(std::max(P.nloc, 1), g->sms), kDB, 0, s>>>(P.psum, P.nloc);
+    GSW_CUDA(cudaGetLastError());
+    auto args = [&](int p, int src) {
+        const DPart &P = d->parts[p];
+        return BcP{P.roff, P.rcol, P.vb, P.nloc, d->bdepth, d->bsigma, d->bomega,
+                   bc + (d->mode == DM_LOOPBACK ? P.vb : 0), P.chunks, P.nchunks, P.psum, P.loc, d->ctl, src};
+    };
+    long long levels_total = 0, edges_total = 0;
+    for (int si = 0; si < nsrc; ++si) {
+        const int src = sources[si];
+        DCtl c0;
+        reset_ctl_host(c0, nnz_g, d->n);
+        GSW_CUDA(cudaMemcpyAsync(d->ctl, &c0, sizeof(c0), cudaMemcpyHostToDevice, s));
+        GSW_CUDA(cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * parts, s));
+        k_bc_init<<<grid_for(d->npad, g->sms), kDB, 0, s>>>(d->bdepth, d->bsigma, d->npad, src);
+        GSW_CUDA(cudaGetLastError());
+        // forward levels (device-side stop, polled two levels behind)
+        int t = 0;
+        for (;; ++t) {
+            for (int p = 0; p < parts; ++p) {
+                if (!d->parts[p].nloc) continue;
+                const BcP a = args(p, src);
+                k_bc_fwd_heavy<<<g->sms * 2, kDB, 0, s>>>(a, t);
+                k_bc_fwd<<<grid, kDB, 0, s>>>(a, t);
+            }
+            GSW_CUDA(cudaGetLastError());
+            if (gsw_status e = ex_allgather(d, d->bdepth, (size_t)d->S * 4, s)) return e;
+            if (gsw_status e = ex_allgather(d, d->bsigma, (size_t)d->S * 8, s)) return e;
+            if (gsw_status e = ex_reduce(d, s)) return e;
+            k_bc_decide<<<1, 32, 0, s>>>(d->ctl, d->recs, d->locs, parts, t);
+            GSW_CUDA(cudaGetLastError());
+            bool stop = false;
+            if (gsw_status e = poll_done(d, t, s, &stop)) return e;
+            if (stop || t + 1 >= kMaxLevels) break;
+        }
+        DCtl cf;
+        GSW_CUDA(cudaMemcpyAsync(&cf, d->ctl, sizeof(cf), cudaMemcpyDeviceToHost, s));
+        GSW_CUDA(cudaStreamSynchronize(s));
+        const int L = std::max(1, cf.t);          // levels 0 .. L-1 are non-empty
+        levels_total += L;
+        edges_total += (long long)L * nnz_g;
+        // backward levels L-2 .. 1 (the deepest level has delta = 0; the source gets no credit)
+        k_bc_omega0<<<grid_for(d->npad, g->sms), kDB, 0, s>>>(d->bdepth, d->bsigma, d->bomega, d->npad);
+        for (int l = L - 2; l >= 1; --l) {
+            for (int p = 0; p < parts; ++p) {
+                if (!d->parts[p].nloc) continue;
+                const BcP a = args(p, src);
+                k_bc_bwd_heavy<<<g->sms * 2, kDB, 0, s>>>(a, l);
+                k_bc_bwd<<<grid, kDB, 0, s>>>(a, l);
+            }
+            GSW_CUDA(cudaGetLastError());
+            if (gsw_status e = ex_allgather(d, d->bomega, (size_t)d->S * 8, s)) return e;
+        }
+    }
+    GSW_CUDA(cudaEventRecord(g->ev1, s));
+    if (!dev_out) GSW_CUDA(cudaMemcpyAsync(bc_out, bc, (size_t)out_len * 8, cudaMemcpyDeviceToHost, s));
+    GSW_CUDA(cudaStreamSynchronize(s));
+    if (st) {
+        float ms = 0.f;
+        GSW_CUDA(cudaEventElapsedTime(&ms, g->ev0, g->ev1));
+        st->iterations = (int32_t)levels_total;
+        st->gpu_ms = ms;
+        st->edges_touched = edges_total;
+        st->bytes_alg = (int64_t)(4ull * (unsigned long long)edges_total * 2);   // forward + backward column reads
     }
     return GSW_OK;
 }

@@ -23,7 +23,7 @@ struct Hist {
 };
 
 struct Ctl {
-    unsigned arrive, gen, err, iters;
+    unsigned arrive, spare, err, iters;   // arrive: the grid barrier's word (flip-bit protocol)
     unsigned long long edges_total, bytes_alg;
     unsigned long long t_start, t_phase, t_expand;   // kernel entry, loop start, output start (%globaltimer)
     float sum_tf, sum_te;
@@ -63,7 +63,7 @@ __device__ __forceinline__ void pub_read(const TeamPub *g, TeamPub &out) {
 }
 
 __device__ __forceinline__ GridBarrier make_bar(const RunCommon &rc) {
-    return GridBarrier{&rc.ctl->arrive, &rc.ctl->gen, &rc.ctl->err};
+    return GridBarrier{&rc.ctl->arrive, &rc.ctl->err};
 }
 
 // Per-run bookkeeping of CTA 0 / thread 0, kept in registers so that nothing on the critical

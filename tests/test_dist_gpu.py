@@ -131,6 +131,11 @@ def _host_worker(rank, ws, port, q):
         dd, _ = Dw.sssp(s0)
         if not np.array_equal(dd.cpu().numpy().view(np.uint32), oracle.sssp(gw, s0)[vb:ve]):
             bad.append("sssp")
+        srcs = gen.sources(g, 2, seed=8)
+        bcx, _ = D.bc(srcs)
+        bcr = oracle.bc(g, srcs)[vb:ve]
+        if (np.abs(bcx.cpu().numpy() - bcr) / np.maximum(np.abs(bcr), 1.0)).max() > 1e-4:
+            bad.append("bc")
         q.put((rank, bad))
         dist.barrier()
         dist.destroy_process_group()
@@ -191,3 +196,30 @@ def test_nccl_single_rank_sssp(gsw):
     assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.sssp(g, s))
     with pytest.raises(gsw.GswError):
         gsw.DistGraph(*gsw.owned_rows(g.off, g.col, 0, 1), g.n, None, 1, 0).sssp(s)   # no weights
+
+
+def _bc_close(x, r):
+    err = np.abs(x - r) / np.maximum(np.abs(r), 1.0)
+    assert err.max() <= 1e-4, err.max()
+
+
+@pytest.mark.parametrize("nparts", [1, 2, 3])
+def test_loopback_bc(gsw, nparts):
+    """Partitioned Brandes BC (forward sigma pull, backward omega pull, replicated level arrays)
+    against the oracle, with heavy rows (> 1,024 entries) among the inputs."""
+    n = 3000
+    hub = gen.from_edges(n, [(0, i) for i in range(1, 1500)] + [(i, i + 1) for i in range(1500, n - 1)] +
+                         [(i, (i * 7) % n) for i in range(1, n, 3)])
+    for g in (gen.rmat(11, seed=3), gen.grid(19, 13), hub):
+        P = gsw.PartitionedGraph(g.off, g.col, nparts)
+        srcs = gen.sources(g, 3, seed=4)
+        x, _ = P.bc(srcs)
+        _bc_close(x.cpu().numpy(), oracle.bc(g, srcs))
+
+
+def test_nccl_single_rank_bc(gsw):
+    g = gen.rmat(12, seed=8)
+    D = gsw.DistGraph(*gsw.owned_rows(g.off, g.col, 0, 1), g.n, None, 1, 0)
+    srcs = gen.sources(g, 2)
+    x, _ = D.bc(srcs)
+    _bc_close(x.cpu().numpy(), oracle.bc(g, srcs))

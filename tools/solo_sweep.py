@@ -15,7 +15,7 @@ import gen
 import paper_conf_ppopp_menglts19_b200 as gsw
 
 jobs = (sys.argv[1] if len(sys.argv) > 1 else "C2:bfs,C2:sssp,C3:bfs,C1:bfs").split(",")
-SETTINGS = [(0, 0), (512, 256), (1024, 512), (2048, 1024), (4096, 1536), (8192, 1536), (16384, 1536)]
+SETTINGS = [(0, 0), (512, 256), (1024, 512), (2048, 512), (2048, 1024), (4096, 512), (4096, 768), (8192, 768), (16384, 768)]
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 cache = {}
 for job in jobs:
