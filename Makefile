@@ -38,6 +38,14 @@ variant:
 	$(NVCC) $(NVFLAGS) -DGSW_MINB=$(MINB) -shared -o build/var_m$(MINB)/libgsw.so $(CU) -lcudart -ldl \
 	    2> build/var_m$(MINB)/ptxas.txt || (tail -20 build/var_m$(MINB)/ptxas.txt; exit 1)
 
+# A/B variant with arbitrary -D flags: make flagvariant VNAME=pb VFLAGS=-DGSW_PULL_BOUNDS=1
+VNAME ?= x
+VFLAGS ?=
+flagvariant:
+	@mkdir -p build/var_$(VNAME)
+	$(NVCC) $(NVFLAGS) $(VFLAGS) -shared -o build/var_$(VNAME)/libgsw.so $(CU) -lcudart -ldl \
+	    2> build/var_$(VNAME)/ptxas.txt || (tail -20 build/var_$(VNAME)/ptxas.txt; exit 1)
+
 clean:
 	rm -rf build $(LIB) gen/libgswgen.so oracle/liboracle.so cpu_baselines/libompbase.so
 

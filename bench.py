@@ -651,6 +651,12 @@ def run_gsw(args, ws, rank, local):
 
 
 def main():
+    # NCCL writes its banner (NCCL_DEBUG=VERSION, set in this image) and debug log to stdout;
+    # keep stdout for the one JSON line
+    if os.environ.get("NCCL_DEBUG", "").upper() == "VERSION":
+        os.environ.pop("NCCL_DEBUG")
+    elif os.environ.get("NCCL_DEBUG") and not os.environ.get("NCCL_DEBUG_FILE"):
+        os.environ["NCCL_DEBUG_FILE"] = "/dev/stderr"
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=32)

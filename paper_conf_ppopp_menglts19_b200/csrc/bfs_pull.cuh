@@ -20,6 +20,11 @@ namespace gsw {
 constexpr int kPullCur = 4;
 constexpr int kPullWordsPerWarp = 16;
 constexpr int kPullList = kPullWordsPerWarp * 32;
+// GSW_PULL_BOUNDS=1: pass 1 also loads the row bounds of every probed vertex (coalesced, in the
+// same batch as in_first), so a hit's degree needs no later round trip (A/B build knob)
+#ifndef GSW_PULL_BOUNDS
+#define GSW_PULL_BOUNDS 0
+#endif
 static __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict__ fb, unsigned *__restrict__ V,
                                                int *__restrict__ depth, const uint32_t *__restrict__ in_off,
                                                const int32_t *__restrict__ in_col, const int32_t *__restrict__ in_first,
@@ -48,6 +53,10 @@ static __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict
 #pragma unroll 1
         while (nz) {
             int y[8], kk[8];
+#if GSW_PULL_BOUNDS
+            uint32_t hb[8], he[8];
+            const uint32_t *o = symmetric ? in_off : out_off;
+#endif
 #pragma unroll
             for (int j = 0; j < 8; ++j) {
                 kk[j] = nz ? __ffs(nz) - 1 : -1;              // warp-uniform
@@ -58,6 +67,11 @@ static __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict
                 const unsigned wm = __shfl_sync(0xffffffffu, word, kk[j] < 0 ? 0 : kk[j]);
                 const bool act = kk[j] >= 0 && ((wm >> lane) & 1u);   // padding bits are set in V: v < n
                 y[j] = act ? __ldg(in_first + (int)((w0 + kk[j]) * 32 + lane)) : -2;
+#if GSW_PULL_BOUNDS
+                const int vv = (int)((w0 + kk[j]) * 32 + lane);
+                hb[j] = act ? __ldg(o + vv) : 0u;
+                he[j] = act ? __ldg(o + vv + 1) : 0u;
+#endif
             }
             unsigned p[8];
 #pragma unroll
@@ -70,8 +84,12 @@ static __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict
                 if (hit) depth[v] = lvl + 1;
                 const unsigned hm = __ballot_sync(0xffffffffu, hit);
                 if (lane == 0 && kk[j] >= 0) found_bits[kk[j]] = hm;
+#if GSW_PULL_BOUNDS
+                if (hit) cnt.add_vertex(he[j] - hb[j]);
+#else
                 if (hit) list[kPullList - 1 - (nhit + __popc(hm & lanemask_lt()))] = v;
                 nhit += __popc(hm);
+#endif
                 const bool miss = y[j] >= 0 && !hit;
                 const unsigned mm = __ballot_sync(0xffffffffu, miss);
                 if (miss) list[total + __popc(mm & lanemask_lt())] = v;

@@ -17,6 +17,8 @@ constexpr int kMaxHist = 1 << 16;   // iterations with stored history / records
 // level costs ~2.7 us at 1 vertex and ~9 us at 300 vertices, a grid level ~13 us.
 constexpr long long kSoloE = 2048;
 constexpr long long kSoloV = 512;
+constexpr long long kSoloESssp = 512;     // SSSP's near/far rounds (re-calibrated in round 2)
+constexpr long long kSoloVSssp = 256;
 
 struct Hist {
     float tf, te, Tf, Te;

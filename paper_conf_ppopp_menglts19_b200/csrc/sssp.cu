@@ -788,6 +788,10 @@ gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_sta
     LaunchInfo li;
     gsw_status s = prepare_common(g, ws, (const void *)sssp_kernel, a.rc, li, kMinBlocksSssp);
     if (s != GSW_OK) return s;
+    // SSSP's own solo thresholds (profiles/r2/solo_sweep_r2.txt, 2 CTAs/SM build): C2 45.2 ms at
+    // (512 edges, 256 vertices) vs 46.6 ms at BFS's (2,048, 512) and 45.4 ms with the tier off
+    if (!std::getenv("GSW_SOLO_E")) a.rc.solo_e = kSoloESssp;
+    if (!std::getenv("GSW_SOLO_V")) a.rc.solo_v = kSoloVSssp;
     if (!a.dist || !a.nb[2] || !a.q[1] || !a.fq[1] || !a.chg || !a.farbit || !a.flen || !a.split || !a.scan) {
         set_error("workspace too small");
         return GSW_ENOMEM;

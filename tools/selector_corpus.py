@@ -110,14 +110,22 @@ def main():
                 if levels is None:
                     levels = [(r["Va"], r["Ea"], r["Via"], r["Eia"]) for r in recs]
             G.force_config()
-            for t, (Va, Ea, Via, Eia) in enumerate(levels):
+            # road-like graphs have thousands of near-identical levels: keep at most 200 per root
+            keep = range(len(levels)) if len(levels) <= 200 else sorted({int(i * (len(levels) - 1) / 199) for i in range(200)})
+            for t in keep:
+                Va, Ea, Via, Eia = levels[t]
                 rows.append({"graph": g.name, "root": int(s), "t": t, "Va": Va, "Ea": Ea, "Via": Via, "Eia": Eia,
-                             "attrs": attrs, "times": {k: v[t] for k, v in per.items() if t < len(v)}})
+                             "attrs": attrs, "times": {k: round(v[t], 2) for k, v in per.items() if t < len(v)}})
         print(f"{g.name}: n={g.n} nnz={g.nnz} levels={len(levels)} rows={len(rows)} {time.time() - t0:.0f}s", flush=True)
         del G
         torch.cuda.empty_cache()
-    with open(a.json, "w") as f:
-        json.dump(rows, f)
+    if a.json.endswith(".gz"):
+        import gzip
+        with gzip.open(a.json, "wt") as f:
+            json.dump(rows, f)
+    else:
+        with open(a.json, "w") as f:
+            json.dump(rows, f)
 
 
 if __name__ == "__main__":

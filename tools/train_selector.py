@@ -108,7 +108,12 @@ def main():
                     "absolute size; the others are scale-free ratios or distribution shapes)")
     a = ap.parse_args()
     from sklearn.tree import DecisionTreeClassifier
-    rows = [r for r in json.load(open(a.corpus)) if r["Va"] > 0 and len(r["times"]) == 60]
+    if a.corpus.endswith(".gz"):
+        import gzip
+        raw = json.load(gzip.open(a.corpus, "rt"))
+    else:
+        raw = json.load(open(a.corpus))
+    rows = [r for r in raw if r["Va"] > 0 and len(r["times"]) == 60]
     keep = [i for i, f in enumerate(FEATURES) if f not in a.drop.split(",")]
     X = np.array([feats(r) for r in rows])[:, keep]
     best = [min(r["times"], key=r["times"].get) for r in rows]
