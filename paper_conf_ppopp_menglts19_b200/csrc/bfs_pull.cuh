@@ -17,7 +17,14 @@ namespace gsw {
 // list, so a lane's time is the SUM of its scan lengths spread over kPullCur chains rather than
 // the maximum over a warp.  Each vertex has exactly one owner lane, so its visited / next-frontier
 // bits are set with fire-and-forget atomicOr (no returned value, no dependent round trip).
-constexpr int kPullCur = 4;
+#ifndef GSW_PULL_CUR
+#define GSW_PULL_CUR 4
+#endif
+#ifndef GSW_PULL_BATCH
+#define GSW_PULL_BATCH 8
+#endif
+constexpr int kPullCur = GSW_PULL_CUR;       // pass-2 cursors per lane
+constexpr int kPullBatch = GSW_PULL_BATCH;   // pass-1 words probed per batch (loads in flight per lane)
 constexpr int kPullWordsPerWarp = 16;
 constexpr int kPullList = kPullWordsPerWarp * 32;
 // GSW_PULL_BOUNDS=1: pass 1 also loads the row bounds of every probed vertex (coalesced, in the
@@ -52,18 +59,18 @@ static __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict
         unsigned nz = __ballot_sync(0xffffffffu, word != 0u);  // words with unvisited vertices
 #pragma unroll 1
         while (nz) {
-            int y[8], kk[8];
+            int y[kPullBatch], kk[kPullBatch];
 #if GSW_PULL_BOUNDS
-            uint32_t hb[8], he[8];
+            uint32_t hb[kPullBatch], he[kPullBatch];
             const uint32_t *o = symmetric ? in_off : out_off;
 #endif
 #pragma unroll
-            for (int j = 0; j < 8; ++j) {
+            for (int j = 0; j < kPullBatch; ++j) {
                 kk[j] = nz ? __ffs(nz) - 1 : -1;              // warp-uniform
                 nz &= nz - 1u;
             }
 #pragma unroll
-            for (int j = 0; j < 8; ++j) {
+            for (int j = 0; j < kPullBatch; ++j) {
                 const unsigned wm = __shfl_sync(0xffffffffu, word, kk[j] < 0 ? 0 : kk[j]);
                 const bool act = kk[j] >= 0 && ((wm >> lane) & 1u);   // padding bits are set in V: v < n
                 y[j] = act ? __ldg(in_first + (int)((w0 + kk[j]) * 32 + lane)) : -2;
@@ -73,11 +80,11 @@ static __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict
                 he[j] = act ? __ldg(o + vv + 1) : 0u;
 #endif
             }
-            unsigned p[8];
+            unsigned p[kPullBatch];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) p[j] = y[j] >= 0 ? fb[y[j] >> 5] : 0u;
+            for (int j = 0; j < kPullBatch; ++j) p[j] = y[j] >= 0 ? fb[y[j] >> 5] : 0u;
 #pragma unroll
-            for (int j = 0; j < 8; ++j) {
+            for (int j = 0; j < kPullBatch; ++j) {
                 const int v = (int)((w0 + kk[j]) * 32 + lane);
                 const bool hit = y[j] >= 0 && ((p[j] >> (y[j] & 31)) & 1u);
                 if (y[j] >= 0) cnt.edges++;
