@@ -416,7 +416,8 @@ __device__ __noinline__ void bfs_solo(const BfsArgs &a, SoloSmem &ss, int t, lon
     }
 }
 
-__global__ void __launch_bounds__(kBlock, kMinBlocksBfs) bfs_kernel(const __grid_constant__ BfsArgs a) {
+template <int kResident>
+__global__ void __launch_bounds__(kBlock, kResident) bfs_kernel(const __grid_constant__ BfsArgs a) {
     __shared__ BfsSmem bsm;
     LbSmem &sm = bsm.lb;
     __shared__ CtaQStore qs;
@@ -657,13 +658,18 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
     a.iso_count = g->attrs.isolated;
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)bfs_kernel, a.rc, li, kMinBlocksBfs);
+    // Residency per graph shape (profiles/r2/minblocks_ab_*): road-like graphs (mean degree below
+    // 8: thousands of tiny levels) run one CTA per SM, the cheapest grid barrier (C2 28 ms vs 31 ms
+    // at 2/SM); scale-free graphs keep kMinBlocksBfs (C3: 0.177 ms at 2/SM vs 0.23 ms at 1/SM).
+    const bool roadlike = g->attrs.dbar < 8.0 && kMinBlocksBfs >= 2 && !std::getenv("GSW_MINB_BFS_FIXED");
+    const void *kern = roadlike ? (const void *)bfs_kernel<1> : (const void *)bfs_kernel<kMinBlocksBfs>;
+    gsw_status s = prepare_common(g, ws, kern, a.rc, li, roadlike ? 1 : kMinBlocksBfs);
     if (s != GSW_OK) return s;
     // BFS selector: hand-set rules (default) or the learned trees (GSW_SELECTOR=trees)
     if (const char *sel = std::getenv("GSW_SELECTOR")) a.rc.base.selector = std::strcmp(sel, "trees") == 0 ? 1 : 0;
     if (!a.depth || !a.V || !a.fb[2] || !a.q[1] || !a.iq || !a.scan) { set_error("workspace too small"); return GSW_ENOMEM; }
     void *args[] = {&a};
-    s = launch_persistent(g, (const void *)bfs_kernel, args, li);
+    s = launch_persistent(g, kern, args, li);
     if (s != GSW_OK) return s;
     if (!dev_out)
         GSW_CUDA(cudaMemcpyAsync(depth_out, relabeled ? a.out : a.depth, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));

@@ -98,7 +98,7 @@ enum DistMode { DM_NCCL = 0, DM_LOOPBACK = 1, DM_HOST = 2 };
 
 constexpr uint32_t kHeavy = 1024;      // rows above this many edges become 1024-edge warp tasks
 constexpr int kMaxLevels = 1 << 16;    // per-level records kept on the device
-constexpr int kLookahead = 2;          // levels enqueued past the one whose done flag is polled
+constexpr int kLookaheadMax = 4;       // levels enqueued past the one whose done flag is polled (max)
 
 struct DTask {
     int row;
@@ -166,8 +166,10 @@ struct DistState {
     gsw_exchange hx{};                      // host-staged backend callbacks
     unsigned char *hsend = nullptr, *hrecv = nullptr;   // pinned staging (host mode)
     size_t hcap = 0;
-    int *hdone = nullptr;                   // pinned done flags, one per lookahead slot
-    cudaEvent_t evs[kLookahead + 1] = {};
+    int *hdone = nullptr;                   // mapped pinned done flags, one per lookahead slot
+    int *hdone_dev = nullptr;               // their device alias (written by k_publish_done)
+    int lookahead = 1;                      // GSW_DIST_LOOKAHEAD (1..4); 1 measured best (profiles/r2/part_ab.txt)
+    cudaEvent_t evs[kLookaheadMax + 1] = {};
 };
 
 int64_t dist_slice(int64_t n, int32_t p) {
@@ -1048,7 +1050,9 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
     }
     for (auto &ev : d->evs)
         if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "events"));
-    if (cudaHostAlloc((void **)&d->hdone, sizeof(int) * (kLookahead + 1), cudaHostAllocDefault) != cudaSuccess)
+    if (const char *e = getenv("GSW_DIST_LOOKAHEAD")) d->lookahead = std::max(1, std::min(kLookaheadMax, atoi(e)));
+    if (cudaHostAlloc((void **)&d->hdone, sizeof(int) * (kLookaheadMax + 1), cudaHostAllocMapped) != cudaSuccess ||
+        cudaHostGetDevicePointer((void **)&d->hdone_dev, d->hdone, 0) != cudaSuccess)
         return fail(cuda_fail(cudaGetLastError(), "pinned flags"));
     Workspace ws{g->ws, ws_bytes, 0};
     d->FB[0] = (unsigned *)ws.take(d->npad / 8);
@@ -1193,11 +1197,18 @@ void dist_destroy(DistState *d) {
 // Pipelined termination: after enqueueing iteration t, poll the done flag of iteration
 // t - LOOKAHEAD (host mode: of t itself, its exchange has synchronised already).  Returns through
 // *stop whether the host should stop enqueueing.
+__global__ void k_publish_done(const DCtl *ctl, volatile int *flag) {
+    if (threadIdx.x == 0) { *flag = ctl->done; __threadfence_system(); }
+}
+
 static gsw_status poll_done(DistState *d, int t, cudaStream_t s, bool *stop) {
-    const int R = kLookahead + 1;
-    GSW_CUDA(cudaMemcpyAsync(d->hdone + (t % R), &d->ctl->done, 4, cudaMemcpyDeviceToHost, s));
+    const int R = d->lookahead + 1;
+    // the flag goes to mapped host memory from a one-thread kernel: no copy-engine round trip in
+    // the stream between two levels
+    k_publish_done<<<1, 32, 0, s>>>(d->ctl, d->hdone_dev + (t % R));
+    GSW_CUDA(cudaGetLastError());
     GSW_CUDA(cudaEventRecord(d->evs[t % R], s));
-    const int lag = d->mode == DM_HOST ? 0 : kLookahead;
+    const int lag = d->mode == DM_HOST ? 0 : d->lookahead;
     *stop = false;
     if (t >= lag) {
         GSW_CUDA(cudaEventSynchronize(d->evs[(t - lag) % R]));

@@ -459,7 +459,8 @@ union SsSmem {
 };
 static_assert(sizeof(SsSoloSmem) <= sizeof(LbSmem), "the solo tier must not grow the kernel's shared memory");
 
-__global__ void __launch_bounds__(kBlock, kMinBlocksSssp) sssp_kernel(const __grid_constant__ SsspArgs a) {
+template <int kResident>
+__global__ void __launch_bounds__(kBlock, kResident) sssp_kernel(const __grid_constant__ SsspArgs a) {
     __shared__ SsSmem sm;
     __shared__ uint32_t red[kWarps + 1];
     __shared__ CtaQStore qs0, qs1;        // staged appends: near queue, far queue
@@ -786,7 +787,12 @@ gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_sta
     a.law = kDefaultLaw;
     if (const char *law = getenv("GSW_SSSP_LAW")) a.law = atoi(law);
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)sssp_kernel, a.rc, li, kMinBlocksSssp);
+    // Residency per graph shape (profiles/r2/minblocks_ab_*): on road-like graphs (mean degree
+    // below 8: every round is a few hundred to a few thousand vertices) one CTA per SM gives the
+    // cheapest grid barrier (C2 43 ms vs 46 ms at 2/SM); scale-free graphs keep kMinBlocksSssp.
+    const bool roadlike = g->attrs.dbar < 8.0 && kMinBlocksSssp >= 2 && !std::getenv("GSW_MINB_SSSP_FIXED");
+    const void *kern = roadlike ? (const void *)sssp_kernel<1> : (const void *)sssp_kernel<kMinBlocksSssp>;
+    gsw_status s = prepare_common(g, ws, kern, a.rc, li, roadlike ? 1 : kMinBlocksSssp);
     if (s != GSW_OK) return s;
     // SSSP's own solo thresholds (profiles/r2/solo_sweep_r2.txt, 2 CTAs/SM build): C2 45.2 ms at
     // (512 edges, 256 vertices) vs 46.6 ms at BFS's (2,048, 512) and 45.4 ms with the tier off
@@ -797,7 +803,7 @@ gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist_out, gsw_run_sta
         return GSW_ENOMEM;
     }
     void *args[] = {&a};
-    s = launch_persistent(g, (const void *)sssp_kernel, args, li);
+    s = launch_persistent(g, kern, args, li);
     if (s != GSW_OK) return s;
     if (!dev_out)
         GSW_CUDA(cudaMemcpyAsync(dist_out, relabeled ? a.out : a.dist, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
