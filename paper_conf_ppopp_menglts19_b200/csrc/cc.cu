@@ -60,9 +60,17 @@ struct CcPushOp {
     }
 };
 
-// pull: label[v] = min(label[v], min over active in-neighbours u of label[u])
+// pull: label[v] = min(label[v], min over active in-neighbours u of label[u]), then the
+// pointer-jumping shortcut label[v] = min(that, label[x]) with x the vertex whose id is that label
+// (Soman et al. [53]; R17): labels are ids of same-component vertices and
+// never exceed their own vertex's id, so the fixpoint (the component's minimum id) is unchanged
+// and long label chains collapse in fewer iterations.  GSW_CC_JUMP=0 builds without it (A/B).
+#ifndef GSW_CC_JUMP
+#define GSW_CC_JUMP 1
+#endif
 struct CcPullOp {
     int *label;
+    const uint32_t *inv;         // caller id -> internal id (labels are caller ids), or nullptr
     const unsigned *fb;          // active set
     const uint32_t *off;         // out-offsets (degree of a changed vertex)
     bool fused;
@@ -81,6 +89,13 @@ struct CcPullOp {
     __device__ __forceinline__ void flush(int v, Acc m, bool exclusive, LocalCnt &c) const {
         if (m == identity()) return;
         int mi = (int)m;
+#if GSW_CC_JUMP
+        if (mi < label[v]) {
+            const int x = inv ? (int)__ldg(inv + mi) : mi;
+            const int lx = label[x];
+            mi = lx < mi ? lx : mi;
+        }
+#endif
         unsigned bit = 1u << (v & 31);
         if (exclusive) {
             if (mi < label[v]) {
@@ -207,7 +222,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksCc) cc_kernel(CcArgs a) {
             else
                 lc = run_lb(c.lb, QueueSrc{a.q, qlen}, adj_out, op, sm.push, red, bar, epoch, rc.partial, a.scan);
         } else {
-            const CcPullOp op{a.label, fbt, a.g.off, fused, mark};
+            const CcPullOp op{a.label, a.g.inv, fbt, a.g.off, fused, mark};
             if (c.lb == GSW_LB_TWC)
                 lc = lbr_tiered(op, adj_in, tiers, n);          // B200 TWC: warp-seg / warp / grid tiers
             else

@@ -31,7 +31,10 @@ namespace gsw {
 
 constexpr int kSBlock = 1024;
 constexpr int kSWarps = kSBlock / 32;
-constexpr int kEpt = 8;                       // edges per lane per warp-tile
+#ifndef GSW_PR_EPT
+#define GSW_PR_EPT 8
+#endif
+constexpr int kEpt = GSW_PR_EPT;              // edges per lane per warp-tile (A/B knob: GSW_PR_EPT)
 constexpr int kWt = 32 * kEpt;                // edges per warp-tile
 constexpr int kWBuf = 320;                    // row offsets a warp keeps in shared memory per tile
 
