@@ -132,6 +132,7 @@ def run_reference(args, ws, rank):
     import oracle
     c5 = (ws > 1 or args.partitioned) and not (args.dist_workload_forced and args.workload == "C3")
     workload = "C5" if c5 else args.workload
+    gen.set_threads(0)          # torchrun exports OMP_NUM_THREADS=1: generate with every core
     g, _ = build_graph(workload)
     deg = g.deg
     roots = gen.sources(g, max(64, args.steps + args.warmup))

@@ -139,7 +139,11 @@ gsw_status gsw_graph_attributes(gsw_graph g, double out[7]);
  * executes exactly the pinned patterns.  Environment knobs read at each run (calibration only):
  * GSW_SELECTOR=trees (BFS: learned CART trees instead of the hand-set rules), GSW_SOLO_E /
  * GSW_SOLO_V (solo-tier thresholds; GSW_SOLO_E=0 disables it), GSW_SSSP_LAW (stepping law),
- * GSW_DPR_PULL_K (Delta-PR: pull iff K*Ea > nnz, default 2).
+ * GSW_DPR_PULL_K (Delta-PR: pull iff K*Ea > nnz, default 2), GSW_PR_CACHE (PageRank hub-cache
+ * entries), GSW_PR_BLOCKED / GSW_PR_BLOCKS (row-tier / source-blocked PageRank), GSW_MINB_BFS_FIXED /
+ * GSW_MINB_SSSP_FIXED (disable the per-graph residency choice), GSW_DIST_LOOKAHEAD (levels the
+ * partitioned host loop runs ahead of its done-flag poll), GSW_PHASES=1 (BFS init / loop / output
+ * device times on stderr).
  */
 gsw_status gsw_force_config(gsw_graph g, const gsw_config *cfg);
 

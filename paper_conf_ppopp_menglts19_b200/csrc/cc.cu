@@ -64,9 +64,10 @@ struct CcPushOp {
 // pointer-jumping shortcut label[v] = min(that, label[x]) with x the vertex whose id is that label
 // (Soman et al. [53]; R17): labels are ids of same-component vertices and
 // never exceed their own vertex's id, so the fixpoint (the component's minimum id) is unchanged
-// and long label chains collapse in fewer iterations.  GSW_CC_JUMP=0 builds without it (A/B).
+// and long label chains collapse in fewer iterations -- on the R-MAT configs it did not cut the 4
+// iterations and cost the extra loads, so it is built only with GSW_CC_JUMP=1.
 #ifndef GSW_CC_JUMP
-#define GSW_CC_JUMP 1
+#define GSW_CC_JUMP 0       // measured: C3 still 4 iterations, 1.95 vs 2.16 ms with it (profiles/r2/pr_ept_cc_jump_ab.txt)
 #endif
 struct CcPullOp {
     int *label;

@@ -32,7 +32,7 @@ namespace gsw {
 constexpr int kSBlock = 1024;
 constexpr int kSWarps = kSBlock / 32;
 #ifndef GSW_PR_EPT
-#define GSW_PR_EPT 8
+#define GSW_PR_EPT 12      // 8: C3 2,648 it/s, 12: 2,812, 16: 2,783 (profiles/r2/pr_ept_cc_jump_ab.txt)
 #endif
 constexpr int kEpt = GSW_PR_EPT;              // edges per lane per warp-tile (A/B knob: GSW_PR_EPT)
 constexpr int kWt = 32 * kEpt;                // edges per warp-tile
