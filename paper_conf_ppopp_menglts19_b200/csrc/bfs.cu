@@ -10,8 +10,11 @@
 // Status (Fig. 11 filter): Active = depth==t, Inactive = depth<0 (not in the visited map),
 // Fixed = visited earlier.  compAtomic = atomicExch in the paper is applied only to
 // Inactive targets (reading R3): an atomicOr test-and-set on the visited bitmap.
+#include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <vector>
 
 #include "engine.cuh"
 #include "internal.h"
@@ -22,6 +25,16 @@
 namespace gsw {
 
 enum { MAT_NONE = 0, MAT_QUEUE = 1, MAT_SQUEUE = 2, MAT_BITMAP = 3 };
+
+// GSW_PULL_PROF=1 (diagnostic builds only): per-warp entry/exit %globaltimer of the list pull of
+// every level, summarised on stderr after each run (where a pull level's time goes: the slowest
+// warps vs the median)
+#ifndef GSW_PULL_PROF
+#define GSW_PULL_PROF 0
+#endif
+#if GSW_PULL_PROF
+__device__ unsigned long long g_pull_prof[8][16384][2];
+#endif
 
 struct BfsArgs {
     DevGraph g;
@@ -585,8 +598,17 @@ __global__ void __launch_bounds__(kBlock, kResident) bfs_kernel(const __grid_con
             const BfsPullOp op{depth, a.V, a.g.off, c.fmt == GSW_BITMAP ? fbt : nullptr, t, fused, a.fb[(t + 1) % 3]};
             if (c.fmt == GSW_BITMAP && c.lb == GSW_LB_THREAD) {
                 static_assert(sizeof(LbSmem) >= sizeof(int) * (kPullList + kPullWordsPerWarp) * kWarps, "pull lists live in the LB smem");
+#if GSW_PULL_PROF
+                const unsigned long long p0 = globaltimer();
+#endif
                 lc = bfs_pull_list(fbt, a.V, depth, a.g.in_off, a.g.in_col, a.g.in_first, a.g.off, a.g.in_off == a.g.off, t,
                                    fused ? a.fb[(t + 1) % 3] : nullptr, n, reinterpret_cast<int *>(&sm));
+#if GSW_PULL_PROF
+                if (t < 8 && lane_id() == 0) {
+                    const long long w = gwarp();
+                    if (w < 16384) { g_pull_prof[t][w][0] = p0; g_pull_prof[t][w][1] = globaltimer(); }
+                }
+#endif
             } else if (c.fmt == GSW_BITMAP) {
                 lc = run_lb(c.lb, BitmapSrc{a.V, (unsigned)n, 0u}, adj_in, op, sm, red, bar, epoch, rc.partial, a.scan);
             } else {
@@ -671,6 +693,30 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     void *args[] = {&a};
     s = launch_persistent(g, kern, args, li);
     if (s != GSW_OK) return s;
+#if GSW_PULL_PROF
+    {
+        static unsigned long long h[8][16384][2];
+        GSW_CUDA(cudaStreamSynchronize(g->stream));
+        GSW_CUDA(cudaMemcpyFromSymbol(h, g_pull_prof, sizeof(h)));
+        const int nw = li.grid * (kBlock / 32);
+        for (int lv = 0; lv < 8; ++lv) {
+            std::vector<double> d;
+            unsigned long long lo = ~0ull, hi = 0;
+            for (int w = 0; w < nw && w < 16384; ++w) {
+                if (!h[lv][w][0] || h[lv][w][1] < h[lv][w][0]) continue;
+                d.push_back((double)(h[lv][w][1] - h[lv][w][0]) * 1e-3);
+                lo = std::min(lo, h[lv][w][0]); hi = std::max(hi, h[lv][w][1]);
+            }
+            if (d.empty()) continue;
+            std::sort(d.begin(), d.end());
+            std::fprintf(stderr, "pull level %d: warps %zu span %.2f us  warp us: min %.2f p50 %.2f p90 %.2f p99 %.2f max %.2f\n",
+                         lv, d.size(), (hi - lo) * 1e-3, d.front(), d[d.size() / 2], d[d.size() * 9 / 10],
+                         d[d.size() * 99 / 100], d.back());
+        }
+        static const unsigned long long z[8][16384][2] = {};
+        GSW_CUDA(cudaMemcpyToSymbol(g_pull_prof, z, sizeof(z)));
+    }
+#endif
     if (!dev_out)
         GSW_CUDA(cudaMemcpyAsync(depth_out, relabeled ? a.out : a.depth, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
     return finish_run(g, a.rc, li, st);

@@ -24,6 +24,14 @@ namespace gsw {
 #define GSW_PULL_BATCH 8
 #endif
 constexpr int kPullCur = GSW_PULL_CUR;       // pass-2 cursors per lane
+// Chunk hand-out: each CTA owns the chunks blockIdx.x, blockIdx.x + gridDim.x, ... (so every CTA
+// sees every region of the degree-ordered id range) and its warps take them one at a time from a
+// shared-memory counter.  Measured per warp (GSW_PULL_PROF, profiles/r2/pull_warp_profile_c3.txt):
+// with the static warp-strided hand-out C3's widest pull level took 51-56 us while the median warp
+// finished in 23 us -- the level's time was its slowest warps.  GSW_PULL_DYN=0: static hand-out.
+#ifndef GSW_PULL_DYN
+#define GSW_PULL_DYN 1
+#endif
 constexpr int kPullBatch = GSW_PULL_BATCH;   // pass-1 words probed per batch (loads in flight per lane)
 constexpr int kPullWordsPerWarp = 16;
 constexpr int kPullList = kPullWordsPerWarp * 32;
@@ -42,7 +50,20 @@ static __device__ __noinline__ LocalCnt bfs_pull_list(const unsigned *__restrict
     const unsigned lane = lane_id();
     int *list = lists + (threadIdx.x >> 5) * (kPullList + kPullWordsPerWarp);
     unsigned *found_bits = reinterpret_cast<unsigned *>(list + kPullList);
+#if GSW_PULL_DYN
+    __shared__ unsigned s_next;
+    __syncthreads();
+    if (threadIdx.x == 0) s_next = 0u;
+    __syncthreads();
+    for (;;) {
+        unsigned k = 0;
+        if (lane == 0) k = atomicAdd(&s_next, 1u);
+        k = __shfl_sync(0xffffffffu, k, 0);
+        const long long chunk = blockIdx.x + (long long)k * gridDim.x;
+        if (chunk * kPullWordsPerWarp >= W) break;
+#else
     for (long long chunk = gwarp(); chunk * kPullWordsPerWarp < W; chunk += gwarps()) {
+#endif
         const long long w0 = chunk * kPullWordsPerWarp;
         unsigned word = 0, orig = ~0u;
         if (lane < (unsigned)kPullWordsPerWarp && w0 + lane < W) {
