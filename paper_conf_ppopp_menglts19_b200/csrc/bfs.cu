@@ -680,12 +680,19 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
     a.iso_count = g->attrs.isolated;
     LaunchInfo li;
-    // Residency per graph shape (profiles/r2/minblocks_ab_*): road-like graphs (mean degree below
-    // 8: thousands of tiny levels) run one CTA per SM, the cheapest grid barrier (C2 28 ms vs 31 ms
-    // at 2/SM); scale-free graphs keep kMinBlocksBfs (C3: 0.177 ms at 2/SM vs 0.23 ms at 1/SM).
-    const bool roadlike = g->attrs.dbar < 8.0 && kMinBlocksBfs >= 2 && !std::getenv("GSW_MINB_BFS_FIXED");
-    const void *kern = roadlike ? (const void *)bfs_kernel<1> : (const void *)bfs_kernel<kMinBlocksBfs>;
-    gsw_status s = prepare_common(g, ws, kern, a.rc, li, roadlike ? 1 : kMinBlocksBfs);
+    // Residency per graph shape (profiles/r2/minblocks_ab_*, ab_m4.txt): road-like graphs (mean
+    // degree below 8: thousands of tiny levels) run one CTA per SM, the cheapest grid barrier (C2
+    // 28 ms vs 31 ms at 2/SM); scale-free graphs keep kMinBlocksBfs (C3: 0.150 ms at 2/SM vs 0.174
+    // at 4/SM, 0.23 at 1/SM), except very large ones (2^24+ vertices), whose levels are long enough
+    // that the extra warps hiding gather latency outweigh the dearer barrier (C5: 1.05 / 2.21 ms per
+    // root at 4/SM vs 1.29 / 3.09 ms at 2/SM).
+    const bool fixed = std::getenv("GSW_MINB_BFS_FIXED") != nullptr;
+    const bool roadlike = g->attrs.dbar < 8.0 && kMinBlocksBfs >= 2 && !fixed;
+    const bool huge = !roadlike && n >= (1ll << 24) && kMinBlocksBfs == 2 && !fixed;
+    const void *kern = roadlike ? (const void *)bfs_kernel<1>
+                       : huge   ? (const void *)bfs_kernel<4>
+                                : (const void *)bfs_kernel<kMinBlocksBfs>;
+    gsw_status s = prepare_common(g, ws, kern, a.rc, li, roadlike ? 1 : huge ? 4 : kMinBlocksBfs);
     if (s != GSW_OK) return s;
     // BFS selector: hand-set rules (default) or the learned trees (GSW_SELECTOR=trees)
     if (const char *sel = std::getenv("GSW_SELECTOR")) a.rc.base.selector = std::strcmp(sel, "trees") == 0 ? 1 : 0;
