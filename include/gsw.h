@@ -159,6 +159,18 @@ gsw_status gsw_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *
 /* Connected components: label[v] = min vertex id of v's component.               */
 gsw_status gsw_cc(gsw_graph g, int32_t *label, gsw_run_stats *stats);
 
+/* Connected components by hooking + pointer jumping: the edge-centric GPU CC the paper compares
+ * its CC against (Soman et al. [53], reading Q8).  Each iteration sweeps
+ * every edge and hangs the tree with the larger root id below the other root (atomicMin on packed
+ * (caller id, internal id) parent pointers), then compresses every pointer to its root; it stops
+ * after a sweep in which no hook succeeded.  Output identical to gsw_cc: label[v] = min vertex id
+ * of v's component.  label: n int32, host or device.  gsw_force_config's load_balance selects the
+ * sweep's mapping (AUTO: THREAD when the degree range r_d <= 16, else STRICT); its other fields
+ * are ignored.  stats->records: one per iteration,
+ * Va = successful hooks, edges = adjacency entries swept.
+ * Errors: GSW_EINVAL (NULL label), GSW_EUNSUPPORTED (distributed handle).                     */
+gsw_status gsw_cc_hook(gsw_graph g, int32_t *label, gsw_run_stats *stats);
+
 /* PageRank power iteration: pr_0 = 1/N, exactly `iters` iterations of
  *   pr'(v) = (1-d)/N + d * (sum_{u->v} pr(u)/deg_out(u) + D/N),  D = sum of dangling pr.
  * rank: n doubles, host or device.                                                            */

@@ -178,6 +178,14 @@ class Graph:
         check(_lib.load().gsw_cc(self._h, out.data_ptr(), ctypes.byref(st)), "gsw_cc")
         return out, _stats_dict(st, recs)
 
+    def cc_hook(self, out=None, records: int = 0):
+        """Connected components by hooking + pointer jumping (Soman et al.)."""
+        import torch
+        out = self._out(out, torch.int32)
+        st, recs = self._stats(records)
+        check(_lib.load().gsw_cc_hook(self._h, out.data_ptr(), ctypes.byref(st)), "gsw_cc_hook")
+        return out, _stats_dict(st, recs)
+
     def pr(self, damping: float = 0.85, iters: int = 20, out=None, records: int = 0):
         import torch
         out = self._out(out, torch.float64)

@@ -80,6 +80,7 @@ SIGNATURES = {
     "gsw_bfs": (ctypes.c_int, [_P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_sssp": (ctypes.c_int, [_P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_cc": (ctypes.c_int, [_P, _P, ctypes.POINTER(gsw_run_stats)]),
+    "gsw_cc_hook": (ctypes.c_int, [_P, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_pr": (ctypes.c_int, [_P, ctypes.c_double, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_dpr": (ctypes.c_int, [_P, ctypes.c_double, ctypes.c_double, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),
     "gsw_bc": (ctypes.c_int, [_P, _P, ctypes.c_int32, _P, ctypes.POINTER(gsw_run_stats)]),

@@ -16,6 +16,8 @@
 #include <cstring>
 #include <vector>
 
+#include <cooperative_groups.h>
+
 #include "engine.cuh"
 #include "internal.h"
 #include "launch.h"
@@ -23,6 +25,7 @@
 #include "bfs_pull.cuh"
 
 namespace gsw {
+namespace cg = cooperative_groups;
 
 enum { MAT_NONE = 0, MAT_QUEUE = 1, MAT_SQUEUE = 2, MAT_BITMAP = 3 };
 
@@ -34,6 +37,20 @@ enum { MAT_NONE = 0, MAT_QUEUE = 1, MAT_SQUEUE = 2, MAT_BITMAP = 3 };
 #endif
 #if GSW_PULL_PROF
 __device__ unsigned long long g_pull_prof[8][16384][2];
+#endif
+// GSW_TEAM_PROF=1 (diagnostic builds only): per-phase %globaltimer sums of the team tier's levels
+// (CTA 0 and CTA k-1, thread 0), printed on stderr after each run
+#ifndef GSW_TEAM_PROF
+#define GSW_TEAM_PROF 0
+#endif
+
+#if GSW_TEAM_PROF
+__device__ unsigned long long g_team_prof[2][10];
+__device__ unsigned long long g_team_late[16];
+#define TEAM_STAMP(i) do { if (tid == 0) { const unsigned long long nw = globaltimer(); \
+    tp_acc[i] += nw - tp_last; tp_last = nw; } } while (0)
+#else
+#define TEAM_STAMP(i) do { } while (0)
 #endif
 
 struct BfsArgs {
@@ -429,6 +446,345 @@ __device__ __noinline__ void bfs_solo(const BfsArgs &a, SoloSmem &ss, int t, lon
     }
 }
 
+// ---------------------------------------------------------------- cluster tier (team)
+// The solo tier's per-level cost grows by ~2.3 ns per edge on its single SM (C2, tools/round_stats.py:
+// 2.9 us at one vertex, 9 us at ~700 vertices): one SM issues about one scattered L1/L2 request
+// per clock, so a 1,000-4,000-edge level is throughput-bound on that SM while the grid path pays
+// its fixed ~7 us of barrier and dependent round trips.  On road-like graphs the persistent
+// kernel is launched as thread-block clusters of k CTAs (one per SM) and the k CTAs of cluster 0
+// run the small levels together; the other clusters park at one grid barrier as in the solo tier.
+//   * each team CTA keeps its part of the frontier (vertex, row begin, degree) in its own shared
+//     memory, triple-buffered by level;
+//   * per level, one hardware cluster barrier: every CTA publishes (|part|, sum/max/min degree)
+//     and reads all k records through distributed shared memory (one DSMEM round trip), so every
+//     CTA evaluates the same Inspector totals and the same selector decision; CTA 0's history
+//     features travel in its record;
+//   * CTA r expands vertices [V r/k, V (r+1)/k) of the concatenated frontier, read from the
+//     owners' shared memory (DSMEM), with the solo tier's merge-path edge split, column loads and
+//     claim + speculative offsets round trips; winners append to the claiming CTA's own part;
+//   * capacity is checked before a level is run (max degree x ceil(V/k) <= kTQ), so no CTA can
+//     overflow its part; a level that does not fit ends the episode and the parts are handed
+//     back to the grid as one queue.
+constexpr int kTQ = 512;       // frontier part per team CTA
+constexpr int kTeamMax = 16;   // cluster size limit (non-portable 16)
+struct TeamRec {
+    unsigned qn, maxd, mind, pad;
+    unsigned long long ea;
+    float4 hist;               // CTA 0 only: history features of this level (lag-2 protocol)
+#if GSW_TEAM_PROF
+    unsigned long long t_arr;
+#endif
+};
+struct TeamSmem {
+    int q[3][kTQ];
+    uint32_t beg[3][kTQ];
+    uint16_t deg[3][kTQ];          // saturated at 65535 (a level with such a vertex fails the capacity check)
+    uint32_t sbeg[kTQ];
+    uint32_t sscan[kTQ + 1];
+    TeamRec rec[2];
+    unsigned cq[kTeamMax + 1];     // prefix of the parts' sizes
+    unsigned long long ea;
+    unsigned maxd, mind, qn_next;
+    int go;
+    float4 hist;
+    unsigned wmx[kWarps], wmn[kWarps];
+    unsigned long long wsum[kWarps];
+    uint32_t red[kWarps + 1];
+    unsigned long long book_raw[(sizeof(Book) + 7) / 8];
+    long long prev_va;
+};
+static_assert(sizeof(TeamSmem) <= sizeof(BfsSmem), "the team tier must not grow the kernel's shared memory");
+
+// Runs levels t, t+1, ... on the k CTAs of cluster 0 until the selector or the capacity check
+// ends the episode; returns with AS_t in a.q[t & 1] (parts concatenated in CTA order), its
+// counters in rc.cnt[t % 3] and the loop state in rc.pub (written by CTA 0).  Called by all
+// threads of CTAs 0..k-1 (cluster 0), which all see the same totals and take the same decisions.
+#ifndef GSW_TEAM_INLINE
+#define GSW_TEAM_INLINE 0
+#endif
+#if GSW_TEAM_INLINE
+__device__ __forceinline__
+#else
+__device__ __noinline__
+#endif
+void bfs_team(const BfsArgs &a, TeamSmem &ts, int t, long long Via, long long Eia,
+                                      const Features fbase, unsigned qn0, int k) {
+    cg::cluster_group cl = cg::this_cluster();
+    const unsigned tid = threadIdx.x, r = blockIdx.x;
+    const bool book0 = r == 0 && tid == 0;
+    Book &book = *reinterpret_cast<Book *>(ts.book_raw);   // CTA 0 / thread 0 only
+    long long &prev_va = ts.prev_va;
+    const RunCommon &rc = a.rc;
+    const uint32_t *__restrict__ off = a.g.off;
+    const int32_t *__restrict__ col = a.g.col;
+    unsigned *V = a.V;
+    int *depth = a.depth;
+    const long long se = rc.solo_e;
+    // AS_t0: my share of the grid's queue, with offsets
+    unsigned qn_l;
+    {
+        const unsigned s0 = (unsigned)((unsigned long long)qn0 * r / k);
+        qn_l = (unsigned)((unsigned long long)qn0 * (r + 1) / k) - s0;
+        const int *gq = a.q[t & 1] + s0;
+        for (unsigned i0 = tid; i0 < qn_l; i0 += kBlock * 4) {
+            int u[4];
+            uint32_t b[4], e[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) u[j] = i0 + j * kBlock < qn_l ? gq[i0 + j * kBlock] : -1;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                b[j] = u[j] >= 0 ? __ldg(off + u[j]) : 0u;
+                e[j] = u[j] >= 0 ? __ldg(off + u[j] + 1) : 0u;
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                if (u[j] < 0) continue;
+                const unsigned i = i0 + j * kBlock;
+                ts.q[0][i] = u[j]; ts.beg[0][i] = b[j]; ts.deg[0][i] = (uint16_t)min(e[j] - b[j], 65535u);
+            }
+        }
+    }
+    float4 hist = make_float4(0.f, 0.f, 0.f, 0.f);   // CTA 0 / thread 0: history of the next level
+    if (book0) {      // the main loop's book_start(t) wrote the history of t+1
+        const IterCnt *cs = rc.cnt + ((t + 1) % 3);
+        hist = make_float4(cs->tf, cs->te, cs->Tf, cs->Te);
+    }
+    int cur = 0, par = 0;
+    bool first = true;
+    unsigned long long E_prev = 0, Ea = 0;
+    unsigned mxd = 0, mnd = 0, qn = 0;
+#if GSW_TEAM_PROF
+    unsigned long long tp_last = globaltimer(), tp_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+    unsigned long long tp_late = 0;
+#endif
+    for (;;) {
+        // (A) my part's features -> my record
+        __syncthreads();
+        TEAM_STAMP(0);
+        {
+            unsigned long long lea = 0;
+            unsigned lmx = 0, lmn = 0xffffffffu;
+            for (unsigned i = tid; i < qn_l; i += kBlock) {
+                const unsigned d = ts.deg[cur][i];
+                lea += d;
+                lmx = d > lmx ? d : lmx;
+                lmn = d < lmn ? d : lmn;
+            }
+            lea = warp_sum(lea);
+            lmx = warp_max(lmx);
+            lmn = warp_min(lmn);
+            const unsigned w = tid >> 5;
+            if (lane_id() == 0) { ts.wsum[w] = lea; ts.wmx[w] = lmx; ts.wmn[w] = lmn; }
+            __syncthreads();
+            if (tid == 0) {
+                for (int i = 1; i < kWarps; ++i) {
+                    lea += ts.wsum[i];
+                    lmx = max(lmx, ts.wmx[i]);
+                    lmn = min(lmn, ts.wmn[i]);
+                }
+                TeamRec &m = ts.rec[par];
+                m.qn = qn_l; m.maxd = lmx; m.mind = lmn; m.ea = lea; m.hist = hist;
+#if GSW_TEAM_PROF
+                m.t_arr = globaltimer();
+#endif
+            }
+        }
+        TEAM_STAMP(1);
+        cluster_barrier();
+        TEAM_STAMP(2);
+        // (B) every part's record (warp 0: lane c reads CTA c) -> totals and the parts' prefix
+        if (tid < 32) {
+            const unsigned c = tid;
+            unsigned cqn = 0, cmx = 0, cmn = 0xffffffffu;
+            unsigned long long cea = 0;
+            float4 h = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (c < (unsigned)k) {
+                const TeamRec *rm = cl.map_shared_rank(&ts.rec[par], c);
+                cqn = rm->qn; cmx = rm->maxd; cmn = rm->mind; cea = rm->ea;
+                if (c == 0) h = rm->hist;
+            }
+#if GSW_TEAM_PROF
+            {
+                const unsigned long long ta = c < (unsigned)k ? cl.map_shared_rank(&ts.rec[par], c)->t_arr : ~0ull;
+                unsigned long long mn = ta;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) { const unsigned long long x = __shfl_xor_sync(0xffffffffu, mn, o); mn = x < mn ? x : mn; }
+                if (r == 0 && c < (unsigned)k) tp_late += ta - mn;
+                if (r == 0 && c == 0) TEAM_STAMP(9);
+            }
+#endif
+            const unsigned inc = warp_incl_scan(cqn);
+            if (c < (unsigned)k) ts.cq[c + 1] = inc;
+            cea = warp_sum(cea);
+            cmx = warp_max(cmx);
+            cmn = warp_min(cmn);
+            if (c == 0) {
+                ts.cq[0] = 0u;
+                ts.ea = cea; ts.maxd = cmx; ts.mind = cmn;
+                ts.hist = h;
+            }
+        }
+        __syncthreads();
+        TEAM_STAMP(3);
+        qn = ts.cq[k];
+        Ea = ts.ea; mxd = ts.maxd; mnd = ts.mind;
+        // (C) the selector on AS_t's totals (identical inputs in every team CTA)
+        if (tid == 0) {
+            int go = first ? 1 : 0;
+            if (!first && qn > 0) {
+                Features f = fbase;
+                f.Va = (long long)qn; f.Ea = (long long)Ea; f.Via = Via - (long long)qn; f.Eia = Eia - (long long)Ea;
+                f.maxd = mxd; f.mind = mnd; f.iter = t;
+                const float4 h = ts.hist;
+                f.tf = h.x; f.te = h.y; f.Tf = h.z; f.Te = h.w;
+                DevCfg c = select_traversal(f, rc.force);
+                const unsigned per = (qn + (unsigned)k - 1) / (unsigned)k;
+                const bool fits = per <= (unsigned)kTQ && (unsigned long long)mxd * per <= (unsigned long long)kTQ;
+                if (c.dir == GSW_PUSH && c.fused == GSW_FUSED && fits && (long long)Ea <= se) {
+                    go = 1;
+                    if (r == 0) {
+                        c.fmt = GSW_QUEUE;
+                        book.bytes += 12ull * (unsigned long long)prev_va + 4ull * E_prev + 8ull * qn;
+                        book.edges += E_prev;
+                        if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)E_prev;
+                        hist = book_start(book, rc, t, rc.cnt + ((t + 1) % 3));
+                        write_record(rc, t, c, f, 0u);
+                        reset_cnt(rc.cnt + ((t + 2) % 3));
+                    }
+                }
+            }
+            if (go && r == 0 && t < kMaxHist) rc.rec[t].ctas = k;
+            ts.go = go;
+            ts.qn_next = 0u;
+        }
+        __syncthreads();
+        TEAM_STAMP(4);
+        if (!ts.go) break;
+        if (!first) { Via -= (long long)qn; Eia -= (long long)Ea; }
+        // (D) my slice [qn r/k, qn (r+1)/k) of the concatenated frontier, from its owners (DSMEM)
+        const unsigned vs = (unsigned)((unsigned long long)qn * r / k);
+        const unsigned m = (unsigned)((unsigned long long)qn * (r + 1) / k) - vs;
+        for (unsigned i = tid; i < m; i += kBlock) {
+            const unsigned idx = vs + i;
+            unsigned lo = 0, hi = (unsigned)k;          // owner c: cq[c] <= idx < cq[c + 1]
+            while (hi - lo > 1) {
+                const unsigned mid = (lo + hi) >> 1;
+                if (ts.cq[mid] <= idx) lo = mid; else hi = mid;
+            }
+            const unsigned j = idx - ts.cq[lo];
+            const uint32_t *rb = cl.map_shared_rank(&ts.beg[cur][0], lo);
+            const uint16_t *rd = cl.map_shared_rank(&ts.deg[cur][0], lo);
+            ts.sbeg[i] = rb[j];
+            ts.sscan[i] = rd[j];
+        }
+        __syncthreads();
+        TEAM_STAMP(5);
+        // exclusive scan of the slice's degrees (consecutive entries per thread)
+        unsigned Em;
+        {
+            const unsigned per = (m + kBlock - 1) / kBlock, i0 = tid * per;
+            uint32_t loc = 0;
+            for (unsigned j = 0; j < per; ++j)
+                if (i0 + j < m) loc += ts.sscan[i0 + j];
+            uint32_t tot;
+            uint32_t ex = block_excl_scan(loc, ts.red, &tot);
+            for (unsigned j = 0; j < per; ++j) {
+                if (i0 + j < m) { const uint32_t d = ts.sscan[i0 + j]; ts.sscan[i0 + j] = ex; ex += d; }
+            }
+            if (tid == 0) ts.sscan[m] = tot;
+            Em = tot;
+            __syncthreads();
+        }
+        TEAM_STAMP(6);
+        if (book0) book_expand(book);
+        // (E) Expand my slice's edges: columns, then claim + the winner's offsets (as bfs_solo)
+        const int nx = cur == 2 ? 0 : cur + 1;
+        {
+            const uint32_t *scan = ts.sscan, *beg = ts.sbeg;
+            const unsigned lo = (unsigned)(((unsigned long long)Em * tid) / kBlock);
+            const unsigned hi = (unsigned)(((unsigned long long)Em * (tid + 1)) / kBlock);
+            const unsigned mine = hi > lo ? (hi - lo + kSoloK - 1) / kSoloK : 0u;
+            const unsigned nb = __reduce_max_sync(0xffffffffu, mine);
+            unsigned i = 0, j = lo;
+            if (lo < hi) {
+                unsigned L = 0, R = m;
+                while (R - L > 1) {
+                    const unsigned mid = (L + R) >> 1;
+                    if (scan[mid] <= lo) L = mid; else R = mid;
+                }
+                i = L;
+            }
+            for (unsigned bt = 0; bt < nb; ++bt) {
+                int v[kSoloK];
+#pragma unroll
+                for (int q = 0; q < kSoloK; ++q) {
+                    v[q] = -1;
+                    if (j < hi) {
+                        while (scan[i + 1] <= j) ++i;
+                        v[q] = __ldg(col + beg[i] + (j - scan[i]));
+                        ++j;
+                    }
+                }
+                unsigned old[kSoloK];
+                uint32_t vb[kSoloK], ve[kSoloK];
+#pragma unroll
+                for (int q = 0; q < kSoloK; ++q) {
+                    old[q] = v[q] >= 0 ? atomicOr(V + (v[q] >> 5), 1u << (v[q] & 31)) : 0xffffffffu;
+                    vb[q] = v[q] >= 0 ? __ldg(off + v[q]) : 0u;
+                    ve[q] = v[q] >= 0 ? __ldg(off + v[q] + 1) : 0u;
+                }
+#pragma unroll
+                for (int q = 0; q < kSoloK; ++q) {
+                    const bool won = v[q] >= 0 && !((old[q] >> (v[q] & 31)) & 1u);
+                    const unsigned mk = __ballot_sync(0xffffffffu, won);
+                    if (!mk) continue;
+                    unsigned base = 0;
+                    if (lane_id() == (unsigned)(__ffs(mk) - 1)) base = atomicAdd(&ts.qn_next, (unsigned)__popc(mk));
+                    base = __shfl_sync(0xffffffffu, base, __ffs(mk) - 1);
+                    if (won) {
+                        depth[v[q]] = t + 1;
+                        const unsigned p = base + __popc(mk & lanemask_lt());
+                        if (p < (unsigned)kTQ) { ts.q[nx][p] = v[q]; ts.beg[nx][p] = vb[q]; ts.deg[nx][p] = (uint16_t)min(ve[q] - vb[q], 65535u); }
+                        else atomicExch(&rc.ctl->err, 0x7E0u);   // impossible by the capacity check
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        TEAM_STAMP(7);
+#if GSW_TEAM_PROF
+        if (tid == 0) tp_acc[8] += 1;
+#endif
+        E_prev = Ea;
+        if (book0) prev_va = (long long)qn;
+        qn_l = ts.qn_next;
+        cur = nx;
+        par ^= 1;
+        ++t;
+        first = false;
+    }
+    // hand AS_t to the grid: my part at cq[r] of the queue; CTA 0 writes the counters and the state
+    {
+        int *gq = a.q[t & 1] + ts.cq[r];
+        for (unsigned i = tid; i < qn_l; i += kBlock) gq[i] = ts.q[cur][i];
+        if (book0) {
+            IterCnt *c = rc.cnt + (t % 3);
+            c->va = qn; c->ea = Ea; c->maxd = mxd; c->mind = mnd; c->qlen = qn; c->edges = E_prev;
+            TeamPub p{};
+            p.t = t; p.Via = Via; p.Eia = Eia;
+            *rc.pub = p;
+        }
+    }
+#if GSW_TEAM_PROF
+    if (tid == 0 && (r == 0 || r == (unsigned)k - 1))
+        for (int i = 0; i < 10; ++i) atomicAdd(&g_team_prof[r == 0 ? 0 : 1][i], tp_acc[i]);
+    if (r == 0 && tid < (unsigned)k) atomicAdd(&g_team_late[tid], tp_late);
+#endif
+    // nobody may reuse this shared memory (aliased with the grid path's) while a peer could still
+    // be reading it through DSMEM
+    cluster_barrier();
+}
+
 template <int kResident>
 __global__ void __launch_bounds__(kBlock, kResident) bfs_kernel(const __grid_constant__ BfsArgs a) {
     __shared__ BfsSmem bsm;
@@ -463,7 +819,8 @@ __global__ void __launch_bounds__(kBlock, kResident) bfs_kernel(const __grid_con
     cta_queue_reset(qs);
     const bool all_auto = rc.force.direction == GSW_AUTO && rc.force.format == GSW_AUTO &&
                           rc.force.load_balance == GSW_AUTO && rc.force.fusion == GSW_AUTO;
-    const bool solo_allowed = rc.solo_e > 0 && all_auto;
+    const int team_k = rc.team_k;
+    const bool solo_allowed = (rc.solo_e > 0 || team_k > 1) && all_auto;
     bool last_small = false;
     long long Via = (long long)n - 1, Eia = (long long)a.g.nnz - dsrc;
     int mat = MAT_SQUEUE;
@@ -500,10 +857,38 @@ __global__ void __launch_bounds__(kBlock, kResident) bfs_kernel(const __grid_con
         // CTA-resident tier: CTA 0 runs the levels alone while the frontier stays tiny
         // (entered only after two consecutive small levels: a one-level episode costs more in
         // park/wake and hand-back than it saves, measured on C1/C3)
-        const bool small = (long long)ea <= rc.solo_e && (long long)va <= rc.solo_v && va <= (unsigned long long)kSQ;
+        // (cluster launch: the team tier of cluster 0 takes the place of the solo CTA, sized by the
+        // capacity of its parts instead of the solo thresholds)
+        const unsigned long long per = (va + (unsigned)team_k - 1) / (unsigned)team_k;
+        const bool small = team_k > 1
+            ? (va > 0 && per <= (unsigned long long)kTQ && (unsigned long long)cv.maxd * per <= (unsigned long long)kTQ &&
+               (long long)ea <= rc.team_e)
+            : ((long long)ea <= rc.solo_e && (long long)va <= rc.solo_v && va <= (unsigned long long)kSQ);
         const bool solo = solo_allowed && small && last_small && c.dir == GSW_PUSH && c.fused == GSW_FUSED &&
                           (mat == MAT_QUEUE || mat == MAT_SQUEUE);
         last_small = small;
+        if (solo && team_k > 1) {
+            TeamSmem &tsm = *reinterpret_cast<TeamSmem *>(&bsm);
+            if ((int)blockIdx.x < team_k) {
+                if (is_book()) { *reinterpret_cast<Book *>(tsm.book_raw) = book; tsm.prev_va = prev_va; }
+                bfs_team(a, tsm, t, Via, Eia, f, cv.qlen, team_k);
+                if (is_book()) { book = *reinterpret_cast<const Book *>(tsm.book_raw); prev_va = tsm.prev_va; }
+                prev_dir = GSW_PUSH;
+                grid_sync(bar, epoch);
+            } else {
+                grid_park(bar, epoch);
+            }
+            TeamPub p;
+            pub_read(rc.pub, p);
+            t = (int)p.t; Via = p.Via; Eia = p.Eia;
+            mat = MAT_QUEUE;
+            if (dirty[0] || dirty[1] || dirty[2]) {
+                for (int i = 0; i < 3; ++i) if (dirty[i]) { clear_words(a.fb[i], W); dirty[i] = false; }
+                grid_sync(bar, epoch);
+            }
+            --t;
+            continue;
+        }
         if (solo) {
             if (blockIdx.x == 0) {
                 if (threadIdx.x == 0) { *reinterpret_cast<Book *>(bsm.solo.book_raw) = book; bsm.solo.prev_va = prev_va; }
@@ -694,6 +1079,8 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
                                 : (const void *)bfs_kernel<kMinBlocksBfs>;
     gsw_status s = prepare_common(g, ws, kern, a.rc, li, roadlike ? 1 : huge ? 4 : kMinBlocksBfs);
     if (s != GSW_OK) return s;
+    // road-like graphs: clustered launch, cluster 0 runs the small levels as a team
+    if (roadlike) setup_team(g, kern, a.rc, li);
     // BFS selector: hand-set rules (default) or the learned trees (GSW_SELECTOR=trees)
     if (const char *sel = std::getenv("GSW_SELECTOR")) a.rc.base.selector = std::strcmp(sel, "trees") == 0 ? 1 : 0;
     if (!a.depth || !a.V || !a.fb[2] || !a.q[1] || !a.iq || !a.scan) { set_error("workspace too small"); return GSW_ENOMEM; }
@@ -722,6 +1109,32 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
         }
         static const unsigned long long z[8][16384][2] = {};
         GSW_CUDA(cudaMemcpyToSymbol(g_pull_prof, z, sizeof(z)));
+    }
+#endif
+#if GSW_TEAM_PROF
+    {
+        unsigned long long h[2][10];
+        GSW_CUDA(cudaStreamSynchronize(g->stream));
+        GSW_CUDA(cudaMemcpyFromSymbol(h, g_team_prof, sizeof(h)));
+        static const char *nm[10] = {"loop/start", "A features", "cluster barrier", "B records", "C selector",
+                                    "D slice copy", "scan", "E expand", "-", "B first reads"};
+        unsigned long long late[16];
+        GSW_CUDA(cudaMemcpyFromSymbol(late, g_team_late, sizeof(late)));
+        if (h[0][8]) {
+            std::fprintf(stderr, "team arrival lateness per CTA (us):");
+            for (int c = 0; c < 16; ++c) std::fprintf(stderr, " %.2f", (double)late[c] * 1e-3 / (double)h[0][8]);
+            std::fprintf(stderr, "\n");
+        }
+        static const unsigned long long zl[16] = {};
+        GSW_CUDA(cudaMemcpyToSymbol(g_team_late, zl, sizeof(zl)));
+        for (int c = 0; c < 2; ++c) {
+            if (!h[c][8]) continue;
+            std::fprintf(stderr, "team prof CTA %s: %llu levels;", c ? "k-1" : "0", h[c][8]);
+            for (int i = 0; i < 10; ++i) if (i != 8) std::fprintf(stderr, " %s %.2f us", nm[i], (double)h[c][i] * 1e-3 / (double)h[c][8]);
+            std::fprintf(stderr, "\n");
+        }
+        static const unsigned long long z[2][10] = {};
+        GSW_CUDA(cudaMemcpyToSymbol(g_team_prof, z, sizeof(z)));
     }
 #endif
     if (!dev_out)

@@ -218,6 +218,12 @@ gsw_status gsw_cc(gsw_graph g, int32_t *label, gsw_run_stats *stats) {
     return run_cc(g, label, stats);
 }
 
+gsw_status gsw_cc_hook(gsw_graph g, int32_t *label, gsw_run_stats *stats) {
+    if (!g) { set_error("null graph"); return GSW_EINVAL; }
+    if (gsw_status s = no_dist(g, "gsw_cc_hook")) return s;
+    return run_cc_hook(g, label, stats);
+}
+
 gsw_status gsw_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *stats) {
     if (!g) { set_error("null graph"); return GSW_EINVAL; }
     if (g->dist) return dist_pr(g, damping, iters, rank, stats);

@@ -58,7 +58,15 @@ __device__ __forceinline__ unsigned lanemask_lt() {
 struct GridBarrier {
     unsigned *arrive;
     unsigned *err;
+    int cluster;      // nonzero: the whole grid is ONE thread-block cluster (cluster tier)
 };
+
+// Hardware cluster barrier with release/acquire at cluster scope: orders the global and shared
+// memory operations of every thread of the cluster (ptxas emits the L1 invalidation the acquire
+// needs), so when the grid is a single cluster it replaces the software grid barrier.
+__device__ __forceinline__ void cluster_barrier() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
 constexpr uint64_t kBarrierTimeoutNs = 20ull * 1000 * 1000 * 1000;
 
 // Flip-bit barrier (the cooperative-groups scheme): CTA 0 adds 2^31 - (gridDim - 1), every other
@@ -72,6 +80,7 @@ __device__ __forceinline__ unsigned ld_volatile_u32(const unsigned *p) {
     return v;
 }
 __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch) {
+    if (b.cluster) { cluster_barrier(); epoch += 1; return; }
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;
@@ -96,6 +105,7 @@ __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch)
 // same protocol as grid_sync, but the wait sleeps between polls so the parked CTAs do not steal
 // issue slots from CTA 0's SM or keep invalidating its L1 with acquire loads.
 __device__ __forceinline__ void grid_park(const GridBarrier &b, unsigned &epoch) {
+    if (b.cluster) { cluster_barrier(); epoch += 1; return; }
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;

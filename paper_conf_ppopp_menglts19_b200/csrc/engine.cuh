@@ -44,6 +44,9 @@ struct RunCommon {
     Features base;           // dataset attributes (runtime fields filled per iteration)
     struct TeamPub *pub;     // loop state handed from CTA 0 to the parked CTAs (solo tier)
     long long solo_e, solo_v;  // solo-tier thresholds on Ea / Va (0 disables the tier)
+    int cluster;             // nonzero: launched as one thread-block cluster (grid barrier = barrier.cluster)
+    int team_k;              // > 1: launched in clusters of team_k CTAs; cluster 0 runs the team tier
+    long long team_e;        // team-tier threshold on Ea (capacity is checked separately)
 };
 
 // Loop state CTA 0 hands to the parked CTAs when a solo episode ends:
@@ -65,7 +68,7 @@ __device__ __forceinline__ void pub_read(const TeamPub *g, TeamPub &out) {
 }
 
 __device__ __forceinline__ GridBarrier make_bar(const RunCommon &rc) {
-    return GridBarrier{&rc.ctl->arrive, &rc.ctl->err};
+    return GridBarrier{&rc.ctl->arrive, &rc.ctl->err, rc.cluster};
 }
 
 // Per-run bookkeeping of CTA 0 / thread 0, kept in registers so that nothing on the critical

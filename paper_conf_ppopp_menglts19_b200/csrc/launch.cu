@@ -9,6 +9,41 @@
 
 namespace gsw {
 
+static long long env_ll(const char *name, long long dflt) {
+    const char *v = std::getenv(name);
+    return (v && *v) ? std::atoll(v) : dflt;
+}
+
+// Can one k-CTA cluster of `kernel` be resident at once?  (Non-portable sizes > 8 need the opt-in
+// attribute; a GPC of B200 has 16-20 SMs.)  Cached per (kernel, k).
+bool cluster_fits(const void *kernel, int k) {
+    static std::mutex mu;
+    static std::map<std::pair<const void *, int>, bool> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto key = std::make_pair(kernel, k);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    if (k > 8 && cudaFuncSetAttribute(kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess)
+        cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(k);
+    cfg.blockDim = dim3(kBlock);
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = k;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int nc = 0;
+    if (cudaOccupancyMaxActiveClusters(&nc, kernel, &cfg) != cudaSuccess) {
+        cudaGetLastError();
+        nc = 0;
+    }
+    cache[key] = nc > 0;
+    return nc > 0;
+}
+
 static int blocks_per_sm(const void *kernel, int max_per_sm) {
     static std::mutex mu;
     static std::map<const void *, int> cache;
@@ -30,14 +65,24 @@ static int blocks_per_sm(const void *kernel, int max_per_sm) {
     return nb;
 }
 
-static long long env_ll(const char *name, long long dflt) {
-    const char *v = std::getenv(name);
-    return (v && *v) ? std::atoll(v) : dflt;
-}
 
 gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li,
                           int max_per_sm) {
     li.grid = g->sms * blocks_per_sm(kernel, max_per_sm);
+    li.cluster = 0;
+    li.team = 0;
+    rc.cluster = 0;
+    rc.team_k = 0;
+    rc.team_e = env_ll("GSW_TEAM_E", 1ll << 40);
+    // A/B knobs for the latency-bound level loops: GSW_GRID_CTAS=k runs the persistent kernel on k
+    // CTAs (software grid barrier); GSW_CLUSTER=k (2..16) launches it as ONE k-CTA thread-block
+    // cluster whose grid barrier is the hardware cluster barrier
+    if (long long k = env_ll("GSW_GRID_CTAS", 0); k > 0 && k < li.grid) li.grid = (int)k;
+    if (long long k = env_ll("GSW_CLUSTER", 0); k >= 2 && k <= 16 && cluster_fits(kernel, (int)k)) {
+        li.grid = (int)k;
+        li.cluster = (int)k;
+        rc.cluster = 1;
+    }
     static_assert(sizeof(Ctl) <= 1024, "control block fits the handle's slot");
     const bool own_ctl = g->ctl != nullptr;   // handle-owned block: zeroed at create, never reset
     rc.ctl = own_ctl ? (Ctl *)g->ctl : (Ctl *)ws.take(sizeof(Ctl));
@@ -65,7 +110,95 @@ gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCom
     return GSW_OK;
 }
 
+// Clusters of k CTAs of `kernel` that can be co-resident (cooperative launch needs them all).
+static int max_clusters(const void *kernel, int k, int sms) {
+    static std::mutex mu;
+    static std::map<std::pair<const void *, int>, int> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    auto key = std::make_pair(kernel, k);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    if (k > 8 && cudaFuncSetAttribute(kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess)
+        cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(k * (sms / k)));
+    cfg.blockDim = dim3(kBlock);
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = k;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int nc = 0;
+    if (cudaOccupancyMaxActiveClusters(&nc, kernel, &cfg) != cudaSuccess) {
+        cudaGetLastError();
+        nc = 0;
+    }
+    nc = std::min(nc, sms / k);
+    cache[key] = nc;
+    return nc;
+}
+
+bool setup_team(gsw_graph g, const void *kernel, RunCommon &rc, LaunchInfo &li) {
+    // off by default: measured slower than the grid path on C2 (profiles/r2/team_*.txt)
+    const long long want = env_ll("GSW_TEAM", 0);
+    if (li.cluster && env_ll("GSW_TEAM_IN_CLUSTER", 0)) {   // A/B: the whole (single-cluster) grid is the team
+        rc.team_k = li.cluster;
+        return true;
+    }
+    if (want < 2 || rc.cluster || li.cluster) return false;
+    for (int k : {16, 8, 4}) {
+        if (k > want) continue;
+        const int nc = max_clusters(kernel, k, g->sms);
+        // keep at least ~3/4 of the SMs for the grid-wide levels
+        if (nc * k * 4 < g->sms * 3) continue;
+        li.grid = nc * k;
+        li.team = k;
+        rc.team_k = k;
+        return true;
+    }
+    return false;
+}
+
 gsw_status launch_persistent(gsw_graph g, const void *kernel, void **args, const LaunchInfo &li) {
+    if (li.team > 0) {
+        if (li.team > 8) GSW_CUDA(cudaFuncSetAttribute(kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(li.grid);
+        cfg.blockDim = dim3(kBlock);
+        cfg.stream = g->stream;
+        cudaLaunchAttribute at[2];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = li.team;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        at[1].id = cudaLaunchAttributeCooperative;
+        at[1].val.cooperative = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 2;
+        GSW_CUDA(cudaLaunchKernelExC(&cfg, kernel, args));
+        GSW_CUDA(cudaEventRecord(g->ev1, g->stream));
+        return GSW_OK;
+    }
+    if (li.cluster > 0) {
+        // one cluster: its CTAs are co-scheduled by construction (no cooperative attribute needed)
+        if (li.cluster > 8) GSW_CUDA(cudaFuncSetAttribute(kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(li.grid);
+        cfg.blockDim = dim3(kBlock);
+        cfg.stream = g->stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = li.cluster;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        GSW_CUDA(cudaLaunchKernelExC(&cfg, kernel, args));
+        GSW_CUDA(cudaEventRecord(g->ev1, g->stream));
+        return GSW_OK;
+    }
     GSW_CUDA(cudaLaunchCooperativeKernel(kernel, dim3(li.grid), dim3(kBlock), args, 0, g->stream));
     GSW_CUDA(cudaEventRecord(g->ev1, g->stream));
     return GSW_OK;

@@ -9,6 +9,8 @@ namespace gsw {
 
 struct LaunchInfo {
     int grid = 0;
+    int cluster = 0;   // > 0: the grid is one thread-block cluster of this many CTAs (no cooperative launch)
+    int team = 0;      // > 0: cooperative launch in clusters of this many CTAs (team tier)
 };
 
 // Blocks per SM of every persistent kernel (kernels declare __launch_bounds__(kBlock, kMinBlocks)).
@@ -29,6 +31,10 @@ constexpr int kMinBlocksBfs = 2, kMinBlocksSssp = 2, kMinBlocksCc = 4, kMinBlock
 
 gsw_status prepare_common(gsw_graph g, Workspace &ws, const void *kernel, RunCommon &rc, LaunchInfo &li,
                           int max_per_sm);
+// Team tier: pick the cluster size (16, else 8) for a cooperative clustered launch of `kernel` at
+// one CTA per SM and set li.grid / li.team / rc.team_k; no-op (returns false) when clusters do not
+// fit or GSW_TEAM=0.
+bool setup_team(gsw_graph g, const void *kernel, RunCommon &rc, LaunchInfo &li);
 gsw_status launch_persistent(gsw_graph g, const void *kernel, void **args, const LaunchInfo &li);
 gsw_status finish_run(gsw_graph g, const RunCommon &rc, const LaunchInfo &li, gsw_run_stats *st);
 
@@ -36,6 +42,7 @@ gsw_status finish_run(gsw_graph g, const RunCommon &rc, const LaunchInfo &li, gs
 gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth, gsw_run_stats *st);
 gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *st);
 gsw_status run_cc(gsw_graph g, int32_t *label, gsw_run_stats *st);
+gsw_status run_cc_hook(gsw_graph g, int32_t *label, gsw_run_stats *st);
 gsw_status run_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st);
 gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, double *rank, gsw_run_stats *st);
 gsw_status run_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc, gsw_run_stats *st);
