@@ -31,6 +31,8 @@ sys.path.insert(0, ROOT)
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_HBM = 6650.0   # GB/s, B200_PROFILING.md fallback
+# random 4-byte L2 gathers per second (G/s), measured by tools/micro_gather.cu (profiles/r2/micro_gather.txt)
+PR_GATHER_PEAK = 356.0
 
 
 def hbm_peak():
@@ -226,6 +228,18 @@ def run_extras(gsw, dev, G3, g3, peak, cpu=True):
         out["C3_pr"]["cpu_baseline"] = {"value": 2 / secs, "unit": "PR iters/s", "cores": oracle.threads(),
                                         "kind": "oracle", "sample": f"2 fp64 iterations, per-vertex loop over "
                                                                     f"{oracle.threads()} OpenMP threads, {secs:.2f} s"}
+    # PR's Expand is bound by random 4-byte gathers of L2-resident contributions, not by HBM:
+    # its ceiling is the measured gather rate of tools/micro_gather.cu
+    gps = g3.nnz * 20 / (st["gpu_ms"] * 1e-3) / 1e9
+    out["C3_pr"]["gather_roofline"] = {
+        "bound": "l2_gather", "achieved": gps, "peak": PR_GATHER_PEAK, "unit": "G gathers/s",
+        "frac": gps / PR_GATHER_PEAK,
+        "peak_source": "tools/micro_gather.cu on B200: 128M streamed power-law indices gathering 4-byte "
+                       "values of a 16.8 MB array with a 28,672-entry shared-memory hub cache "
+                       "(profiles/r2/micro_gather.txt; uniform indices without cache: 265)"}
+    # hooking + pointer-jumping CC (gsw_cc_hook, Soman et al.) beside the GSWITCH CC
+    st = best(lambda: G3.cc_hook())
+    out["C3_cc_hook"] = rec(g3.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
     # Delta-PR (DESIGN R16): tol = 1e-6 in L1; GTEPS over the edges its Expand read
     st = best(lambda: G3.dpr(0.85, 1e-6))
     out["C3_dpr"] = rec(st["edges_touched"] / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS (edges read)", st)
@@ -239,7 +253,13 @@ def run_extras(gsw, dev, G3, g3, peak, cpu=True):
         out["C2_sssp"]["cpu_baseline"] = {"value": g2.nnz / 2 / secs / 1e9, "unit": "GTEPS", "cores": 1,
                                           "kind": "oracle", "sample": f"binary-heap Dijkstra from vertex 0, {secs:.2f} s "
                                                                       "(no parallel CPU variant: Dijkstra is serial)"}
-    del G2, g2
+    # CC on the road grid: label propagation needs ~4,000 iterations (the grid's diameter), hooking 2
+    G2u = gsw.Graph(g2.off, g2.col, device=dev)
+    st = best(lambda: G2u.cc())
+    out["C2_cc"] = rec(g2.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
+    st = best(lambda: G2u.cc_hook())
+    out["C2_cc_hook"] = rec(g2.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)
+    del G2, G2u, g2
     g4 = gen.config_graph("C4")
     G4 = gsw.Graph(g4.off, g4.col, device=dev)
     srcs = gen.sources(g4, 16)
