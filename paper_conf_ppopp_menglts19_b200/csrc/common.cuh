@@ -80,7 +80,9 @@ __device__ __forceinline__ unsigned ld_volatile_u32(const unsigned *p) {
     return v;
 }
 __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch) {
+#ifndef GSW_NO_CLUSTER_BAR
     if (b.cluster) { cluster_barrier(); epoch += 1; return; }
+#endif
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;
@@ -105,7 +107,9 @@ __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch)
 // same protocol as grid_sync, but the wait sleeps between polls so the parked CTAs do not steal
 // issue slots from CTA 0's SM or keep invalidating its L1 with acquire loads.
 __device__ __forceinline__ void grid_park(const GridBarrier &b, unsigned &epoch) {
+#ifndef GSW_NO_CLUSTER_BAR
     if (b.cluster) { cluster_barrier(); epoch += 1; return; }
+#endif
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;

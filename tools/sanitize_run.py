@@ -69,6 +69,29 @@ def main():
     G = gsw.Graph(g.off, g.col)
     chk("bfs solo overflow", G.bfs(s)[0].cpu().numpy(), oracle.bfs(g, s))
     del os.environ["GSW_SOLO_E"]
+    # hooking + pointer-jumping CC under every sweep mapping (round 2, session 3)
+    G = gsw.Graph(g.off, g.col)
+    for lb in ("auto", "thread", "twc", "wm", "cm", "strict"):
+        if lb == "auto":
+            G.force_config()
+        else:
+            G.force_config(load_balance=lb)
+        chk(f"cc_hook {lb}", G.cc_hook()[0].cpu().numpy(), oracle.cc(g))
+    G.force_config()
+    Gg = gsw.Graph(grid.off, grid.col, grid.w)
+    chk("cc_hook grid", Gg.cc_hook()[0].cpu().numpy(), oracle.cc(grid))
+    # cluster launches: the BFS team tier (DSMEM frontier parts) and the single-cluster grid
+    for env in ({"GSW_TEAM": "16"}, {"GSW_TEAM": "4"}, {"GSW_CLUSTER": "8"}):
+        os.environ.update(env)
+        tag = ",".join(f"{k}={v}" for k, v in env.items())
+        chk(f"bfs grid [{tag}]", Gg.bfs(0)[0].cpu().numpy(), oracle.bfs(grid, 0))
+        chk(f"bfs rmat [{tag}]", G.bfs(s)[0].cpu().numpy(), oracle.bfs(g, s))
+        for k in env:
+            del os.environ[k]
+    os.environ.update({"GSW_CLUSTER": "8"})
+    chk("sssp grid [GSW_CLUSTER=8]", Gg.sssp(0)[0].cpu().numpy().view(np.uint32), oracle.sssp(grid, 0))
+    del os.environ["GSW_CLUSTER"]
+    del G, Gg
     P = gsw.PartitionedGraph(g.off, g.col, 3)
     chk("partitioned bfs p=3", P.bfs(s)[0].cpu().numpy(), oracle.bfs(g, s))
     chk("partitioned pr p=3", P.pr(0.85, 20)[0].cpu().numpy().astype(np.float64), oracle.pr(g, 0.85, 20), (1e-5, 0.0))
