@@ -117,7 +117,7 @@ struct DCtl {
     double dtot;                   // all-reduced f64 (PR dangling mass)
     double pad0;
     long long Via, Eia, nnz_g;     // unvisited vertices / their edges, global nnz
-    int dir, done, t, pad1;
+    int dir, done, t, cur;         // cur: the level the next expand runs (graph mode reads it)
     unsigned long long theta, delta;   // SSSP priority threshold and its step (P4)
 };
 
@@ -170,6 +170,12 @@ struct DistState {
     int *hdone_dev = nullptr;               // their device alias (written by k_publish_done)
     int lookahead = 1;                      // GSW_DIST_LOOKAHEAD (1..4); 1 measured best (profiles/r2/part_ab.txt)
     cudaEvent_t evs[kLookaheadMax + 1] = {};
+    // graph mode (NCCL / loopback): the whole level loop is one CUDA graph with a device-side WHILE
+    // node; instantiated once and re-launched while the output buffer and forced direction match
+    cudaGraphExec_t bfs_exec = nullptr;
+    const void *bfs_exec_depth = nullptr;
+    int bfs_exec_dir = -1;
+    cudaStream_t cap = nullptr;             // private stream the graph is captured on (the caller's may be the legacy stream)
 };
 
 int64_t dist_slice(int64_t n, int32_t p) {
@@ -196,6 +202,35 @@ __global__ void k_rebase_offsets_u32(const uint32_t *in, uint32_t base, uint32_t
 }
 __global__ void k_first(const uint32_t *roff, const int32_t *rcol, int nloc, int32_t *first) {
     for (long long v = gtid(); v < nloc; v += gthreads()) first[v] = roff[v + 1] > roff[v] ? rcol[roff[v]] : -1;
+}
+// Hub first (create time): every owned row moves its highest-degree neighbour to the front, so
+// the pull's first probe (k_first) meets the likeliest frontier member, as the single-GPU engine's
+// degree-ordered relabeling does (C3 p=1: the widest pull level scanned 5.3M edges
+// vs 2.8M).  deg: the replicated degree array (all-gathered).  A row's order is irrelevant to
+// every other kernel (weights move with their columns).
+__global__ void k_degrees(const uint32_t *roff, int nloc, int64_t S, uint32_t *deg_slice) {
+    for (long long v = gtid(); v < S; v += gthreads()) deg_slice[v] = v < nloc ? roff[v + 1] - roff[v] : 0u;
+}
+__global__ void k_hub_first(const uint32_t *roff, int32_t *rcol, uint32_t *rw, int nloc, const uint32_t *deg) {
+    for (long long v = gwarp(); v < nloc; v += gwarps()) {
+        const uint32_t b = roff[v], e = roff[v + 1];
+        unsigned best = 0u;
+        uint32_t at = b;
+        for (uint32_t k = b + lane_id(); k < e; k += 32) {
+            const unsigned dk = deg[rcol[k]];
+            if (dk > best || (dk == best && k < at)) { best = dk; at = k; }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const unsigned ob = __shfl_xor_sync(0xffffffffu, best, o);
+            const uint32_t oa = __shfl_xor_sync(0xffffffffu, at, o);
+            if (ob > best || (ob == best && oa < at)) { best = ob; at = oa; }
+        }
+        if (lane_id() == 0 && e > b && at != b) {
+            const int32_t c = rcol[b]; rcol[b] = rcol[at]; rcol[at] = c;
+            if (rw) { const uint32_t w = rw[b]; rw[b] = rw[at]; rw[at] = w; }
+        }
+    }
 }
 // column slice "global source -> owned targets": count, scan, fill
 __global__ void k_slice_count(const uint32_t *roff, const int32_t *rcol, int nloc, uint32_t *cnt) {
@@ -281,20 +316,20 @@ struct BfsP {
     uint32_t task_cap;
     unsigned long long *loc;
     const DCtl *ctl;
-    int lvl;
+    int lvl;                  // < 0: graph mode, the level is ctl->cur
 };
+__device__ __forceinline__ int bfs_lvl(const BfsP &a) { return a.lvl >= 0 ? a.lvl : a.ctl->cur; }
 
 __global__ void k_bfs_init(BfsP a, int64_t src, unsigned *fb0) {
     const int W = (a.nloc + 31) >> 5;
     for (long long v = gtid(); v < a.nloc; v += gthreads()) a.depth[v] = (a.vb + v == src) ? 0 : -1;
-    for (long long w = gtid(); w < W; w += gthreads()) {
-        unsigned m = 0;
-        for (int b = 0; b < 32; ++b) {
-            const long long v = w * 32 + b;
-            const bool done = v >= a.nloc || a.roff[v + 1] == a.roff[v] || a.vb + v == src;   // padding, isolated, source
-            m |= (done ? 1u : 0u) << b;
-        }
-        a.vis[w] = m;
+    // visited words: a warp per word, a lane per vertex (coalesced offsets, one ballot); the
+    // serial 32-vertex loop per thread this replaces cost 56 us at C3
+    for (long long w = gwarp(); w < W; w += gwarps()) {
+        const long long v = w * 32 + lane_id();
+        const bool done = v >= a.nloc || a.roff[v + 1] == a.roff[v] || a.vb + v == src;   // padding, isolated, source
+        const unsigned m = __ballot_sync(0xffffffffu, done);
+        if (lane_id() == 0) a.vis[w] = m;
     }
     if (gtid() == 0 && src >= a.vb && src < a.vb + a.nloc) {
         const int v = (int)(src - a.vb);
@@ -304,20 +339,33 @@ __global__ void k_bfs_init(BfsP a, int64_t src, unsigned *fb0) {
     }
 }
 
-// claim local target v for level lvl+1 (push): returns 1 if this call won it
-__device__ __forceinline__ bool push_claim(const BfsP &a, int v, unsigned long long &va, unsigned long long &ea) {
-    const unsigned bit = 1u << (v & 31);
-    if (a.vis[v >> 5] & bit) return false;
-    if (atomicOr(a.vis + (v >> 5), bit) & bit) return false;
-    a.depth[v] = a.lvl + 1;
-    atomicOr(a.nfb + ((a.vb + v) >> 5), bit);      // vb is a multiple of 64
-    va++;
-    ea += a.roff[v + 1] - a.roff[v];
-    return true;
+// claim up to 4 local targets (v < 0: none) with their round trips overlapped: visited words,
+// then the atomics of the unvisited ones, then the winners' stores and degree loads
+__device__ __forceinline__ void push_claim4(const BfsP &a, const int (&v)[4], unsigned long long &va,
+                                           unsigned long long &ea, unsigned long long &ed) {
+    unsigned w[4], old[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) w[k] = v[k] >= 0 ? a.vis[v[k] >> 5] : ~0u;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const unsigned bit = v[k] >= 0 ? 1u << (v[k] & 31) : 0u;
+        old[k] = (v[k] >= 0 && !(w[k] & bit)) ? atomicOr(a.vis + (v[k] >> 5), bit) : ~0u;
+        ed += v[k] >= 0 ? 1ull : 0ull;
+    }
+    const int lvl1 = bfs_lvl(a) + 1;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        if (v[k] < 0 || (old[k] >> (v[k] & 31)) & 1u) continue;
+        a.depth[v[k]] = lvl1;
+        atomicOr(a.nfb + ((a.vb + v[k]) >> 5), 1u << (v[k] & 31));      // vb is a multiple of 64
+        va++;
+        ea += a.roff[v[k] + 1] - a.roff[v[k]];
+    }
 }
 
 // push, light part: a lane per frontier vertex of the warp's bitmap word (rows <= 32 edges, 4
-// columns in flight), the whole warp for rows of 33..kHeavy edges, tasks for longer rows
+// columns in flight), the whole warp for rows of 33..kHeavy edges (4 edges per lane in flight),
+// CTA-wide tasks for longer rows (k_bfs_push_heavy)
 __device__ __noinline__ void bfs_push_body(const BfsP &a) {
     const long long FW = a.npad >> 5;
     const unsigned lane = lane_id();
@@ -341,8 +389,7 @@ __device__ __noinline__ void bfs_push_body(const BfsP &a) {
                 int v[4];
 #pragma unroll
                 for (int k = 0; k < 4; ++k) v[k] = e + k < s1 ? __ldg(a.scol + e + k) : -1;
-#pragma unroll
-                for (int k = 0; k < 4; ++k) if (v[k] >= 0) { ed++; push_claim(a, v[k], va, ea); }
+                push_claim4(a, v, va, ea, ed);
             }
         }
         unsigned mid = __ballot_sync(0xffffffffu, mine && L > 32 && L <= kHeavy);
@@ -350,19 +397,34 @@ __device__ __noinline__ void bfs_push_body(const BfsP &a) {
             const int j = __ffs(mid) - 1;
             mid &= mid - 1;
             const uint32_t b = __shfl_sync(0xffffffffu, s0, j), e = __shfl_sync(0xffffffffu, s1, j);
-            for (uint32_t k = b + lane; k < e; k += 32) { ed++; push_claim(a, __ldg(a.scol + k), va, ea); }
+            for (uint32_t k = b + lane; k < e; k += 128) {
+                int v[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) v[q] = k + 32 * q < e ? __ldg(a.scol + k + 32 * q) : -1;
+                push_claim4(a, v, va, ea, ed);
+            }
         }
     }
     flush_loc(va, ea, ed, 0.0, a.loc);
 }
 
+// heavy rows: a CTA per kHeavy-edge task, 4 edges per thread with their round trips overlapped
+// (a warp per task walked 32 dependent claim chains: C3's first push level took 80 us here)
 __global__ void __launch_bounds__(kDB) k_bfs_push_heavy(BfsP a) {
     if (a.ctl->done || a.ctl->dir != GSW_PUSH) return;
+    a.lvl = bfs_lvl(a);
     const unsigned nt = min(*a.ntasks, a.task_cap);
     unsigned long long va = 0, ea = 0, ed = 0;
-    for (long long k = gwarp(); k < nt; k += gwarps()) {
+    static_assert(kHeavy <= 4 * kDB, "a task fits one pass of the CTA");
+    for (unsigned k = blockIdx.x; k < nt; k += gridDim.x) {
         const DTask tk = a.tasks[k];
-        for (uint32_t e = tk.beg + lane_id(); e < tk.end; e += 32) { ed++; push_claim(a, __ldg(a.scol + e), va, ea); }
+        int v[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const uint32_t e = tk.beg + threadIdx.x + q * kDB;
+            v[q] = e < tk.end ? __ldg(a.scol + e) : -1;
+        }
+        push_claim4(a, v, va, ea, ed);
     }
     flush_loc(va, ea, ed, 0.0, a.loc);
 }
@@ -371,6 +433,7 @@ __global__ void __launch_bounds__(kDB) k_bfs_push_heavy(BfsP a) {
 // push or the pull body; heavy push rows are finished by k_bfs_push_heavy
 __global__ void __launch_bounds__(kDB) k_bfs_level(BfsP a) {
     if (a.ctl->done) return;
+    a.lvl = bfs_lvl(a);
     if (a.ctl->dir == GSW_PUSH) {
         bfs_push_body(a);
         return;
@@ -384,16 +447,26 @@ __global__ void __launch_bounds__(kDB) k_bfs_level(BfsP a) {
 // account level t (its expand and exchange finished, tot = counts of AS_{t+1}) and decide t+1
 // (block 0 / thread 0); every thread also clears the bitmap level t+1 will write (FB_t, read by
 // level t) and thread 0 the parts' push-task counters, so a level needs no separate memsets
+// Graph mode: t = -2 reads the level from ctl->cur, and the WHILE node's condition is set to
+// "not done" (cudaGraphSetConditional) so the device decides whether the loop body runs again.
 __global__ void k_bfs_decide(DCtl *ctl, DRec *recs, unsigned long long *locs, int parts, int t, long long n,
-                             int force_dir, unsigned *clear, long long clear_words, unsigned *ntasks) {
+                             int force_dir, unsigned *clear, long long clear_words, unsigned *ntasks,
+                             cudaGraphConditionalHandle cond, int use_cond) {
     for (long long w = gtid(); w < clear_words; w += gthreads()) clear[w] = 0u;
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    if (t == -2) t = ctl->cur;
+    ctl->cur = t + 1;
     for (int p = 0; p < parts; ++p) ntasks[p * 32] = 0u;
     const unsigned long long va = ctl->tot[0], ea = ctl->tot[1], ed = ctl->tot[2];
     for (int i = 0; i < parts * kLocStride; ++i) locs[i] = 0ull;
-    if (ctl->done) return;
+    if (ctl->done) { if (use_cond) cudaGraphSetConditional(cond, 0u); return; }
     if (t >= 0 && t < kMaxLevels) recs[t].edges = (long long)ed;
-    if (va == 0) { ctl->done = 1; return; }
+    if (va == 0) {
+        ctl->done = 1;
+        if (use_cond) cudaGraphSetConditional(cond, 0u);
+        return;
+    }
+    if (use_cond) cudaGraphSetConditional(cond, 1u);
     ctl->Via -= (long long)va;
     ctl->Eia -= (long long)ea;
     // the single-GPU direction split (select.cuh, R6) on the GLOBAL features
@@ -1156,6 +1229,20 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
         task_cur += chunk_cap(P.nnz);
         d->parts.push_back(P);
     }
+    // hub first: all-gather the degrees into rep[0], reorder every owned row, redo the first-neighbour table
+    if (!(std::getenv("GSW_DIST_HUBFIRST") && *std::getenv("GSW_DIST_HUBFIRST") == '0')) {
+        for (auto &P : d->parts)
+            k_degrees<<<grid_for(S, g->sms), kDB, 0, s>>>(P.roff, P.nloc, S, d->rep[0] + P.vb);
+        if (cudaGetLastError() != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "degrees"));
+        if (gsw_status st = ex_allgather(d, d->rep[0], (size_t)S * 4, s)) return fail(st);
+        for (auto &P : d->parts) {
+            if (!P.nloc) continue;
+            k_hub_first<<<grid_for((long long)P.nloc * 32, g->sms), kDB, 0, s>>>(P.roff, const_cast<int32_t *>(P.rcol),
+                                                                               const_cast<uint32_t *>(P.rw), P.nloc, d->rep[0]);
+            k_first<<<grid_for(P.nloc, g->sms), kDB, 0, s>>>(P.roff, P.rcol, P.nloc, P.rfirst);
+        }
+        if (cudaGetLastError() != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "hub first"));
+    }
     g->scratch = (char *)ws.take((size_t)d->npad * 8);      // output staging (host outputs)
     g->scratch_bytes = (size_t)d->npad * 8;
     if (!g->scratch) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
@@ -1186,6 +1273,8 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
 
 void dist_destroy(DistState *d) {
     if (!d) return;
+    if (d->bfs_exec) cudaGraphExecDestroy(d->bfs_exec);
+    if (d->cap) cudaStreamDestroy(d->cap);
     if (d->comm && g_nccl.ok) g_nccl.commDestroy(d->comm);
     for (auto &ev : d->evs) if (ev) cudaEventDestroy(ev);
     if (d->hdone) cudaFreeHost(d->hdone);
@@ -1265,10 +1354,70 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
     if (gsw_status e = ex_reduce(d, s)) return e;
     const int grid = g->sms * 8;
     const long long FBW = d->npad / 32;
-    k_bfs_decide<<<g->sms, kDB, 0, s>>>(d->ctl, d->recs, d->locs, parts, -1, d->n, fdir, d->FB[1], FBW, d->ntasks);
+    k_bfs_decide<<<g->sms, kDB, 0, s>>>(d->ctl, d->recs, d->locs, parts, -1, d->n, fdir, d->FB[1], FBW, d->ntasks,
+                                        cudaGraphConditionalHandle{}, 0);
     GSW_CUDA(cudaGetLastError());
+    // graph mode: the level loop as one CUDA graph whose WHILE node the decide kernel drives, so
+    // the host neither polls nor enqueues per level (NCCL / loopback; GSW_DIST_GRAPH=0 disables)
+    const char *gm = std::getenv("GSW_DIST_GRAPH");
+    const bool graph_mode = d->mode != DM_HOST && !(gm && *gm == '0');
+    if (graph_mode) {
+        if (!d->bfs_exec || d->bfs_exec_depth != (const void *)depth || d->bfs_exec_dir != fdir) {
+            if (d->bfs_exec) { cudaGraphExecDestroy(d->bfs_exec); d->bfs_exec = nullptr; }
+            cudaGraph_t gr = nullptr;
+            GSW_CUDA(cudaGraphCreate(&gr, 0));
+            cudaGraphConditionalHandle cond;
+            GSW_CUDA(cudaGraphConditionalHandleCreate(&cond, gr, 1u, cudaGraphCondAssignDefault));
+            cudaGraphNodeParams cp = {};
+            cp.type = cudaGraphNodeTypeConditional;
+            cp.conditional.handle = cond;
+            cp.conditional.type = cudaGraphCondTypeWhile;
+            cp.conditional.size = 1;
+            cudaGraphNode_t node;
+            GSW_CUDA(cudaGraphAddNode(&node, gr, nullptr, 0, &cp));
+            cudaGraph_t body = cp.conditional.phGraph_out[0];
+            if (!d->cap) GSW_CUDA(cudaStreamCreateWithFlags(&d->cap, cudaStreamNonBlocking));
+            const cudaStream_t run = s;
+            s = d->cap;                                   // the enqueues below are captured, not run
+            GSW_CUDA(cudaStreamBeginCaptureToGraph(s, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+            gsw_status cs = GSW_OK;
+            for (int par = 0; par < 2 && cs == GSW_OK; ++par) {      // two levels per body: fixed FB parity
+                unsigned *fb = d->FB[par], *nfb = d->FB[par ^ 1];
+                for (int p = 0; p < parts; ++p) {
+                    BfsP a = pa[p];
+                    a.fb = fb; a.nfb = nfb; a.lvl = -1;
+                    if (!a.nloc) continue;
+                    k_bfs_level<<<grid, kDB, 0, s>>>(a);
+                    k_bfs_push_heavy<<<g->sms * 2, kDB, 0, s>>>(a);
+                }
+                if (cudaGetLastError() != cudaSuccess) { cs = GSW_ECUDA; break; }
+                if ((cs = ex_allgather(d, nfb, (size_t)d->S / 8, s)) != GSW_OK) break;
+                if ((cs = ex_reduce(d, s)) != GSW_OK) break;
+                k_bfs_decide<<<g->sms, kDB, 0, s>>>(d->ctl, d->recs, d->locs, parts, -2, d->n, fdir, fb, FBW, d->ntasks,
+                                                    cond, 1);
+            }
+            cudaGraph_t cap = nullptr;
+            const cudaError_t ce = cudaStreamEndCapture(s, &cap);
+            s = run;
+            if (cs != GSW_OK || ce != cudaSuccess) {
+                cudaGraphDestroy(gr);
+                if (cs == GSW_OK) { set_error(std::string("dist bfs graph capture: ") + cudaGetErrorString(ce)); cs = GSW_ECUDA; }
+                return cs;
+            }
+            const cudaError_t ie = cudaGraphInstantiate(&d->bfs_exec, gr, 0);
+            cudaGraphDestroy(gr);
+            if (ie != cudaSuccess) {
+                d->bfs_exec = nullptr;
+                set_error(std::string("dist bfs graph instantiate: ") + cudaGetErrorString(ie));
+                return GSW_ECUDA;
+            }
+            d->bfs_exec_depth = depth;
+            d->bfs_exec_dir = fdir;
+        }
+        GSW_CUDA(cudaGraphLaunch(d->bfs_exec, s));
+    }
     int t = 0;
-    for (;; ++t) {
+    for (; !graph_mode; ++t) {
         unsigned *fb = d->FB[t & 1], *nfb = d->FB[(t + 1) & 1];
         for (int p = 0; p < parts; ++p) {
             BfsP a = pa[p];
@@ -1280,7 +1429,8 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
         GSW_CUDA(cudaGetLastError());
         if (gsw_status e = ex_allgather(d, nfb, (size_t)d->S / 8, s)) return e;
         if (gsw_status e = ex_reduce(d, s)) return e;
-        k_bfs_decide<<<g->sms, kDB, 0, s>>>(d->ctl, d->recs, d->locs, parts, t, d->n, fdir, fb, FBW, d->ntasks);
+        k_bfs_decide<<<g->sms, kDB, 0, s>>>(d->ctl, d->recs, d->locs, parts, t, d->n, fdir, fb, FBW, d->ntasks,
+                                            cudaGraphConditionalHandle{}, 0);
         GSW_CUDA(cudaGetLastError());
         bool stop = false;
         if (gsw_status e = poll_done(d, t, s, &stop)) return e;
