@@ -20,6 +20,15 @@
 
 namespace gsw {
 
+// Resident CTAs per SM (A/B knob).  With 24-byte tokens (two packed 64-bit pointers + the
+// pre-check value per edge in flight) the sweep spilled and the spill stores reached DRAM (ncu:
+// 11 GB written in an 8.5 ms C3 run, profiles/r2/ncu_cc_hook_c3.md); with the 16-byte token below,
+// 4 CTAs/SM measured best (C3 7.65 ms vs 10.4 at 2/SM; C4 9.0 vs 12.5; profiles/r2/cc_hook_minb_ab.txt)
+#ifndef GSW_HOOK_MINB
+#define GSW_HOOK_MINB 4
+#endif
+constexpr int kMinBlocksCcHook = GSW_HOOK_MINB;
+
 #ifndef GSW_HOOK_PRECHECK
 #define GSW_HOOK_PRECHECK 1     // read the larger root's pointer before the atomic (A/B knob)
 #endif
@@ -42,8 +51,10 @@ __device__ __forceinline__ unsigned long long hk_pack(const uint32_t *perm, unsi
 // (another edge may already have hooked it below something at least as small -- then the atomic
 // is skipped, which removes most of the contended atomics on hub roots in the first sweep); aux
 // issues the hook.
+// keys are unique (caller ids), so comparing packed pointers is comparing their keys: the token
+// keeps 32-bit halves (16 bytes per edge in flight instead of 24)
 struct HookTok {
-    unsigned long long lo, hi, cur;
+    unsigned lo_key, lo_id, hi_id, cur_key;
 };
 struct HookOp {
     unsigned long long *P;
@@ -58,17 +69,19 @@ struct HookOp {
         return make_ulonglong2(P[x], P[y]);
     }
     __device__ __forceinline__ Tok act(int, uint32_t, int, Probe p) const {
-        if (p.x == p.y) return HookTok{0ull, 0ull, 0ull};
+        if (p.x == p.y) return HookTok{0u, 0u, 0u, 0u};
         const unsigned long long lo = p.x < p.y ? p.x : p.y, hi = p.x < p.y ? p.y : p.x;
 #if GSW_HOOK_PRECHECK
-        return HookTok{lo, hi, P[(unsigned)hi]};
+        const unsigned ck = (unsigned)(P[(unsigned)hi] >> 32);
 #else
-        return HookTok{lo, hi, ~0ull};
+        const unsigned ck = 0xffffffffu;
 #endif
+        return HookTok{(unsigned)(lo >> 32), (unsigned)lo, (unsigned)hi, ck};
     }
     __device__ __forceinline__ Aux aux(int, uint32_t, int, Tok t) const {
-        if (t.cur <= t.lo) return 0u;                                  // equal roots, or already lower
-        return atomicMin(P + (unsigned)t.hi, t.lo) > t.lo ? 1u : 0u;
+        if (t.cur_key <= t.lo_key) return 0u;                          // equal roots, or already lower
+        const unsigned long long lo = ((unsigned long long)t.lo_key << 32) | t.lo_id;
+        return atomicMin(P + t.hi_id, lo) > lo ? 1u : 0u;
     }
     __device__ __forceinline__ bool commit(int, uint32_t, int, Tok, Aux h, LocalCnt &c) const {
         c.aux += h;
@@ -76,7 +89,7 @@ struct HookOp {
     }
 };
 
-__global__ void __launch_bounds__(kBlock, kMinBlocksCc) cc_hook_kernel(const __grid_constant__ CcHookArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocksCcHook) cc_hook_kernel(const __grid_constant__ CcHookArgs a) {
     __shared__ LbSmem sm;
     __shared__ uint32_t red[kWarps + 1];
     const RunCommon &rc = a.rc;
@@ -163,7 +176,7 @@ gsw_status run_cc_hook(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     a.out = dev_out ? label_out : (int *)ws.take((size_t)n * 4);
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);
     LaunchInfo li;
-    gsw_status s = prepare_common(g, ws, (const void *)cc_hook_kernel, a.rc, li, kMinBlocksCc);
+    gsw_status s = prepare_common(g, ws, (const void *)cc_hook_kernel, a.rc, li, kMinBlocksCcHook);
     if (s != GSW_OK) return s;
     if (!a.P || !a.out || !a.scan) { set_error("workspace too small"); return GSW_ENOMEM; }
     void *args[] = {&a};

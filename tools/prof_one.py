@@ -17,4 +17,5 @@ for _ in range(2):
     elif algo == "sssp": G.sssp(0)
     elif algo == "bc": G.bc(gen.sources(g, 2))
     elif algo == "dpr": G.dpr(0.85, 1e-6)
+    elif algo == "cc_hook": G.cc_hook()
 print("done")
