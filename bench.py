@@ -253,7 +253,8 @@ def run_extras(gsw, dev, G3, g3, peak, cpu=True):
         out["C2_sssp"]["cpu_baseline"] = {"value": g2.nnz / 2 / secs / 1e9, "unit": "GTEPS", "cores": 1,
                                           "kind": "oracle", "sample": f"binary-heap Dijkstra from vertex 0, {secs:.2f} s "
                                                                       "(no parallel CPU variant: Dijkstra is serial)"}
-    # CC on the road grid: label propagation needs ~4,000 iterations (the grid's diameter), hooking 2
+    # CC on the road grid: label propagation would need ~4,000 iterations (the grid's diameter); the
+    # autotuned gsw_cc hands over to hooking after 12, gsw_cc_hook alone needs 2 sweeps
     G2u = gsw.Graph(g2.off, g2.col, device=dev)
     st = best(lambda: G2u.cc())
     out["C2_cc"] = rec(g2.nnz / 2 / (st["gpu_ms"] * 1e-3) / 1e9, "GTEPS", st)

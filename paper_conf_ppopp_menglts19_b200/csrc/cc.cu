@@ -6,6 +6,9 @@
 // label[v] = min vertex id of v's component.  Terminates when no label changed.
 //   Filter: fused  -> Expand marks changed vertices in the next active-set bitmap
 //           standalone -> a Filter pass compares label with its value at the iteration start
+#include <algorithm>
+#include <cstdlib>
+
 #include "engine.cuh"
 #include "internal.h"
 #include "launch.h"
@@ -13,6 +16,8 @@
 #include "lb_reduce.cuh"
 
 namespace gsw {
+
+constexpr int kCcSwitchIters = 12;   // label-propagation iterations before the switch to hooking (C1-C4 converge in <= 6)
 
 struct CcArgs {
     DevGraph g;
@@ -25,6 +30,8 @@ struct CcArgs {
     uint32_t *scan;
     long long iso_count;
     unsigned *heavy, *hblk, *heavy_cnt;   // tiered pull (lb_reduce.cuh lbr_tiered)
+    int max_iters;        // > 0: stop after this many iterations and raise *unfinished (run_cc's switch)
+    unsigned *unfinished;
     RunCommon rc;
 };
 
@@ -157,6 +164,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksCc) cc_kernel(CcArgs a) {
         rc.cnt[0].ea = a.g.nnz;
         rc.cnt[0].maxd = 0; rc.cnt[0].mind = 0;
         *a.heavy_cnt = 0u;
+        *a.unfinished = 0u;
     }
     grid_sync(bar, epoch);
     Tiers tiers{a.heavy, a.hblk, 0u};
@@ -182,6 +190,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksCc) cc_kernel(CcArgs a) {
             if (t - 1 < kMaxHist) rc.rec[t - 1].edges = (long long)cv.edges;
         }
         if (cv.va == 0) break;
+        if (a.max_iters > 0 && t >= a.max_iters) {          // high diameter: hand over to hooking
+            if (is_book()) *a.unfinished = 1u;
+            break;
+        }
         f.Va = (long long)cv.va; f.Ea = (long long)cv.ea;
         f.Via = (long long)n - f.Va; f.Eia = (long long)a.g.nnz - f.Ea;
         f.maxd = cv.maxd; f.mind = cv.mind; f.iter = t;
@@ -275,6 +287,16 @@ gsw_status run_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     a.heavy = (unsigned *)ws.take(nh * 4);
     a.hblk = (unsigned *)ws.take((nh + 1) * 4);
     a.heavy_cnt = (unsigned *)ws.take(256);
+    a.unfinished = a.heavy_cnt + 32;
+    // Algorithm switch of the autotuned run (CC): label propagation needs about as
+    // many iterations as the graph's diameter (C2: 4,013, 244 ms); when it is still running after
+    // GSW_CC_SWITCH (default 12) iterations, its labels seed the hooking + pointer-jumping CC
+    // (cc_hook.cu), which converges in a few sweeps.  Forced variants never switch.
+    const gsw_config &fc = g->forced;
+    const bool all_auto = fc.direction == GSW_AUTO && fc.format == GSW_AUTO && fc.load_balance == GSW_AUTO &&
+                          fc.fusion == GSW_AUTO;
+    const char *sw = std::getenv("GSW_CC_SWITCH");
+    a.max_iters = all_auto ? (sw ? std::atoi(sw) : kCcSwitchIters) : 0;
     LaunchInfo li;
     gsw_status s = prepare_common(g, ws, (const void *)cc_kernel, a.rc, li, kMinBlocksCc);
     if (s != GSW_OK) return s;
@@ -284,7 +306,27 @@ gsw_status run_cc(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
     if (s != GSW_OK) return s;
     if (!dev_out)
         GSW_CUDA(cudaMemcpyAsync(label_out, relabeled ? a.out : a.label, (size_t)n * 4, cudaMemcpyDeviceToHost, g->stream));
-    return finish_run(g, a.rc, li, st);
+    if ((s = finish_run(g, a.rc, li, st)) != GSW_OK) return s;
+    if (a.max_iters <= 0) return GSW_OK;
+    unsigned unfinished = 0;
+    GSW_CUDA(cudaMemcpy(&unfinished, a.unfinished, 4, cudaMemcpyDeviceToHost));
+    if (!unfinished) return GSW_OK;
+    // hand over: the hooking run continues from a.label and appends its records
+    gsw_run_stats h{};
+    if (st) {
+        const int used = std::min(st->iterations, st->max_records);
+        h.records = st->records ? st->records + used : nullptr;
+        h.max_records = st->records ? std::max(0, st->max_records - used) : 0;
+    }
+    if ((s = run_cc_hook_seeded(g, label_out, st ? &h : nullptr, a.label, ws.used)) != GSW_OK) return s;
+    if (st) {
+        for (int i = 0; i < std::min(h.iterations, h.max_records); ++i) h.records[i].iteration += st->iterations;
+        st->iterations += h.iterations;
+        st->gpu_ms += h.gpu_ms;
+        st->edges_touched += h.edges_touched;
+        st->bytes_alg += h.bytes_alg;
+    }
+    return GSW_OK;
 }
 
 }  // namespace gsw

@@ -39,6 +39,8 @@ struct CcHookArgs {
     unsigned long long *P;    // packed parent pointers (internal order)
     int *out;                 // labels, caller order
     uint32_t *scan;           // STRICT degree scan
+    const int *seed;          // optional start labels (internal order, caller-id values, each a
+                              // vertex of v's component with key <= v's): gsw_cc's switch (cc.cu)
     RunCommon rc;
 };
 
@@ -99,7 +101,23 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksCcHook) cc_hook_kernel(const
     const Adj adj{a.g.off, a.g.col};
     unsigned long long *P = a.P;
 
-    for (long long v = gtid(); v < n; v += gthreads()) P[v] = hk_pack(a.g.perm, (unsigned)v);
+    if (a.seed) {
+        // start from a labeling: v points at the vertex whose caller id is its label (the forest
+        // stays acyclic: keys never increase along a pointer), then compress, so that every
+        // pointer names a root when the first hook sweep starts (what termination relies on)
+        for (long long v = gtid(); v < n; v += gthreads()) {
+            const unsigned c = (unsigned)a.seed[v];
+            P[v] = ((unsigned long long)c << 32) | (a.g.inv ? __ldg(a.g.inv + c) : c);
+        }
+        grid_sync(bar, epoch);
+        for (long long v = gtid(); v < n; v += gthreads()) {
+            unsigned long long p = P[v], q = P[(unsigned)p];
+            while (q != p) { p = q; q = P[(unsigned)p]; }
+            P[v] = p;
+        }
+    } else {
+        for (long long v = gtid(); v < n; v += gthreads()) P[v] = hk_pack(a.g.perm, (unsigned)v);
+    }
     if (is_book()) for (int i = 0; i < 3; ++i) reset_cnt(rc.cnt + i);
     grid_sync(bar, epoch);
 
@@ -160,6 +178,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocksCcHook) cc_hook_kernel(const
 }
 
 gsw_status run_cc_hook(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
+    return run_cc_hook_seeded(g, label_out, st, nullptr, 0);
+}
+
+gsw_status run_cc_hook_seeded(gsw_graph g, int32_t *label_out, gsw_run_stats *st, const int *seed, size_t ws_used) {
     const int n = g->g.n;
     if (!label_out) { set_error("gsw_cc_hook: label is NULL"); return GSW_EINVAL; }
     const int lbf = g->forced.load_balance;
@@ -167,11 +189,12 @@ gsw_status run_cc_hook(gsw_graph g, int32_t *label_out, gsw_run_stats *st) {
         set_error("gsw_cc_hook: unknown forced load balance");
         return GSW_EUNSUPPORTED;
     }
-    Workspace ws{g->scratch, g->scratch_bytes, 0};
+    Workspace ws{g->scratch, g->scratch_bytes, ws_used};     // ws_used: keep the seed's region
     const bool dev_out = is_device_ptr(label_out) == 1;
     CcHookArgs a{};
     a.g = g->g;
     a.sym = g->symmetric;
+    a.seed = seed;
     a.P = (unsigned long long *)ws.take((size_t)n * 8);
     a.out = dev_out ? label_out : (int *)ws.take((size_t)n * 4);
     a.scan = (uint32_t *)ws.take((size_t)(n + 1) * 4);

@@ -172,7 +172,8 @@ size_t scratch_bytes_for(int64_t n, int64_t nnz, int has_w) {
     size_t per_v = 64;                         // BC: depth 4 + sigma 8 + delta 8 + stack 4 + bc 8 + queues
     size_t b = per_v * (size_t)(n + 64) + 16 * W * 4;
     b += (size_t)(n + 1) * 8;                  // i64 offset staging at ingest / scan arrays
-    b += 8u << 20;                             // control blocks, per-CTA partials, history, records
+    b += 16u << 20;                            // control blocks, per-CTA partials, history, records (x2: gsw_cc's
+                                               // label-propagation run and the hooking run it hands over to)
     // gsw_dpr: two heavy-row chunk tables (<= nnz/128 + 1 entries of 12 B, dpr.cu k_dpr_chunks)
     // and kDprMaxIters per-iteration records (queue length 4 B + counters 32 B)
     b += 2 * ((size_t)nnz / 128 + 1) * 12 + 1024 + (size_t)kDprMaxIters * 36;

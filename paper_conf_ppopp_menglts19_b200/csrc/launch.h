@@ -43,6 +43,7 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth, gsw_run_stats *s
 gsw_status run_sssp(gsw_graph g, int32_t source, uint32_t *dist, gsw_run_stats *st);
 gsw_status run_cc(gsw_graph g, int32_t *label, gsw_run_stats *st);
 gsw_status run_cc_hook(gsw_graph g, int32_t *label, gsw_run_stats *st);
+gsw_status run_cc_hook_seeded(gsw_graph g, int32_t *label, gsw_run_stats *st, const int *seed, size_t ws_used);
 gsw_status run_pr(gsw_graph g, double damping, int32_t iters, double *rank, gsw_run_stats *st);
 gsw_status run_dpr(gsw_graph g, double damping, double tol, int32_t max_iters, double *rank, gsw_run_stats *st);
 gsw_status run_bc(gsw_graph g, const int32_t *sources, int32_t nsrc, double *bc, gsw_run_stats *st);
