@@ -34,6 +34,7 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -176,6 +177,7 @@ struct DistState {
     const void *bfs_exec_depth = nullptr;
     int bfs_exec_dir = -1;
     cudaStream_t cap = nullptr;             // private stream the graph is captured on (the caller's may be the legacy stream)
+    bool graph_failed = false;              // capture / instantiation failed once: host-driven loop
 };
 
 int64_t dist_slice(int64_t n, int32_t p) {
@@ -1359,8 +1361,13 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
     GSW_CUDA(cudaGetLastError());
     // graph mode: the level loop as one CUDA graph whose WHILE node the decide kernel drives, so
     // the host neither polls nor enqueues per level (NCCL / loopback; GSW_DIST_GRAPH=0 disables)
+    // Default: loopback and single-rank NCCL.  With several NCCL ranks the graph holds NCCL's
+    // collectives inside a conditional body, which only this one-GPU build could not exercise, so
+    // it is opt-in there (GSW_DIST_GRAPH=1); a capture or instantiation failure falls back to the
+    // host-driven loop either way.
     const char *gm = std::getenv("GSW_DIST_GRAPH");
-    const bool graph_mode = d->mode != DM_HOST && !(gm && *gm == '0');
+    bool graph_mode = d->mode != DM_HOST && !d->graph_failed &&
+                      (gm ? *gm != '0' : (d->mode == DM_LOOPBACK || d->nranks == 1));
     if (graph_mode) {
         if (!d->bfs_exec || d->bfs_exec_depth != (const void *)depth || d->bfs_exec_dir != fdir) {
             if (d->bfs_exec) { cudaGraphExecDestroy(d->bfs_exec); d->bfs_exec = nullptr; }
@@ -1399,22 +1406,24 @@ gsw_status dist_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_sta
             cudaGraph_t cap = nullptr;
             const cudaError_t ce = cudaStreamEndCapture(s, &cap);
             s = run;
-            if (cs != GSW_OK || ce != cudaSuccess) {
-                cudaGraphDestroy(gr);
-                if (cs == GSW_OK) { set_error(std::string("dist bfs graph capture: ") + cudaGetErrorString(ce)); cs = GSW_ECUDA; }
-                return cs;
-            }
-            const cudaError_t ie = cudaGraphInstantiate(&d->bfs_exec, gr, 0);
+            cudaError_t ie = cudaErrorUnknown;
+            if (cs == GSW_OK && ce == cudaSuccess) ie = cudaGraphInstantiate(&d->bfs_exec, gr, 0);
             cudaGraphDestroy(gr);
             if (ie != cudaSuccess) {
+                // fall back to the host-driven loop for this handle (nothing of the capture ran)
+                cudaGetLastError();
                 d->bfs_exec = nullptr;
-                set_error(std::string("dist bfs graph instantiate: ") + cudaGetErrorString(ie));
-                return GSW_ECUDA;
+                d->graph_failed = true;
+                graph_mode = false;
+                if (std::getenv("GSW_VERBOSE"))
+                    std::fprintf(stderr, "gsw: dist BFS graph capture failed (%s), host-driven loop\n",
+                                 cudaGetErrorString(ce != cudaSuccess ? ce : ie));
+            } else {
+                d->bfs_exec_depth = depth;
+                d->bfs_exec_dir = fdir;
             }
-            d->bfs_exec_depth = depth;
-            d->bfs_exec_dir = fdir;
         }
-        GSW_CUDA(cudaGraphLaunch(d->bfs_exec, s));
+        if (graph_mode) GSW_CUDA(cudaGraphLaunch(d->bfs_exec, s));
     }
     int t = 0;
     for (; !graph_mode; ++t) {
