@@ -39,6 +39,7 @@
 #include <string>
 #include <vector>
 
+#include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 #include <nccl.h>
 
@@ -134,6 +135,7 @@ struct DPart {
     int32_t *rfirst = nullptr;// first in-neighbour of each owned row (-1: empty)
     uint32_t *soff = nullptr; // n_global+1: global source u -> owned targets
     int32_t *scol = nullptr;  // local target ids
+    uint32_t *rcol_h = nullptr;   // owned in-edge columns renamed to hub order (PR gathers; nullptr: off)
     unsigned *vis = nullptr;  // visited words of the owned slice (S/32); SSSP: improved in the last push
     unsigned *far = nullptr;  // SSSP far set of the owned slice (S/32)
     const uint32_t *rw = nullptr;   // weights of the owned rows (weighted graphs)
@@ -178,6 +180,12 @@ struct DistState {
     int bfs_exec_dir = -1;
     cudaStream_t cap = nullptr;             // private stream the graph is captured on (the caller's may be the legacy stream)
     bool graph_failed = false;              // capture / instantiation failed once: host-driven loop
+    // hub order for PR: vertices ranked by global degree (descending); the
+    // replicated contributions are re-laid out in that order every iteration so the gathers of
+    // the hubs share cache lines, as after the single-GPU engine's relabeling
+    uint32_t *horder = nullptr;             // npad: vertex of rank i
+    uint32_t *hrank = nullptr;              // npad: rank of vertex v
+    float *crank = nullptr;                 // npad: contributions in hub order
 };
 
 int64_t dist_slice(int64_t n, int32_t p) {
@@ -233,6 +241,19 @@ __global__ void k_hub_first(const uint32_t *roff, int32_t *rcol, uint32_t *rw, i
             if (rw) { const uint32_t w = rw[b]; rw[b] = rw[at]; rw[at] = w; }
         }
     }
+}
+__global__ void k_iota(uint32_t *x, int64_t n) {
+    for (long long i = gtid(); i < n; i += gthreads()) x[i] = (uint32_t)i;
+}
+__global__ void k_invert(const uint32_t *order, int64_t n, uint32_t *rank) {
+    for (long long i = gtid(); i < n; i += gthreads()) rank[order[i]] = (uint32_t)i;
+}
+__global__ void k_rename(const int32_t *col, uint32_t m, const uint32_t *rank, uint32_t *out) {
+    for (long long e = gtid(); e < m; e += gthreads()) out[e] = rank[__ldg(col + e)];
+}
+// contributions re-laid out in hub order: coalesced writes, gathers from the all-gathered array
+__global__ void k_hub_layout(const float *c, const uint32_t *order, int64_t n, float *cr) {
+    for (long long i = gtid(); i < n; i += gthreads()) cr[i] = c[__ldg(order + i)];
 }
 // column slice "global source -> owned targets": count, scan, fill
 __global__ void k_slice_count(const uint32_t *roff, const int32_t *rcol, int nloc, uint32_t *cnt) {
@@ -981,6 +1002,7 @@ static size_t dist_bytes(int64_t n, int64_t nnz_total, int32_t nranks, int32_t n
     b += al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // scol (all parts)
     b += al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // rcol copy
     if (weighted) b += 2 * al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // row + slice weights
+    b += 3 * al((size_t)npad * 4) + al((size_t)std::max<int64_t>(nnz_total, 1) * 4);   // PR hub order: order, rank, contributions, renamed columns
     if (mode == DM_LOOPBACK) b += al((size_t)(n + 1) * 4);  // full u32 offsets
     size_t cub = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, cub, (uint32_t *)nullptr, (uint32_t *)nullptr, (int)(n + 1));
@@ -1244,6 +1266,41 @@ gsw_status dist_create(const gsw_csr *rows, int64_t n, const void *nccl_id, cons
             k_first<<<grid_for(P.nloc, g->sms), kDB, 0, s>>>(P.roff, P.rcol, P.nloc, P.rfirst);
         }
         if (cudaGetLastError() != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "hub first"));
+    }
+    // PR hub order: rank every vertex by its global degree (the degrees are in rep[0] after the hub
+    // step; they are gathered here otherwise), rename the owned columns once
+    const char *ho = std::getenv("GSW_DIST_PR_HUBORDER");
+    if (!(ho && *ho == '0')) {
+        d->horder = (uint32_t *)ws.take((size_t)d->npad * 4);
+        d->hrank = (uint32_t *)ws.take((size_t)d->npad * 4);
+        d->crank = (float *)ws.take((size_t)d->npad * 4);
+        if (!d->horder || !d->hrank || !d->crank) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
+        const char *hf = std::getenv("GSW_DIST_HUBFIRST");
+        if (hf && *hf == '0') {                        // degrees not gathered by the hub-first step
+            for (auto &P : d->parts)
+                k_degrees<<<grid_for(S, g->sms), kDB, 0, s>>>(P.roff, P.nloc, S, d->rep[0] + P.vb);
+            if (gsw_status st = ex_allgather(d, d->rep[0], (size_t)S * 4, s)) return fail(st);
+        }
+        // descending radix sort of (degree, vertex) with double buffers: rep[0]/rep[1] for the keys,
+        // the BC scratch (bdepth) and horder for the values, bsigma as the sort's temp storage
+        k_iota<<<grid_for(d->npad, g->sms), kDB, 0, s>>>(reinterpret_cast<uint32_t *>(d->bdepth), d->npad);
+        cub::DoubleBuffer<uint32_t> keys(d->rep[0], d->rep[1]);
+        cub::DoubleBuffer<uint32_t> vals(reinterpret_cast<uint32_t *>(d->bdepth), d->horder);
+        size_t tb = 0;
+        cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, keys, vals, (int)d->npad, 0, 32, s);
+        if (tb > (size_t)d->npad * 8) { set_error("dist workspace too small (hub-order sort)"); return fail(GSW_ENOMEM); }
+        if (cub::DeviceRadixSort::SortPairsDescending(d->bsigma, tb, keys, vals, (int)d->npad, 0, 32, s) != cudaSuccess)
+            return fail(cuda_fail(cudaGetLastError(), "hub-order sort"));
+        if (vals.Current() != d->horder &&
+            cudaMemcpyAsync(d->horder, vals.Current(), (size_t)d->npad * 4, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+            return fail(cuda_fail(cudaGetLastError(), "hub order"));
+        k_invert<<<grid_for(d->npad, g->sms), kDB, 0, s>>>(d->horder, d->npad, d->hrank);
+        for (auto &P : d->parts) {
+            P.rcol_h = (uint32_t *)ws.take((size_t)std::max<uint32_t>(P.nnz, 1) * 4);
+            if (!P.rcol_h) { set_error("dist workspace too small"); return fail(GSW_ENOMEM); }
+            if (P.nnz) k_rename<<<grid_for(P.nnz, g->sms), kDB, 0, s>>>(P.rcol, P.nnz, d->hrank, P.rcol_h);
+        }
+        if (cudaGetLastError() != cudaSuccess) return fail(cuda_fail(cudaGetLastError(), "hub order"));
     }
     g->scratch = (char *)ws.take((size_t)d->npad * 8);      // output staging (host outputs)
     g->scratch_bytes = (size_t)d->npad * 8;
@@ -1683,16 +1740,22 @@ gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out,
     GSW_CUDA(cudaEventRecord(g->ev0, s));
     GSW_CUDA(cudaMemsetAsync(d->locs, 0, (size_t)kLocStride * 8 * parts, s));
     GSW_CUDA(cudaMemsetAsync(C[0], 0, (size_t)d->npad * 4, s));
+    const bool hub = d->crank != nullptr;          // gathers in hub order (create time)
     auto args = [&](int p, const float *cur, float *next, bool last) {
         const DPart &P = d->parts[p];
-        return PrP{P.roff, P.rcol, P.vb, P.nloc, cur, next, last ? out + (d->mode == DM_LOOPBACK ? P.vb : 0) : nullptr,
+        return PrP{P.roff, hub ? reinterpret_cast<const int32_t *>(P.rcol_h) : P.rcol, P.vb, P.nloc,
+                   hub ? d->crank : cur, next, last ? out + (d->mode == DM_LOOPBACK ? P.vb : 0) : nullptr,
                    P.chunks, P.nchunks, P.psum, P.loc, d->ctl, damping, invN};
+    };
+    auto relayout = [&](const float *c) {
+        if (hub) k_hub_layout<<<grid_for(d->npad, g->sms), kDB, 0, s>>>(c, d->horder, d->npad, d->crank);
     };
     for (int p = 0; p < parts; ++p)
         k_pr_init<<<grid_for(std::max(d->parts[p].nloc, 1), g->sms), kDB, 0, s>>>(args(p, nullptr, C[0], iters == 0));
     GSW_CUDA(cudaGetLastError());
     if (gsw_status e = ex_allgather(d, C[0], (size_t)d->S * 4, s)) return e;
     if (gsw_status e = ex_reduce(d, s)) return e;
+    relayout(C[0]);
     const int grid = g->sms * 8;
     unsigned long long nnz_loc = 0;
     for (auto &P : d->parts) nnz_loc += P.nnz;
@@ -1707,6 +1770,7 @@ gsw_status dist_pr(gsw_graph g, double damping, int32_t iters, double *rank_out,
         GSW_CUDA(cudaGetLastError());
         if (gsw_status e = ex_allgather(d, C[(t + 1) & 1], (size_t)d->S * 4, s)) return e;
         if (gsw_status e = ex_reduce(d, s)) return e;
+        if (t + 1 < iters) relayout(C[(t + 1) & 1]);
     }
     GSW_CUDA(cudaEventRecord(g->ev1, s));
     if (!dev_out) GSW_CUDA(cudaMemcpyAsync(rank_out, out, (size_t)out_len * 8, cudaMemcpyDeviceToHost, s));
