@@ -39,6 +39,10 @@ struct BcArgs {
     RunCommon rc;
 };
 
+#ifndef GSW_BC_COND
+#define GSW_BC_COND 1   // gather sigma / omega only for the edges whose depth matches (A/B knob)
+#endif
+
 struct BcProbe { int dv; unsigned su_lo, su_hi; };
 
 // forward push
@@ -96,6 +100,14 @@ struct BcPullOp {
         const int d = depth[v];
         return d >= 0 && d <= lvl;
     }
+#if GSW_BC_COND
+    // depth[u] first; sigma[u] (8 B) only for the parents on level lvl -- most scanned in-edges
+    // of the wide pull levels are not parents, and the two gathers per edge were the level's cost
+    __device__ __forceinline__ Probe probe(int, uint32_t, int u) const { return BcProbe{depth[u], 0u, 0u}; }
+    __device__ __forceinline__ Acc val(int, uint32_t, int u, Probe p) const {
+        return p.dv == lvl ? sigma[u] : 0ull;
+    }
+#else
     __device__ __forceinline__ Probe probe(int, uint32_t, int u) const {
         unsigned long long su = sigma[u];
         return BcProbe{depth[u], (unsigned)su, (unsigned)(su >> 32)};
@@ -103,6 +115,7 @@ struct BcPullOp {
     __device__ __forceinline__ Acc val(int, uint32_t, int, Probe p) const {
         return p.dv == lvl ? (((unsigned long long)p.su_hi << 32) | p.su_lo) : 0ull;
     }
+#endif
     __device__ __forceinline__ void flush(int v, Acc s, bool exclusive, LocalCnt &c) const {
         if (s == 0ull) return;
         bool won;
@@ -126,18 +139,27 @@ struct BcBackOp {
     int lvl;
     bool owner;
     bool by_level;        // items are all vertices; only those on level lvl take part
+#if GSW_BC_COND
+    using Probe = int;    // depth[w]; omega[w] is gathered in val() only for the successors
+#else
     using Probe = double;
+#endif
     using Acc = double;
     static constexpr bool kFlushEmpty = true;
     static __device__ __forceinline__ Acc identity() { return 0.0; }
     static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a + b; }
     __device__ __forceinline__ bool skip(int v) const { return by_level && depth[v] != lvl; }
+#if GSW_BC_COND
+    __device__ __forceinline__ Probe probe(int, uint32_t, int w) const { return depth[w]; }
+    __device__ __forceinline__ Acc val(int, uint32_t, int w, Probe p) const { return p == lvl + 1 ? omega[w] : 0.0; }
+#else
     __device__ __forceinline__ Probe probe(int, uint32_t, int w) const {
         const int dw = depth[w];
         const double ow = omega[w];                // issued together with depth[w]
         return dw == lvl + 1 ? ow : 0.0;
     }
     __device__ __forceinline__ Acc val(int, uint32_t, int, Probe p) const { return p; }
+#endif
     __device__ __forceinline__ void finish(int v, double a) const {
         double sv = (double)sigma[v];
         double dv = sv * a;
