@@ -33,6 +33,18 @@ def corpus(gen, size="full"):
     """~110 synthetic graphs (none of them C1-C5: other seeds and sizes).  size="small" keeps the
     round-1 list of 24."""
     out = []
+    if size == "large":
+        # round-2 addition: graphs as large as the evaluation configs (the 106-graph corpus stops at
+        # scale 20 / 3M vertices, and its trees lost on C3/C4); other seeds and skews than C1-C5
+        for scale, ef, abc, seed in [(21, 16, (.57, .19, .19), 301), (22, 16, (.57, .19, .19), 302),
+                                     (22, 8, (.60, .15, .15), 303), (21, 32, (.50, .20, .20), 304),
+                                     (23, 16, (.57, .19, .19), 305), (22, 24, (.65, .15, .15), 306)]:
+            out.append(gen.rmat(scale, ef, *abc, seed=seed))
+        for k, (n, pairs, gamma) in enumerate([(4_000_000, 60_000_000, 2.3), (5_000_000, 70_000_000, 2.2),
+                                               (3_500_000, 50_000_000, 2.5), (6_000_000, 90_000_000, 2.4)]):
+            out.append(gen.chung_lu(n, pairs, gamma=gamma, i0=150.0, seed=310 + k))
+        out.append(gen.grid(1800, 1800))
+        return out
     if size == "small":
         for scale, ef, abc, seed in [(14, 8, (.57, .19, .19), 11), (14, 32, (.57, .19, .19), 12),
                                      (15, 16, (.45, .25, .15), 13), (15, 16, (.70, .10, .10), 14),
@@ -84,7 +96,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--json", required=True)
     ap.add_argument("--roots", type=int, default=2)
-    ap.add_argument("--size", default="full", choices=["full", "small"])
+    ap.add_argument("--size", default="full", choices=["full", "small", "large"])
     a = ap.parse_args()
     import torch
     import gen
