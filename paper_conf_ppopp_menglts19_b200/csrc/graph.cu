@@ -1,5 +1,6 @@
 // graph.cu -- step a0 of the hot path: ingest + dataset attributes (Table 1; "computed
 // only once while loading the data into the memory").  Not inside any timed run.
+#include <cstdlib>
 #include <cmath>
 #include <cstring>
 #include <vector>
@@ -132,6 +133,39 @@ __global__ void k_permute_rows_keys(const uint32_t *noff, const uint32_t *off, c
         for (uint32_t k = b + lane_id(); k < e; k += 32) {
             keys[nb + (k - b)] = hi | inv[col[k]];
             if (w) nw[nb + (k - b)] = w[k];
+        }
+    }
+}
+// symmetric unweighted fast path (relabel_csr): (new column, new row) pairs in new-row order;
+// rows of kRelabelHeavy+ edges are skipped here and written by k_permute_heavy (a warp walking a
+// 163K-edge hub row serially was most of this pass)
+constexpr uint32_t kRelabelHeavy = 8192;
+__global__ void k_permute_rows_pairs(const uint32_t *noff, const uint32_t *off, const int32_t *col, const uint32_t *perm,
+                                     const uint32_t *inv, int n, uint32_t *keys, uint32_t *vals, uint32_t *heavy,
+                                     unsigned *nheavy) {
+    for (long long i = gwarp(); i < n; i += gwarps()) {
+        const uint32_t o = perm[i];
+        const uint32_t b = off[o], e = off[o + 1], nb = noff[i];
+        if (e - b >= kRelabelHeavy) {
+            if (lane_id() == 0) heavy[atomicAdd(nheavy, 1u)] = (uint32_t)i;
+            continue;
+        }
+        for (uint32_t k = b + lane_id(); k < e; k += 32) {
+            keys[nb + (k - b)] = inv[col[k]];
+            vals[nb + (k - b)] = (uint32_t)i;
+        }
+    }
+}
+__global__ void k_permute_heavy(const uint32_t *noff, const uint32_t *off, const int32_t *col, const uint32_t *perm,
+                                const uint32_t *inv, uint32_t *keys, uint32_t *vals, const uint32_t *heavy,
+                                const unsigned *nheavy) {
+    const unsigned nh = *nheavy;
+    for (unsigned h = blockIdx.x; h < nh; h += gridDim.x) {
+        const uint32_t i = heavy[h], o = perm[i];
+        const uint32_t b = off[o], e = off[o + 1], nb = noff[i];
+        for (uint32_t k = b + threadIdx.x; k < e; k += blockDim.x) {
+            keys[nb + (k - b)] = inv[col[k]];
+            vals[nb + (k - b)] = i;
         }
     }
 }
@@ -293,7 +327,10 @@ size_t relabel_temp_bytes(int64_t n, int64_t nnz, int has_w) {
     cub::DoubleBuffer<uint32_t> vb(nullptr, nullptr);
     if (has_w) cub::DeviceRadixSort::SortPairs(nullptr, t3, kb, vb, (int)nnz, 0, key_end_bit(n));
     else cub::DeviceRadixSort::SortKeys(nullptr, t3, kb, (int)nnz, 0, key_end_bit(n));
-    size_t t = std::max(t1, std::max(t2, t3));
+    size_t t4 = 0;
+    cub::DoubleBuffer<uint32_t> kb32(nullptr, nullptr), vb32(nullptr, nullptr);
+    cub::DeviceRadixSort::SortPairs(nullptr, t4, kb32, vb32, (int)nnz, 0, key_end_bit(n) - 32);
+    size_t t = std::max(std::max(t1, t4), std::max(t2, t3));
     const size_t m = (size_t)std::max<int64_t>(nnz, 1);
     return al256(t) + 3 * al256((size_t)n * 4) + al256((size_t)(n + 1) * 4) + 2 * al256(m * 8) +
            (has_w ? 2 * al256(m * 4) : 0) + 4096;
@@ -312,6 +349,28 @@ static gsw_status relabel_csr(gsw_graph g, uint32_t *off, int32_t *col, uint32_t
     size_t cb = cub_bytes;
     GSW_CUDA(cub::DeviceScan::InclusiveSum(cub_tmp, cb, degp, noff + 1, n, s));
     k_set_u32<<<1, 1, 0, s>>>(noff, 0u);
+    if (g->symmetric && !w && nnz > 0 && !std::getenv("GSW_RELABEL_KEYS64")) {
+        // Symmetric graph: new row x holds {y : x in N(y)}.  Emitting (x, y) pairs in ascending y
+        // (new rows in order) and sorting them STABLY by x alone yields every row's columns in
+        // ascending order -- a radix sort over log2(n) key bits with 32-bit keys and values
+        // instead of the (row << 32 | column) 64-bit keys below (C3: half the passes).
+        uint32_t *ka = reinterpret_cast<uint32_t *>(k0), *kb2 = ka + nnz;
+        uint32_t *va = reinterpret_cast<uint32_t *>(k1), *vb2 = va + nnz;
+        uint32_t *heavy = degp;                      // degp is consumed by the scan above
+        unsigned *nheavy = reinterpret_cast<unsigned *>(w0 ? w0 : (uint32_t *)cub_tmp);
+        (void)w1;
+        GSW_CUDA(cudaMemsetAsync(nheavy, 0, 4, s));
+        k_permute_rows_pairs<<<grid_for((long long)n * 32, g->sms), kBlock, 0, s>>>(noff, off, col, perm, inv, n, ka, va,
+                                                                                   heavy, nheavy);
+        k_permute_heavy<<<g->sms * 2, kBlock, 0, s>>>(noff, off, col, perm, inv, ka, va, heavy, nheavy);
+        GSW_CUDA(cudaGetLastError());
+        GSW_CUDA(cudaMemcpyAsync(off, noff, (size_t)(n + 1) * 4, cudaMemcpyDeviceToDevice, s));
+        cub::DoubleBuffer<uint32_t> kd(ka, kb2), vd(va, vb2);
+        cb = cub_bytes;
+        GSW_CUDA(cub::DeviceRadixSort::SortPairs(cub_tmp, cb, kd, vd, (int)nnz, 0, key_end_bit(n) - 32, s));
+        GSW_CUDA(cudaMemcpyAsync(col, vd.Current(), (size_t)nnz * 4, cudaMemcpyDeviceToDevice, s));
+        return GSW_OK;
+    }
     k_permute_rows_keys<<<grid_for((long long)n * 32, g->sms), kBlock, 0, s>>>(noff, off, col, w, perm, inv, n, k0, w0);
     GSW_CUDA(cudaGetLastError());
     GSW_CUDA(cudaMemcpyAsync(off, noff, (size_t)(n + 1) * 4, cudaMemcpyDeviceToDevice, s));
