@@ -223,3 +223,44 @@ def test_nccl_single_rank_bc(gsw):
     srcs = gen.sources(g, 2)
     x, _ = D.bc(srcs)
     _bc_close(x.cpu().numpy(), oracle.bc(g, srcs))
+
+
+KNOBS = {
+    "graph_loop": {"GSW_DIST_GRAPH": "1"},
+    "host_loop": {"GSW_DIST_GRAPH": "0"},
+    "no_hub_first": {"GSW_DIST_HUBFIRST": "0"},
+    "no_pr_hub_order": {"GSW_DIST_PR_HUBORDER": "0"},
+    "plain": {"GSW_DIST_GRAPH": "0", "GSW_DIST_HUBFIRST": "0", "GSW_DIST_PR_HUBORDER": "0"},
+}
+
+
+@pytest.mark.parametrize("knob", sorted(KNOBS))
+@pytest.mark.parametrize("nparts", [1, 3])
+def test_loopback_execution_choices(gsw, monkeypatch, knob, nparts):
+    """The partitioned path's execution choices (CUDA-graph level loop, hub-first
+    rows, PR hub order) change nothing in the results: BFS depths and per-level features, CC labels,
+    SSSP distances (weights follow the reordered columns), PR within 1e-5, BC within 1e-4."""
+    for k, v in KNOBS[knob].items():
+        monkeypatch.setenv(k, v)
+    g = gen.rmat(13, seed=12)
+    P = gsw.PartitionedGraph(g.off, g.col, nparts)
+    for s in gen.sources(g, 2, seed=7):
+        d, st = P.bfs(s, records=128)
+        assert np.array_equal(d.cpu().numpy(), oracle.bfs(g, s)), (knob, nparts, s)
+        Va, Ea, _, _ = oracle.bfs_features(g, s)
+        assert [r["Va"] for r in st["records"]] == Va.tolist()
+        d2, _ = P.bfs(s)                   # second call: the cached graph (graph mode) is re-launched
+        assert np.array_equal(d2.cpu().numpy(), d.cpu().numpy())
+    lab, _ = P.cc()
+    assert np.array_equal(lab.cpu().numpy(), oracle.cc(g))
+    x, _ = P.pr(0.85, 20)
+    r = oracle.pr(g, 0.85, 20)
+    assert (np.abs(x.cpu().numpy() - r) / r).max() <= 1e-5
+    srcs = gen.sources(g, 3, seed=3)
+    b, _ = P.bc(srcs)
+    ref = oracle.bc(g, srcs)
+    assert (np.abs(b.cpu().numpy() - ref) / np.maximum(np.abs(ref), 1.0)).max() <= 1e-4
+    gw = gen.with_hash_weights(gen.grid(33, 21), 12345, 64)
+    W = gsw.PartitionedGraph(gw.off, gw.col, nparts, weights=gw.w)
+    dd, _ = W.sssp(0)
+    assert np.array_equal(dd.cpu().numpy().view(np.uint32), oracle.sssp(gw, 0)), (knob, nparts)
