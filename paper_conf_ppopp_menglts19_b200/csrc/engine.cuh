@@ -4,6 +4,7 @@
 //   unsorted queue: compact ids in any order, warp-aggregated atomics
 //   sorted queue  : compact ids ascending via a scan of bitmap words
 #pragma once
+#include <cstddef>
 #include "common.cuh"
 #include "gsw.h"
 #include "select.cuh"
@@ -111,15 +112,17 @@ __device__ __forceinline__ void hist_features(const CntView &v, Features &f) {
 __device__ __forceinline__ void write_record(const RunCommon &rc, int t, const DevCfg &c, const Features &f,
                                              unsigned theta) {
     if (blockIdx.x == 0 && threadIdx.x == 0 && t < kMaxHist) {
-        gsw_iter_record r;
-        r.iteration = t;
-        r.direction = c.dir; r.format = c.fmt; r.load_balance = c.lb; r.stepping = c.step; r.fusion = c.fused;
-        r.Va = f.Va; r.Ea = f.Ea; r.Via = f.Via; r.Eia = f.Eia;
-        r.edges = 0;
-        r.theta = theta;
-        r.filter_us = 0.f; r.expand_us = 0.f;
-        r.ctas = (int32_t)gridDim.x;
-        rc.rec[t] = r;
+        // five 16-byte stores straight from registers (a gsw_iter_record temporary went through
+        // the stack: local-memory round trips on the critical path of every level)
+        static_assert(sizeof(gsw_iter_record) == 80 && offsetof(gsw_iter_record, Va) == 24 &&
+                      offsetof(gsw_iter_record, theta) == 64, "record layout");
+        int4 *p = reinterpret_cast<int4 *>(rc.rec + t);
+        p[0] = make_int4(t, c.dir, c.fmt, c.lb);
+        p[1] = make_int4(c.step, c.fused, (int)(unsigned long long)f.Va, (int)((unsigned long long)f.Va >> 32));
+        p[2] = make_int4((int)(unsigned long long)f.Ea, (int)((unsigned long long)f.Ea >> 32),
+                         (int)(unsigned long long)f.Via, (int)((unsigned long long)f.Via >> 32));
+        p[3] = make_int4((int)(unsigned long long)f.Eia, (int)((unsigned long long)f.Eia >> 32), 0, 0);
+        p[4] = make_int4((int)theta, 0, 0, (int)gridDim.x);
     }
 }
 
