@@ -68,6 +68,9 @@ __device__ __forceinline__ void cluster_barrier() {
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 constexpr uint64_t kBarrierTimeoutNs = 20ull * 1000 * 1000 * 1000;
+#ifndef GSW_BAR_SC
+#define GSW_BAR_SC 0
+#endif
 
 // Flip-bit barrier (the cooperative-groups scheme): CTA 0 adds 2^31 - (gridDim - 1), every other
 // CTA adds 1, so the counter's top bit flips exactly when the last CTA arrives; waiters poll the
@@ -79,6 +82,15 @@ __device__ __forceinline__ unsigned ld_volatile_u32(const unsigned *p) {
     asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+// Release before the arrival, acquire after the flip is seen: fence.acq_rel.gpu on both sides
+// (GSW_BAR_SC=1: __threadfence, i.e. the sequentially consistent MEMBAR.SC.GPU, A/B knob).
+__device__ __forceinline__ void bar_fence() {
+#if GSW_BAR_SC
+    __threadfence();
+#else
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#endif
+}
 __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch) {
 #ifndef GSW_NO_CLUSTER_BAR
     if (b.cluster) { cluster_barrier(); epoch += 1; return; }
@@ -86,7 +98,7 @@ __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch)
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;
-        __threadfence();
+        bar_fence();
         const unsigned old = atomicAdd(b.arrive, add);
         uint64_t t0 = 0;
         unsigned spins = 0;
@@ -97,7 +109,7 @@ __device__ __forceinline__ void grid_sync(const GridBarrier &b, unsigned &epoch)
                 else if (now - t0 > kBarrierTimeoutNs) { atomicExch(b.err, 0xBA4u); __trap(); }
             }
         }
-        __threadfence();
+        bar_fence();
     }
     epoch += 1;
     __syncthreads();
@@ -113,7 +125,7 @@ __device__ __forceinline__ void grid_park(const GridBarrier &b, unsigned &epoch)
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned add = blockIdx.x == 0 ? 0x80000000u - (gridDim.x - 1u) : 1u;
-        __threadfence();
+        bar_fence();
         const unsigned old = atomicAdd(b.arrive, add);
         const uint64_t t0 = globaltimer();
         unsigned spins = 0;
@@ -124,7 +136,7 @@ __device__ __forceinline__ void grid_park(const GridBarrier &b, unsigned &epoch)
                 __trap();
             }
         }
-        __threadfence();
+        bar_fence();
     }
     epoch += 1;
     __syncthreads();
