@@ -80,3 +80,21 @@ def test_c3_full_size(gsw):
     g = gen.config_graph("C3")
     lab, st = _hook(gsw.Graph(g.off, g.col), records=64)
     assert np.array_equal(lab, oracle.cc(g))
+
+
+def test_directed_input_weak_components(gsw):
+    """A directed CSR (with its CSC): every adjacency entry hooks both trees, so the labels are the
+    weakly connected components, as the union-find oracle computes them over the same entries."""
+    rng = np.random.default_rng(8)
+    n = 700
+    edges = [(int(u), int(v)) for u, v in rng.integers(0, n, size=(500, 2)) if u != v]
+    g = gen.from_edges(n, edges, symmetric=False)
+    csc = gen.from_edges(n, [(v, u) for u, v in edges], symmetric=False)
+    G = gsw.Graph(g.off, g.col, csc=(csc.off, csc.col))
+    for lb in ("auto", "thread", "strict"):
+        if lb == "auto":
+            G.force_config()
+        else:
+            G.force_config(load_balance=lb)
+        lab, _ = _hook(G)
+        assert np.array_equal(lab, oracle.cc(g)), lb
