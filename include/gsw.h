@@ -143,7 +143,14 @@ gsw_status gsw_graph_attributes(gsw_graph g, double out[7]);
  * entries), GSW_PR_BLOCKED / GSW_PR_BLOCKS (row-tier / source-blocked PageRank), GSW_MINB_BFS_FIXED /
  * GSW_MINB_SSSP_FIXED (disable the per-graph residency choice), GSW_DIST_LOOKAHEAD (levels the
  * partitioned host loop runs ahead of its done-flag poll), GSW_PHASES=1 (BFS init / loop / output
- * device times on stderr).
+ * device times on stderr), GSW_CC_SWITCH=k (autotuned gsw_cc: label-propagation iterations before
+ * it hands over to hooking, default 12, 0 = never), GSW_TEAM=k (BFS: clustered launch whose first
+ * k-CTA cluster runs the small levels, road-like graphs, default off), GSW_CLUSTER=k (run a
+ * persistent kernel as ONE k-CTA cluster, barrier.cluster as its grid barrier), GSW_GRID_CTAS=k
+ * (persistent grid of k CTAs), GSW_DIST_GRAPH=0|1 (partitioned BFS level loop as a CUDA graph;
+ * default on for loopback / one NCCL rank), GSW_DIST_HUBFIRST=0 / GSW_DIST_PR_HUBORDER=0
+ * (partitioned create-time row reordering / PageRank hub-order layout off), GSW_RELABEL_KEYS64=1
+ * (graph create: the 64-bit key sort instead of the symmetric pair sort).
  */
 gsw_status gsw_force_config(gsw_graph g, const gsw_config *cfg);
 
