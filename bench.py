@@ -35,6 +35,23 @@ FALLBACK_HBM = 6650.0   # GB/s, B200_PROFILING.md fallback
 PR_GATHER_PEAK = 356.0
 
 
+def workload_label(workload, g):
+    """The `config.workload` string both arms print for the same graph (the driver compares them)."""
+    scale = {"C3": 22, "C5": 26}.get(workload, 22)
+    return (f"{workload}: BFS on R-MAT scale {scale} ef 16 (Graph500 a,b,c=.57,.19,.19), n={g.n}, nnz={g.nnz}, "
+            "roots per SURVEY Q12")
+
+
+def csr_hash(g):
+    """Content hash of the generated CSR (recorded in every result line), so lines
+    from different runs can be checked to have timed the same graph."""
+    import hashlib
+    h = hashlib.sha256()
+    h.update(np.ascontiguousarray(g.off).view(np.uint8))
+    h.update(np.ascontiguousarray(g.col).view(np.uint8))
+    return "sha256:" + h.hexdigest()[:16]
+
+
 def hbm_peak():
     try:
         with open(PEAKS_FILE) as f:
@@ -150,13 +167,12 @@ def run_reference(args, ws, rank):
         secs += time.perf_counter() - t0
         edges += m_cc(deg, d)
     v = edges / secs / 1e9
-    scale = {"C3": 22, "C5": 26}.get(workload, 22)
     line = {"impl": "reference", "metric": "BFS GTEPS", "value": v, "unit": "GTEPS", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs * 1e3 / nsteps,
             "higher_is_better": True, "scaling": "strong" if c5 else "weak", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic",
-            "config": {"workload": f"{workload}: BFS on R-MAT scale {scale} ef 16 (Graph500 a,b,c=.57,.19,.19), "
-                                   "roots per SURVEY Q12", "parallelism": "single host thread"},
+            "config": {"workload": workload_label(workload, g), "csr_hash": csr_hash(g)},
+            "parallelism": "single host thread",
             "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                              "sample": f"{nsteps} BFS roots, full {workload} graph, oracle.bfs (FIFO queue, 1 thread)"},
             "e2e": {"value": v, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -641,12 +657,11 @@ def run_gsw(args, ws, rank, local):
             "metric": "BFS GTEPS", "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": f"{args.workload}: BFS on R-MAT scale {22 if args.workload == 'C3' else 26} ef 16 "
-                                   "(Graph500 a,b,c=.57,.19,.19), "
-                                   f"n={g.n}, nnz={g.nnz}, roots per SURVEY Q12, autotuned",
-                       "l2": "flushed between steps (256 MiB write outside the timed span)",
-                       "parallelism": (f"root-sharded replicas x{ws} (one graph copy per GPU, no collective)"
-                                       if replicas else "single GPU")},
+            "config": {"workload": workload_label(args.workload, g), "csr_hash": csr_hash(g)},
+            "selector": "autotuned (hand-set rules, DESIGN.md R13)",
+            "l2": "flushed between steps (256 MiB write outside the timed span)",
+            "parallelism": (f"root-sharded replicas x{ws} (one graph copy per GPU, no collective)"
+                            if replicas else "single GPU"),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": sane_frac(achieved / peak, "BFS"), "traffic": traffic, "peak_source": peak_src,
                          "kernel": "gsw::bfs_kernel (persistent, 1 launch/step)",
