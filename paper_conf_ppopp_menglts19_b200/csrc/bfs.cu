@@ -1086,7 +1086,9 @@ gsw_status run_bfs(gsw_graph g, int32_t source, int32_t *depth_out, gsw_run_stat
     a.depth = (dev_out && !relabeled) ? depth_out : (int *)ws.take((size_t)n * 4);
     a.out = relabeled ? (dev_out ? depth_out : (int *)ws.take((size_t)n * 4)) : nullptr;
     // scatter measured faster on C3 (0.1556 vs 0.1594 ms per root, profiles/r2/bfs_output_scatter_ab.txt)
-    a.scatter = std::getenv("GSW_BFS_SCATTER") ? std::atoi(std::getenv("GSW_BFS_SCATTER")) : 1;
+    // but only while the caller-order array stays in L2: at C5 (268 MB) the scattered 4-byte stores
+    // become DRAM read-modify-writes (single-GPU BFS 653 -> 466 GTEPS), so it is used up to 8M vertices
+    a.scatter = std::getenv("GSW_BFS_SCATTER") ? std::atoi(std::getenv("GSW_BFS_SCATTER")) : (n <= (1 << 23) ? 1 : 0);
     a.V = (unsigned *)ws.take((size_t)W * 4);
     for (int i = 0; i < 3; ++i) a.fb[i] = (unsigned *)ws.take((size_t)W * 4);
     for (int i = 0; i < 2; ++i) a.q[i] = (int *)ws.take((size_t)n * 4);
