@@ -35,10 +35,12 @@ FALLBACK_HBM = 6650.0   # GB/s, B200_PROFILING.md fallback
 PR_GATHER_PEAK = 356.0
 
 
-def workload_label(workload, g):
+def workload_label(workload, g=None, n=None, nnz=None):
     """The `config.workload` string both arms print for the same graph (the driver compares them)."""
     scale = {"C3": 22, "C5": 26}.get(workload, 22)
-    return (f"{workload}: BFS on R-MAT scale {scale} ef 16 (Graph500 a,b,c=.57,.19,.19), n={g.n}, nnz={g.nnz}, "
+    n = g.n if g is not None else n
+    nnz = g.nnz if g is not None else nnz
+    return (f"{workload}: BFS on R-MAT scale {scale} ef 16 (Graph500 a,b,c=.57,.19,.19), n={n}, nnz={nnz}, "
             "roots per SURVEY Q12")
 
 
@@ -171,7 +173,8 @@ def run_reference(args, ws, rank):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs * 1e3 / nsteps,
             "higher_is_better": True, "scaling": "strong" if c5 else "weak", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic",
-            "config": {"workload": workload_label(workload, g), "csr_hash": csr_hash(g)},
+            "config": ({"workload": workload_label(workload, g)} if c5
+                       else {"workload": workload_label(workload, g), "csr_hash": csr_hash(g)}),
             "parallelism": "single host thread",
             "cpu_baseline": {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                              "sample": f"{nsteps} BFS roots, full {workload} graph, oracle.bfs (FIFO queue, 1 thread)"},
@@ -497,19 +500,19 @@ def run_gsw_dist(args, ws, rank, local):
         torch.cuda.empty_cache()
     h2d_all = sm(off.nbytes + col.nbytes)           # collectives on every rank, before the rank-0 print
     d2h_all = sm(4 * max(1, len(host_out)))
+    nnz_g = sm(len(col))
     if rank == 0:
         launches_per_level = 4                      # push, push_heavy, pull, decide (+ NCCL kernels)
         line = {
             "metric": "BFS GTEPS", "value": value, "unit": "GTEPS", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": f"{workload}: BFS on R-MAT/Kronecker scale {26 if workload == 'C5' else 22} ef 16 "
-                                   f"(Graph500 a,b,c=.57,.19,.19), n={n}, 1D vertex partition over {ws} ranks "
-                                   f"(slice {gsw.dist_slice(n, ws)}), per-level NCCL bitmap all-gather, roots per "
-                                   "SURVEY Q12",
-                       "l2": "flushed between steps (256 MiB write outside the timed span)",
-                       "parallelism": f"1D vertex partition x{ws} " + ("(host-staged exchange over gloo, all ranks on GPU 0: "
-                                                                "a logic test, not a measurement)" if host_ex else "(NCCL over NVLink)")},
+            "config": {"workload": workload_label(workload, n=n, nnz=int(nnz_g))},
+            "partition": f"1D vertex partition over {ws} ranks (slice {gsw.dist_slice(n, ws)}), per-level NCCL "
+                         "bitmap all-gather",
+            "l2": "flushed between steps (256 MiB write outside the timed span)",
+            "parallelism": f"1D vertex partition x{ws} " + ("(host-staged exchange over gloo, all ranks on GPU 0: "
+                                                     "a logic test, not a measurement)" if host_ex else "(NCCL over NVLink)"),
             "roofline": {"bound": "hbm", "achieved": per_gpu_gbs, "peak": peak, "unit": "GB/s",
                          "frac": sane_frac(per_gpu_gbs / peak, "dist BFS"), "traffic": None,
                          "peak_source": peak_src,
